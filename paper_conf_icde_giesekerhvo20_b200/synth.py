@@ -1,0 +1,173 @@
+"""Seeded synthetic image stacks shaped like the paper's workloads.
+
+This module is the ONLY code shared by the CUDA path's tests/bench and the
+oracle's tests: it draws inputs and holds none of BFAST-Monitor's
+arithmetic (no design matrix, no fit, no MOSUM).  It uses plain torch ops on
+whatever device the caller names (PyTorch is plumbing here), so a stack of
+26.8 GB can be generated directly in HBM.
+
+Recipe (parameters mimic the Landsat NDMI stacks
+of L47/L377 and the Table I structure of L303-L319):
+  dates   d_t = year0 + t/f, t = 1..N (f = 23: 16-day Landsat, L53).
+  signal  y = a + b (d_t - d_1) + sum_{j=1..3} (u_j sin 2 pi j d_t + w_j cos 2 pi j d_t)
+          + eps,  a ~ U[0.3,0.8], b ~ U[-0.01,0.01], u_j, w_j ~ U[-0.1,0.1],
+          eps ~ N(0, s^2), s ~ U[0.01,0.05] per pixel.
+  breaks  a fraction of pixels gets a step -delta, delta ~ U[0.1,0.5], from
+          t0 ~ U{n, ..., N-1} (0-based) on.
+  missing "iid": Bernoulli(miss) per (t, p)  (Table I's f_NaN, L309);
+          "cloud": per date a cover c_t ~ U[max(0,2m-1), min(1,2m)] and the
+          pixels below the c_t-quantile of a smooth value-noise field
+          (64-pixel lattice, bilinear) are NaN (cloud masks, L95).
+The stack is time-major Y[t][p] with leading dimension ldY >= P (the
+paper's Y^T, L185); columns P..ldY-1 are NaN padding.
+"""
+from __future__ import annotations
+
+import math
+from dataclasses import dataclass, asdict
+
+import numpy as np
+import torch
+
+
+@dataclass
+class StackSpec:
+    P: int
+    N: int
+    n_hist: int
+    k: int = 3
+    hf: float = 0.25
+    lam: float = 1.65
+    miss: float = 0.5
+    mask: str = "iid"          # "iid" | "cloud" | "none"
+    break_frac: float = 0.1
+    f: float = 23.0
+    year0: float = 2000.0
+    seed: int = 1
+    noise_lo: float = 0.01
+    noise_hi: float = 0.05
+
+    def asdict(self):
+        return asdict(self)
+
+
+# The configs of BASELINE.json (configs[0..4]); n_hist = N/2 where BASELINE is
+# silent (as in D1-D5, L319), k = 3, hf = 0.25, lambda = 1.65.
+CONFIGS = {
+    "tiny": StackSpec(P=4096, N=228, n_hist=114, miss=0.5, mask="iid", break_frac=0.3, seed=1),
+    "landsat": StackSpec(P=4096 * 4096, N=400, n_hist=200, miss=0.6, mask="cloud",
+                         break_frac=0.1, seed=2),
+    "sentinel2": StackSpec(P=10980 * 10980, N=700, n_hist=350, miss=0.5, mask="iid",
+                           f=73.0, year0=2016.0, break_frac=0.1, seed=4),
+}
+
+
+def sweep_spec(N: int, miss: float, k: int, P: int = 4096 * 4096, index: int = 0) -> StackSpec:
+    """configs[2]: N in {100,250,500,1000} x miss in {.1,.5,.9} x k in {1,3,5}."""
+    return StackSpec(P=P, N=N, n_hist=N // 2, k=k, miss=miss, mask="iid",
+                     break_frac=0.1, seed=100 + index)
+
+
+def make_dates(N: int, f: float = 23.0, year0: float = 2000.0) -> np.ndarray:
+    t = np.arange(1, N + 1, dtype=np.float64)
+    return year0 + t / f
+
+
+def _gen(device, seed: int, stream: int) -> torch.Generator:
+    g = torch.Generator(device=device)
+    g.manual_seed((int(seed) * 1_000_003 + int(stream) * 7919 + 12345) % (2**63 - 1))
+    return g
+
+
+def _grid_shape(P: int):
+    W = int(math.isqrt(P))
+    if W * W < P:
+        W += 1
+    H = (P + W - 1) // W
+    return H, W
+
+
+def _cloud_field(H: int, W: int, g: torch.Generator, device) -> torch.Tensor:
+    """Smooth value noise: U[0,1) lattice every 64 px, bilinear in between."""
+    gh, gw = H // 64 + 2, W // 64 + 2
+    lat = torch.rand(1, 1, gh, gw, generator=g, device=device)
+    up = torch.nn.functional.interpolate(lat, size=((gh - 1) * 64 + 1, (gw - 1) * 64 + 1),
+                                         mode="bilinear", align_corners=True)
+    return up[0, 0, :H, :W].reshape(-1)
+
+
+def generate(spec: StackSpec, device="cpu", ldY: int | None = None, out: torch.Tensor | None = None,
+             return_truth: bool = False, chunk_elems: int = 1 << 28):
+    """Return (Y [N][ldY] float32 on `device`, dates float64 numpy[, truth])."""
+    P, N = int(spec.P), int(spec.N)
+    ldY = P if ldY is None else int(ldY)
+    if ldY < P:
+        raise ValueError("ldY < P")
+    dev = torch.device(device)
+    if out is None:
+        Y = torch.empty((N, ldY), dtype=torch.float32, device=dev)
+    else:
+        Y = out
+        assert Y.shape == (N, ldY) and Y.dtype == torch.float32
+    dates = make_dates(N, spec.f, spec.year0)
+
+    g = _gen(dev, spec.seed, 0)
+    u = lambda lo, hi, *shape: torch.rand(*shape, generator=g, device=dev) * (hi - lo) + lo
+    a = u(0.3, 0.8, P)
+    b = u(-0.01, 0.01, P)
+    amp_s = u(-0.1, 0.1, 3, P)
+    amp_c = u(-0.1, 0.1, 3, P)
+    s = u(spec.noise_lo, spec.noise_hi, P)
+    has_break = torch.rand(P, generator=g, device=dev) < spec.break_frac
+    delta = u(0.1, 0.5, P) * has_break
+    t0 = torch.randint(spec.n_hist, N, (P,), generator=g, device=dev)
+    cover = None
+    if spec.mask == "cloud":
+        m = float(spec.miss)
+        lo, hi = max(0.0, 2 * m - 1), min(1.0, 2 * m)
+        cover = (torch.rand(N, generator=g, device=dev) * (hi - lo) + lo).cpu().numpy()
+    H, W = _grid_shape(P)
+
+    Tc = max(1, min(N, chunk_elems // max(P, 1)))
+    dd = torch.tensor(dates - dates[0], dtype=torch.float32, device=dev)
+    two_pi = 2.0 * math.pi
+    sin_t = torch.tensor(np.stack([np.sin(two_pi * j * dates) for j in (1, 2, 3)]),
+                         dtype=torch.float32, device=dev)
+    cos_t = torch.tensor(np.stack([np.cos(two_pi * j * dates) for j in (1, 2, 3)]),
+                         dtype=torch.float32, device=dev)
+    tidx = torch.arange(N, device=dev)
+    for c0 in range(0, N, Tc):
+        c1 = min(N, c0 + Tc)
+        gc = _gen(dev, spec.seed, 1 + c0)
+        blk = a[None, :] + b[None, :] * dd[c0:c1, None]
+        for j in range(3):
+            blk += amp_s[j][None, :] * sin_t[j, c0:c1, None]
+            blk += amp_c[j][None, :] * cos_t[j, c0:c1, None]
+        blk += torch.randn(c1 - c0, P, generator=gc, device=dev) * s[None, :]
+        blk -= delta[None, :] * (tidx[c0:c1, None] >= t0[None, :])
+        if spec.mask == "iid":
+            miss = torch.rand(c1 - c0, P, generator=gc, device=dev) < spec.miss
+            blk.masked_fill_(miss, float("nan"))
+        elif spec.mask == "cloud":
+            for t in range(c0, c1):
+                field = _cloud_field(H, W, gc, dev)[:P]
+                sub = field[:: max(1, P // (1 << 20))]
+                thr = torch.quantile(sub, float(cover[t]))
+                blk[t - c0].masked_fill_(field < thr, float("nan"))
+        elif spec.mask != "none":
+            raise ValueError(spec.mask)
+        Y[c0:c1, :P] = blk
+        del blk
+    if ldY > P:
+        Y[:, P:] = float("nan")
+    if return_truth:
+        truth = {"has_break": has_break, "delta": delta, "t0": t0, "noise_sd": s}
+        return Y, dates, truth
+    return Y, dates
+
+
+def sample_columns(Y: torch.Tensor, P: int, count: int, seed: int = 0) -> np.ndarray:
+    """Uniformly sampled pixel indices (sorted), for sampled parity/baselines."""
+    rng = np.random.default_rng(seed)
+    count = min(count, P)
+    return np.sort(rng.choice(P, size=count, replace=False)).astype(np.int64)
