@@ -1,0 +1,362 @@
+#!/usr/bin/env python
+"""bench.py -- BFAST-Monitor throughput on B200 (BASELINE.json metric).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                  [--config landsat|tiny|sweep:N:miss:k] [--no-e2e] [--no-cpu-baseline]
+
+One "step" = one pass of the whole hot path (the fused monitor kernel plus
+the fp64 refit kernel) over one synthetic scene resident in HBM.  At N=1 the
+workload is BASELINE configs[1] (Landsat-like: 4096x4096 pixels, N=400
+dates, n_hist=200, k=3, h=0.25, lambda=1.65, 60% cloud-masked).  Under
+torchrun each rank processes its own Landsat-shaped scene (weak scaling:
+pixels are independent, L142; no collective on the data path) and the
+device-timed max over ranks is reported.  Timing: CUDA events on the launch
+stream, W warm-up steps, barrier + synchronize on both sides; the 26.8 GB
+stack per GPU is far larger than the 126 MB L2, so no explicit flush.
+
+--impl reference times the fp64 CPU oracle (oracle/, the paper's
+definitions, OpenMP over the host cores) on a bounded sample of the same
+workload: the base contract's reference arm for this paper-only tier.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "BFAST-Monitor pixels/sec at 1/2/4/8 B200; achieved HBM GB/s vs peak"
+UNIT = "pixels/s"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="landsat")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=10.0, help="target oracle wall time")
+    return ap.parse_args()
+
+
+def spec_for(name: str):
+    from paper_conf_icde_giesekerhvo20_b200 import synth
+    if name.startswith("sweep:"):
+        _, N, miss, k = name.split(":")
+        return synth.sweep_spec(int(N), float(miss), int(k)), f"sweep N={N} miss={miss} k={k}"
+    spec = synth.CONFIGS[name]
+    desc = {
+        "landsat": "Landsat-like scene (BASELINE configs[1]): 4096x4096 px x N=400 dates "
+                   "(n_hist=200), k=3, h=0.25, lambda=1.65, 60% missing (cloud masks)",
+        "tiny": "tiny (BASELINE configs[0]): 4096 px x N=228 (n_hist=114), k=3, h=0.25, "
+                "lambda=1.65, 50% NaN i.i.d.",
+        "sentinel2": "Sentinel-2-like tile: 10980x10980 px x N=700",
+    }[name]
+    return spec, desc
+
+
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons sampled during the timed region."""
+
+    Q = ("timestamp,index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device_index: int):
+        self.dev = device_index
+        self.proc = None
+        self.lines = []
+        self.t0 = self.t1 = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits", "-lms", "20",
+                 "-i", str(self.dev)], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thr = threading.Thread(target=self._read, daemon=True)
+            self.thr.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append((time.time(), line.strip()))
+
+    def mark(self, begin: bool):
+        if begin:
+            self.t0 = time.time()
+        else:
+            self.t1 = time.time()
+
+    def stop(self):
+        if self.proc:
+            time.sleep(0.05)
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        rows = [l for (ts, l) in self.lines if self.t0 is not None and self.t0 - 0.02 <= ts <= self.t1 + 0.05]
+        if not rows:
+            rows = [l for (_, l) in self.lines][-3:]
+        sm, smax, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            f = [x.strip() for x in r.split(",")]
+            if len(f) < 10:
+                continue
+            try:
+                sm.append(float(f[2]))
+                smax = float(f[3])
+            except ValueError:
+                continue
+            for n, v in zip(names, f[6:10]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        sm.sort()
+        return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": smax, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+
+
+def ncu_traffic(workload_key: str):
+    """dram read+write bytes per launch of the fused kernel from the committed
+    ncu --set full summary (profiles/), or None."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        d = json.load(open(p))
+        e = d.get(workload_key)
+        return None if e is None else float(e["dram_bytes_per_launch"])
+    except Exception:
+        return None
+
+
+def oracle_sample(Y, dates, spec, count, seed=0):
+    """Run the oracle on `count` sampled pixel columns of the device stack Y;
+    returns (oracle outputs, seconds, threads, idx)."""
+    import numpy as np
+    import torch
+    import oracle
+    from paper_conf_icde_giesekerhvo20_b200 import synth
+    idx = synth.sample_columns(Y, spec.P, count, seed=seed)
+    it = torch.tensor(idx, device=Y.device)
+    Ys = np.ascontiguousarray(Y.index_select(1, it).cpu().numpy())
+    t0 = time.perf_counter()
+    out = oracle.monitor(Ys, dates, spec.n_hist, spec.k, spec.hf, spec.lam)
+    dt = time.perf_counter() - t0
+    return out, dt, oracle.max_threads(), idx
+
+
+def run_reference(args):
+    """The reference arm: the fp64 oracle on the host cores."""
+    import numpy as np
+    world, rank, local = dist_env()
+    if rank != 0:
+        return 0
+    import oracle
+    spec, desc = spec_for(args.config)
+    import torch
+    from paper_conf_icde_giesekerhvo20_b200 import synth
+    oracle.build()
+    # bounded sample of the workload: a sub-scene of the same recipe on CPU
+    sub = synth.StackSpec(**{**spec.asdict(), "P": min(spec.P, 1 << 14)})
+    Y, dates = synth.generate(sub, "cpu")
+    Yn = Y.numpy()
+    threads = oracle.max_threads()
+    times = []
+    for i in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        oracle.monitor(Yn, dates, sub.n_hist, sub.k, sub.hf, sub.lam)
+        dt = time.perf_counter() - t0
+        if i >= args.warmup:
+            times.append(dt)
+    ms = 1000 * sum(times) / len(times)
+    value = sub.P / (ms / 1000)
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": desc, "sample": f"{sub.P} pixels per step (same recipe, CPU sub-scene)"},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
+                             "sample": f"{sub.P} pixels of the workload per step"},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    from paper_conf_icde_giesekerhvo20_b200 import _build, binding, synth
+
+    world, rank, local = dist_env()
+    if world != args.gpus and world > 1:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    if not os.path.exists(binding.LIB_PATH):
+        _build.build()
+
+    spec, desc = spec_for(args.config)
+    # each rank: its own scene of the configured shape (weak scaling); seed per rank
+    rspec = synth.StackSpec(**{**spec.asdict(), "seed": spec.seed + 1000 * rank})
+    Y, dates = synth.generate(rspec, dev)
+    P, N = rspec.P, rspec.N
+    plan = binding.Plan(local, N, dates, rspec.n_hist, rspec.k, rspec.hf, rspec.lam)
+    stream = torch.cuda.Stream(device=dev)
+    out = {"break": torch.empty(P, dtype=torch.int32, device=dev),
+           "magnitude": torch.empty(P, dtype=torch.float32, device=dev)}
+    torch.cuda.synchronize()
+
+    def step():
+        plan.execute(Y, stream=stream, out=out)
+
+    with torch.cuda.stream(stream):
+        for _ in range(args.warmup):
+            step()
+    torch.cuda.synchronize()
+
+    sampler = ClockSampler(local)
+    sampler.start()
+    time.sleep(0.6)  # let nvidia-smi start sampling
+    with torch.cuda.stream(stream):   # keep the GPU busy while the sampler starts
+        for _ in range(2):
+            step()
+    binding.profile_enable(True)
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    sampler.mark(True)
+    ev0.record(stream)
+    launches = 0
+    for _ in range(args.steps):
+        step()
+        launches += binding.last_launch_count()
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    sampler.mark(False)
+    if world > 1:
+        dist.barrier()
+    kernel_ms = binding.profile_collect()
+    binding.profile_enable(False)
+    sampler.stop()
+    ms_total = ev0.elapsed_time(ev1)
+    t = torch.tensor([ms_total], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_step = float(t.item()) / args.steps
+    total_pixels = P * world
+    value = total_pixels / (ms_step / 1000.0)
+
+    # roofline of the dominant (fused) kernel: algorithmic bytes per launch
+    alg_bytes = P * (4 * N + 8)
+    kms = sorted(kernel_ms)
+    k_avg = sum(kms) / len(kms) if kms else float("nan")
+    peak, peak_src = load_peaks()
+    achieved = alg_bytes / (k_avg / 1000.0) / 1e9
+    workload_key = f"{args.config}:P={P}:N={N}:k={rspec.k}"
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                "frac": achieved / peak, "traffic": ncu_traffic(workload_key),
+                "kernel": "monitor_simt_kernel<8>", "kernel_ms_avg": k_avg,
+                "kernel_share_of_step": k_avg / ms_step if ms_step else None,
+                "alg_bytes_per_launch": alg_bytes, "peak_source": peak_src}
+
+    clocks = sampler.summary()
+    line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": desc, "pixels_per_gpu": P, "N": N, "n_hist": rspec.n_hist, "k": rspec.k,
+                       "h": rspec.hf, "lambda": rspec.lam, "missing": rspec.miss, "mask": rspec.mask,
+                       "l2": "inputs larger than L2 (stack %.1f GB/GPU vs 126 MB L2), no flush" % (4 * N * P / 1e9),
+                       "parallelism": f"dp{world}: pixel shards, no collective"},
+            "roofline": roofline, "gpu_launches": launches, "clocks": clocks}
+
+    # cpu baseline + sampled parity (rank 0, N = 1 only)
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        from oracle import parity
+        probe = 1 << 13
+        _, dt, threads, _ = oracle_sample(Y, dates, rspec, probe, seed=7)
+        count = int(min(1 << 21, max(probe, probe * args.cpu_seconds / max(dt, 1e-3))))
+        orc, dt, threads, idx = oracle_sample(Y, dates, rspec, count, seed=11)
+        it = torch.tensor(idx, device=dev)
+        gpu = {"break": out["break"].index_select(0, it).cpu().numpy(),
+               "magnitude": out["magnitude"].index_select(0, it).cpu().numpy()}
+        rep = parity.compare(gpu, orc)
+        line["cpu_baseline"] = {"value": count / dt, "unit": UNIT, "cores": threads, "kind": "oracle",
+                                "sample": f"{count} uniformly sampled pixel columns of the same scene, "
+                                          f"{dt:.1f} s"}
+        line["parity_sample"] = {k: rep[k] for k in ("pixels", "ok", "break_mismatch",
+                                                     "break_mismatch_unexcused", "invalid_mismatch",
+                                                     "mag_fail", "mag_max_scaled_err")}
+
+    # end to end through the public host-buffer API: H2D + kernels + D2H
+    if not args.no_e2e:
+        Yh = torch.empty((N, P), dtype=torch.float32, pin_memory=True)
+        Yh.copy_(Y)
+        del Y
+        torch.cuda.empty_cache()
+        ob = np.empty(P, np.int32)
+        om = np.empty(P, np.float32)
+        binding.bfast_monitor_host(Yh, dates, rspec.n_hist, rspec.k, rspec.hf, rspec.lam, ob, om, device=local)
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for _ in range(args.e2e_steps):
+            binding.bfast_monitor_host(Yh, dates, rspec.n_hist, rspec.k, rspec.hf, rspec.lam, ob, om,
+                                       device=local)
+        e2e_s = (time.perf_counter() - t0) / args.e2e_steps
+        te = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        e2e_s = float(te.item())
+        line["e2e"] = {"value": total_pixels / e2e_s, "unit": UNIT, "h2d_bytes_per_step": 4 * N * P,
+                       "d2h_bytes_per_step": 8 * P, "steps": args.e2e_steps,
+                       "path": "bfast_monitor_host: pinned host stack, slab-pipelined H2D overlapped "
+                               "with the kernels, D2H of results; host wall clock"}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

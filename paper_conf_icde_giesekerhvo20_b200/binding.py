@@ -1,0 +1,278 @@
+"""ctypes binding of libbfast.so (include/bfast.h) -- argument marshalling only.
+
+Every step of BFAST-Monitor runs in the library's CUDA kernels; this module
+turns torch tensors / numpy arrays into pointers and statuses into
+exceptions.  There is no CPU fallback: if libbfast.so is missing or the
+device path fails, the call raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from typing import Optional
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libbfast.so")
+_lib = None
+
+BFAST_OK, BFAST_EINVAL, BFAST_EUNSUPPORTED, BFAST_ECUDA, BFAST_ENOMEM = 0, -1, -2, -3, -4
+NO_BREAK, INVALID_PIXEL = -1, -2
+FLAG_DEGENERATE, FLAG_REFIT_FP64 = 0x01, 0x02
+K_MAX_HARMONICS = 6
+
+# names declared in include/bfast.h (checked by tests/test_abi.py)
+EXPORTS = ("bfast_monitor", "bfast_monitor_ex", "bfast_plan_create", "bfast_plan_execute",
+           "bfast_plan_destroy", "bfast_monitor_host", "bfast_monitor_multi",
+           "bfast_shard_range", "bfast_last_launch_count", "bfast_last_error",
+           "bfast_status_string", "bfast_abi_version", "bfast_profile_enable",
+           "bfast_profile_collect")
+
+
+class BfastError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{msg} (status {status})")
+        self.status = status
+
+
+class _Args(ctypes.Structure):
+    _fields_ = [("Y", ctypes.c_void_p), ("N", ctypes.c_int64), ("P", ctypes.c_int64),
+                ("ldY", ctypes.c_int64), ("dates", ctypes.c_void_p), ("n_hist", ctypes.c_int32),
+                ("k", ctypes.c_int32), ("h", ctypes.c_float), ("lambda_", ctypes.c_float),
+                ("out_break", ctypes.c_void_p), ("out_magnitude", ctypes.c_void_p),
+                ("out_beta", ctypes.c_void_p), ("out_sigma", ctypes.c_void_p),
+                ("out_nbar", ctypes.c_void_p), ("out_flags", ctypes.c_void_p),
+                ("stream", ctypes.c_void_p)]
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} is missing: run __graft_entry__.build() "
+                              "(there is no CPU fallback)")
+        L = ctypes.CDLL(LIB_PATH)
+        V, i64, i32, f32, I = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_float, ctypes.c_int
+        L.bfast_monitor.argtypes = [V, i64, i64, V, i32, i32, f32, f32, V, V]
+        L.bfast_monitor.restype = I
+        L.bfast_monitor_ex.argtypes = [ctypes.POINTER(_Args)]
+        L.bfast_monitor_ex.restype = I
+        L.bfast_plan_create.argtypes = [ctypes.POINTER(V), I, i64, V, i32, i32, f32, f32]
+        L.bfast_plan_create.restype = I
+        L.bfast_plan_execute.argtypes = [V, ctypes.POINTER(_Args)]
+        L.bfast_plan_execute.restype = I
+        L.bfast_plan_destroy.argtypes = [V]
+        L.bfast_plan_destroy.restype = None
+        L.bfast_monitor_host.argtypes = [V, i64, i64, i64, V, i32, i32, f32, f32, V, V, I]
+        L.bfast_monitor_host.restype = I
+        L.bfast_monitor_multi.argtypes = [V, i64, i64, i64, V, i32, i32, f32, f32, V, I, V, V]
+        L.bfast_monitor_multi.restype = I
+        L.bfast_shard_range.argtypes = [i64, I, I, ctypes.POINTER(i64), ctypes.POINTER(i64)]
+        L.bfast_shard_range.restype = None
+        L.bfast_last_launch_count.restype = I
+        L.bfast_last_error.restype = ctypes.c_char_p
+        L.bfast_status_string.argtypes = [I]
+        L.bfast_status_string.restype = ctypes.c_char_p
+        L.bfast_abi_version.restype = I
+        L.bfast_profile_enable.argtypes = [I]
+        L.bfast_profile_enable.restype = I
+        L.bfast_profile_collect.argtypes = [V, I]
+        L.bfast_profile_collect.restype = I
+        _lib = L
+    return _lib
+
+
+def _check(rc: int):
+    if rc != BFAST_OK:
+        L = lib()
+        raise BfastError(rc, f"{L.bfast_status_string(rc).decode()}: {L.bfast_last_error().decode()}")
+
+
+def _dates(dates) -> np.ndarray:
+    return np.ascontiguousarray(np.asarray(dates, dtype=np.float64))
+
+
+def _dptr(t) -> Optional[int]:
+    if t is None:
+        return None
+    return int(t.data_ptr())
+
+
+def _stream_ptr(stream):
+    if stream is None:
+        import torch
+        return int(torch.cuda.current_stream().cuda_stream)
+    return int(getattr(stream, "cuda_stream", stream))
+
+
+def abi_version() -> int:
+    return int(lib().bfast_abi_version())
+
+
+def last_launch_count() -> int:
+    return int(lib().bfast_last_launch_count())
+
+
+def last_error() -> str:
+    return lib().bfast_last_error().decode()
+
+
+def profile_enable(on: bool = True):
+    _check(lib().bfast_profile_enable(1 if on else 0))
+
+
+def profile_collect(max_events: int = 100000):
+    """Milliseconds of each fused-kernel launch recorded since enabling."""
+    buf = (ctypes.c_float * max_events)()
+    n = lib().bfast_profile_collect(ctypes.cast(buf, ctypes.c_void_p), max_events)
+    if n < 0:
+        _check(n)
+    return [float(buf[i]) for i in range(n)]
+
+
+def shard_range(P: int, rank: int, world: int):
+    b, e = ctypes.c_int64(), ctypes.c_int64()
+    lib().bfast_shard_range(int(P), int(rank), int(world), ctypes.byref(b), ctypes.byref(e))
+    return int(b.value), int(e.value)
+
+
+def _make_args(Y, dates_np, n_hist, k, h, lam, out_break, out_magnitude, P=None, ldY=None,
+               out_beta=None, out_sigma=None, out_nbar=None, out_flags=None, stream=None) -> _Args:
+    N = int(Y.shape[0])
+    ldY = int(Y.stride(0)) if ldY is None else int(ldY)
+    P = int(Y.shape[1]) if P is None else int(P)
+    a = _Args()
+    a.Y = _dptr(Y)
+    a.N, a.P, a.ldY = N, P, ldY
+    a.dates = dates_np.ctypes.data
+    a.n_hist, a.k, a.h, a.lambda_ = int(n_hist), int(k), float(h), float(lam)
+    a.out_break, a.out_magnitude = _dptr(out_break), _dptr(out_magnitude)
+    a.out_beta, a.out_sigma = _dptr(out_beta), _dptr(out_sigma)
+    a.out_nbar, a.out_flags = _dptr(out_nbar), _dptr(out_flags)
+    a.stream = _stream_ptr(stream)
+    return a
+
+
+def _outputs(Y, P, k, want_diag):
+    import torch
+    dev = Y.device
+    out = {"break": torch.empty(P, dtype=torch.int32, device=dev),
+           "magnitude": torch.empty(P, dtype=torch.float32, device=dev)}
+    if want_diag:
+        out["beta"] = torch.empty((P, 2 + 2 * k), dtype=torch.float32, device=dev)
+        out["sigma"] = torch.empty(P, dtype=torch.float32, device=dev)
+        out["nbar"] = torch.empty(P, dtype=torch.int32, device=dev)
+        out["flags"] = torch.empty(P, dtype=torch.uint8, device=dev)
+    return out
+
+
+def _check_stack(Y):
+    import torch
+    if not (isinstance(Y, torch.Tensor) and Y.is_cuda and Y.dtype == torch.float32 and Y.dim() == 2
+            and Y.stride(1) == 1):
+        raise TypeError("Y must be a CUDA float32 [N][P] tensor with unit column stride")
+
+
+def bfast_monitor(Y, dates, n_hist, k, h, lam, out_break=None, out_magnitude=None):
+    """North-star entry (synchronous).  Y: CUDA float32 [N][P] contiguous."""
+    _check_stack(Y)
+    N, P = Y.shape
+    if Y.stride(0) != P:
+        raise ValueError("bfast_monitor needs ldY == P; use bfast_monitor_ex")
+    d = _dates(dates)
+    if out_break is None or out_magnitude is None:
+        o = _outputs(Y, P, k, False)
+        out_break, out_magnitude = o["break"], o["magnitude"]
+    _check(lib().bfast_monitor(_dptr(Y), N, P, d.ctypes.data, int(n_hist), int(k), float(h),
+                               float(lam), _dptr(out_break), _dptr(out_magnitude)))
+    return out_break, out_magnitude
+
+
+def bfast_monitor_ex(Y, dates, n_hist, k, h, lam, P=None, diagnostics=False, stream=None, out=None):
+    """Asynchronous extended entry on `stream` (default: torch's current
+    stream).  Y may be a [N][ldY] view with P <= ldY columns used."""
+    _check_stack(Y)
+    P = int(Y.shape[1]) if P is None else int(P)
+    out = out if out is not None else _outputs(Y, P, k, diagnostics)
+    d = _dates(dates)
+    a = _make_args(Y, d, n_hist, k, h, lam, out["break"], out["magnitude"], P=P,
+                   out_beta=out.get("beta"), out_sigma=out.get("sigma"), out_nbar=out.get("nbar"),
+                   out_flags=out.get("flags"), stream=stream)
+    _check(lib().bfast_monitor_ex(ctypes.byref(a)))
+    out["_dates_keepalive"] = d
+    return out
+
+
+class Plan:
+    """bfast_plan_* wrapper: device constants for one (N, dates, n, k, h, lambda)."""
+
+    def __init__(self, device: int, N: int, dates, n_hist: int, k: int, h: float, lam: float):
+        self._h = ctypes.c_void_p()
+        self.dates = _dates(dates)
+        self.N, self.n_hist, self.k, self.hf, self.lam = int(N), int(n_hist), int(k), float(h), float(lam)
+        self.device = int(device)
+        _check(lib().bfast_plan_create(ctypes.byref(self._h), self.device, self.N, self.dates.ctypes.data,
+                                       self.n_hist, self.k, self.hf, self.lam))
+
+    def execute(self, Y, P=None, diagnostics=False, stream=None, out=None):
+        _check_stack(Y)
+        P = int(Y.shape[1]) if P is None else int(P)
+        out = out if out is not None else _outputs(Y, P, self.k, diagnostics)
+        a = _make_args(Y, self.dates, self.n_hist, self.k, self.hf, self.lam, out["break"],
+                       out["magnitude"], P=P, out_beta=out.get("beta"), out_sigma=out.get("sigma"),
+                       out_nbar=out.get("nbar"), out_flags=out.get("flags"), stream=stream)
+        _check(lib().bfast_plan_execute(self._h, ctypes.byref(a)))
+        return out
+
+    def close(self):
+        if self._h:
+            lib().bfast_plan_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def _host_ptr(a):
+    import torch
+    if isinstance(a, torch.Tensor):
+        assert not a.is_cuda and a.is_contiguous()
+        return int(a.data_ptr())
+    assert a.flags["C_CONTIGUOUS"]
+    return int(a.ctypes.data)
+
+
+def bfast_monitor_host(Y_host, dates, n_hist, k, h, lam, out_break=None, out_magnitude=None,
+                       P=None, device=-1):
+    """End-to-end on host buffers (pinned for full PCIe rate): H2D + kernels + D2H."""
+    N, ldY = int(Y_host.shape[0]), int(Y_host.shape[1])
+    P = ldY if P is None else int(P)
+    if out_break is None:
+        out_break = np.empty(P, np.int32)
+    if out_magnitude is None:
+        out_magnitude = np.empty(P, np.float32)
+    d = _dates(dates)
+    _check(lib().bfast_monitor_host(_host_ptr(Y_host), N, P, ldY, d.ctypes.data, int(n_hist), int(k),
+                                    float(h), float(lam), _host_ptr(out_break), _host_ptr(out_magnitude),
+                                    int(device)))
+    return out_break, out_magnitude
+
+
+def bfast_monitor_multi(Y_host, dates, n_hist, k, h, lam, devices, out_break=None, out_magnitude=None,
+                        P=None):
+    N, ldY = int(Y_host.shape[0]), int(Y_host.shape[1])
+    P = ldY if P is None else int(P)
+    if out_break is None:
+        out_break = np.empty(P, np.int32)
+    if out_magnitude is None:
+        out_magnitude = np.empty(P, np.float32)
+    devs = (ctypes.c_int * len(devices))(*devices)
+    d = _dates(dates)
+    _check(lib().bfast_monitor_multi(_host_ptr(Y_host), N, P, ldY, d.ctypes.data, int(n_hist), int(k),
+                                     float(h), float(lam), ctypes.cast(devs, ctypes.c_void_p),
+                                     len(devices), _host_ptr(out_break), _host_ptr(out_magnitude)))
+    return out_break, out_magnitude

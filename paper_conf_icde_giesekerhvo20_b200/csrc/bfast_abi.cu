@@ -1,0 +1,566 @@
+// bfast_abi.cu -- host side of libbfast.so: argument validation, plans
+// (design matrix in fp64 -> fp32 device constants), kernel launches, the
+// host-buffer (end-to-end) path and the multi-device shard driver.
+// Declarations and contracts: include/bfast.h.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "../../include/bfast.h"
+#include "monitor_simt.cuh"
+#include "refit_fp64.cuh"
+
+namespace {
+
+thread_local std::string g_err;
+thread_local int g_launches = 0;
+thread_local bool g_prof_on = false;
+thread_local std::vector<std::pair<cudaEvent_t, cudaEvent_t>> g_prof;
+
+int fail(int status, const char *fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return status;
+}
+
+#define CUDA_TRY(expr)                                                                 \
+  do {                                                                                 \
+    cudaError_t e_ = (expr);                                                           \
+    if (e_ != cudaSuccess)                                                             \
+      return fail(e_ == cudaErrorMemoryAllocation ? BFAST_ENOMEM : BFAST_ECUDA,        \
+                  "%s: %s (%s:%d)", #expr, cudaGetErrorString(e_), __FILE__, __LINE__); \
+  } while (0)
+
+constexpr int kMaxSmem = 227 * 1024;
+
+int validate_scalar(int64_t N, const double *dates, int32_t n_hist, int32_t k, float h,
+                    float lambda) {
+  if (N < 2) return fail(BFAST_EINVAL, "N=%lld < 2", (long long)N);
+  if (N > (int64_t)1 << 24) return fail(BFAST_EUNSUPPORTED, "N=%lld too large", (long long)N);
+  if (n_hist < 1 || n_hist > N - 1)
+    return fail(BFAST_EINVAL, "n_hist=%d outside [1, N-1]", n_hist);
+  if (k < 0) return fail(BFAST_EINVAL, "k=%d < 0", k);
+  if (!(h > 0.f && h <= 1.f)) return fail(BFAST_EINVAL, "h=%g outside (0, 1]", (double)h);
+  if (!(lambda > 0.f) || !std::isfinite(lambda))
+    return fail(BFAST_EINVAL, "lambda=%g must be finite and > 0", (double)lambda);
+  if (!dates) return fail(BFAST_EINVAL, "dates is NULL");
+  for (int64_t t = 0; t < N; ++t) {
+    if (!std::isfinite(dates[t])) return fail(BFAST_EINVAL, "dates[%lld] not finite", (long long)t);
+    if (t && !(dates[t] > dates[t - 1]))
+      return fail(BFAST_EINVAL, "dates not strictly increasing at %lld", (long long)t);
+  }
+  if (k > BFAST_K_MAX_HARMONICS)
+    return fail(BFAST_EUNSUPPORTED, "k=%d > %d", k, BFAST_K_MAX_HARMONICS);
+  return BFAST_OK;
+}
+
+int host_window(int nbar, float hf) {  // Fig. 12 L516 in f32, as the kernel
+  volatile float prod = (float)nbar * hf;
+  return (int)prod;
+}
+
+}  // namespace
+
+struct bfast_plan {
+  int device = 0;
+  int64_t N = 0;
+  int32_t n = 0, k = 0, K = 0, KP = 0;
+  float hf = 0.f, lambda = 0.f;
+  std::vector<double> dates;
+  double tc = 0.0, ts = 1.0;
+  int hcap = 1;
+  float *dX = nullptr;      // [N][KP] fp32
+  double *dX64 = nullptr;   // [N][K] fp64
+  int32_t *dcount = nullptr;
+  int32_t *dlist = nullptr;
+  int64_t list_cap = 0;
+  cudaEvent_t scratch_free = nullptr;  // orders executions sharing the refit scratch
+  std::mutex mu;
+  ~bfast_plan() {
+    int prev = -1;
+    cudaGetDevice(&prev);
+    cudaSetDevice(device);
+    cudaFree(dX);
+    cudaFree(dX64);
+    cudaFree(dcount);
+    cudaFree(dlist);
+    if (scratch_free) cudaEventDestroy(scratch_free);
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+namespace {
+
+// Design matrix of Eq. (3) (L65-L68) in fp64, with the trend regressor
+// centred and scaled, t' = (t - tc)/ts; rows padded
+// to KP columns.
+void build_design(const bfast_plan &pl, std::vector<float> &X, std::vector<double> &X64) {
+  const double two_pi = 6.283185307179586476925286766559;
+  X.assign((size_t)pl.N * pl.KP, 0.f);
+  X64.assign((size_t)pl.N * pl.K, 0.0);
+  for (int64_t t = 0; t < pl.N; ++t) {
+    double row[2 + 2 * BFAST_K_MAX_HARMONICS];
+    row[0] = 1.0;
+    row[1] = ((double)(t + 1) - pl.tc) / pl.ts;
+    for (int j = 1; j <= pl.k; ++j) {
+      double F = two_pi * (double)j * pl.dates[t];
+      row[2 * j] = std::sin(F);
+      row[2 * j + 1] = std::cos(F);
+    }
+    for (int i = 0; i < pl.K; ++i) {
+      X[(size_t)t * pl.KP + i] = (float)row[i];
+      X64[(size_t)t * pl.K + i] = row[i];
+    }
+  }
+}
+
+size_t simt_smem(const bfast_plan &pl, int bp) {
+  return (size_t)pl.N * pl.KP * sizeof(float) + (size_t)pl.hcap * bp * (sizeof(float) + sizeof(int));
+}
+
+template <int K>
+int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t st) {
+  static thread_local int configured_dev = -1;
+  int bp = 128;
+  while (bp > 32 && simt_smem(pl, bp) > (size_t)kMaxSmem) bp >>= 1;
+  size_t smem = simt_smem(pl, bp);
+  if (smem > (size_t)kMaxSmem) return fail(BFAST_EUNSUPPORTED, "shared memory %zu B too large", smem);
+  if (configured_dev != pl.device) {
+    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_simt_kernel<K>,
+                                  cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmem));
+    CUDA_TRY(cudaFuncSetAttribute(bfast::refit_fp64_kernel<K>,
+                                  cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmem));
+    configured_dev = pl.device;
+  }
+  const int64_t blocks = (prm.P + bp - 1) / bp;
+  if (blocks > 0x7fffffff) return fail(BFAST_EUNSUPPORTED, "P too large");
+  // the refit list/counter are plan scratch: order executions on any stream
+  CUDA_TRY(cudaStreamWaitEvent(st, pl.scratch_free, 0));
+  CUDA_TRY(cudaMemsetAsync(prm.refit_count, 0, sizeof(int32_t), st));
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  if (g_prof_on) {
+    CUDA_TRY(cudaEventCreate(&e0));
+    CUDA_TRY(cudaEventCreate(&e1));
+    CUDA_TRY(cudaEventRecord(e0, st));
+  }
+  bfast::monitor_simt_kernel<K><<<(unsigned)blocks, bp, smem, st>>>(prm);
+  CUDA_TRY(cudaGetLastError());
+  if (g_prof_on) {
+    CUDA_TRY(cudaEventRecord(e1, st));
+    g_prof.emplace_back(e0, e1);
+  }
+  // fp64 refit of flagged pixels; exits at once when the list is empty
+  const int rwarps = 4;
+  const size_t rsmem = (size_t)rwarps * (pl.N + 1) * sizeof(double);
+  if (rsmem > (size_t)kMaxSmem) return fail(BFAST_EUNSUPPORTED, "refit smem too large");
+  int sms = 148;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, pl.device);
+  bfast::refit_fp64_kernel<K><<<sms * 4, rwarps * 32, rsmem, st>>>(prm);
+  CUDA_TRY(cudaGetLastError());
+  CUDA_TRY(cudaEventRecord(pl.scratch_free, st));
+  g_launches = 2;
+  return BFAST_OK;
+}
+
+int launch(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t st) {
+  switch (pl.k) {
+    case 0: return launch_k<2>(pl, prm, st);
+    case 1: return launch_k<4>(pl, prm, st);
+    case 2: return launch_k<6>(pl, prm, st);
+    case 3: return launch_k<8>(pl, prm, st);
+    case 4: return launch_k<10>(pl, prm, st);
+    case 5: return launch_k<12>(pl, prm, st);
+    case 6: return launch_k<14>(pl, prm, st);
+  }
+  return fail(BFAST_EUNSUPPORTED, "k=%d", pl.k);
+}
+
+// --- one-shot plan cache (bfast_monitor / bfast_monitor_ex / host paths)
+std::mutex g_cache_mu;
+std::vector<std::unique_ptr<bfast_plan>> g_cache;
+
+bool same_plan(const bfast_plan &pl, int dev, int64_t N, const double *dates, int32_t n, int32_t k,
+               float h, float lambda) {
+  return pl.device == dev && pl.N == N && pl.n == n && pl.k == k && pl.hf == h &&
+         pl.lambda == lambda && std::memcmp(pl.dates.data(), dates, sizeof(double) * N) == 0;
+}
+
+int cached_plan(int dev, int64_t N, const double *dates, int32_t n, int32_t k, float h, float lambda,
+                bfast_plan **out) {
+  std::lock_guard<std::mutex> g(g_cache_mu);
+  for (auto &p : g_cache)
+    if (same_plan(*p, dev, N, dates, n, k, h, lambda)) {
+      *out = p.get();
+      return BFAST_OK;
+    }
+  bfast_plan *pl = nullptr;
+  int rc = bfast_plan_create(&pl, dev, N, dates, n, k, h, lambda);
+  if (rc) return rc;
+  if (g_cache.size() >= 16) g_cache.erase(g_cache.begin());
+  g_cache.emplace_back(pl);
+  *out = pl;
+  return BFAST_OK;
+}
+
+int ensure_list(bfast_plan &pl, int64_t P) {
+  if (P <= pl.list_cap) return BFAST_OK;
+  cudaFree(pl.dlist);
+  pl.dlist = nullptr;
+  pl.list_cap = 0;
+  CUDA_TRY(cudaMalloc(&pl.dlist, sizeof(int32_t) * (size_t)std::max<int64_t>(P, 1)));
+  pl.list_cap = P;
+  return BFAST_OK;
+}
+
+int execute_range(bfast_plan &pl, const bfast_args *a, int64_t p0, int64_t P) {
+  if (P == 0) {
+    g_launches = 0;
+    return BFAST_OK;
+  }
+  int rc = ensure_list(pl, P);
+  if (rc) return rc;
+  bfast::MonitorParams prm{};
+  prm.Y = a->Y;
+  prm.ldY = a->ldY;
+  prm.P = P;
+  prm.p0 = p0;
+  prm.N = (int)pl.N;
+  prm.n = pl.n;
+  prm.X = pl.dX;
+  prm.X64 = pl.dX64;
+  prm.KP = pl.KP;
+  prm.hf = pl.hf;
+  prm.lambda = pl.lambda;
+  prm.hcap = pl.hcap;
+  prm.tc = pl.tc;
+  prm.ts = pl.ts;
+  prm.out_break = a->out_break;
+  prm.out_mag = a->out_magnitude;
+  prm.out_beta = a->out_beta;
+  prm.out_sigma = a->out_sigma;
+  prm.out_nbar = a->out_nbar;
+  prm.out_flags = a->out_flags;
+  prm.refit_list = pl.dlist;
+  prm.refit_count = pl.dcount;
+  return launch(pl, prm, (cudaStream_t)a->stream);
+}
+
+int validate_args(const bfast_args *a) {
+  if (!a) return fail(BFAST_EINVAL, "args is NULL");
+  int rc = validate_scalar(a->N, a->dates, a->n_hist, a->k, a->h, a->lambda);
+  if (rc) return rc;
+  if (a->P < 0) return fail(BFAST_EINVAL, "P < 0");
+  if (a->ldY < a->P) return fail(BFAST_EINVAL, "ldY < P");
+  if (a->P > 0 && (!a->Y || !a->out_break || !a->out_magnitude))
+    return fail(BFAST_EINVAL, "NULL Y/out_break/out_magnitude");
+  if ((a->N - 1) * (double)a->ldY + a->P > 9.0e18) return fail(BFAST_EINVAL, "stack too large");
+  return BFAST_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int bfast_abi_version(void) { return BFAST_ABI_VERSION; }
+
+const char *bfast_last_error(void) { return g_err.c_str(); }
+
+int bfast_last_launch_count(void) { return g_launches; }
+
+int bfast_profile_enable(int on) {
+  g_prof_on = on != 0;
+  if (!g_prof_on) {
+    for (auto &e : g_prof) {
+      cudaEventDestroy(e.first);
+      cudaEventDestroy(e.second);
+    }
+    g_prof.clear();
+  }
+  return BFAST_OK;
+}
+
+int bfast_profile_collect(float *ms_out, int max) {
+  int n = 0;
+  int rc = BFAST_OK;
+  for (auto &e : g_prof) {
+    float ms = 0.f;
+    if (rc == BFAST_OK) {
+      cudaError_t err = cudaEventSynchronize(e.second);
+      if (err == cudaSuccess) err = cudaEventElapsedTime(&ms, e.first, e.second);
+      if (err != cudaSuccess) rc = fail(BFAST_ECUDA, "profile: %s", cudaGetErrorString(err));
+    }
+    if (rc == BFAST_OK && ms_out && n < max) ms_out[n++] = ms;
+    cudaEventDestroy(e.first);
+    cudaEventDestroy(e.second);
+  }
+  g_prof.clear();
+  return rc == BFAST_OK ? n : rc;
+}
+
+const char *bfast_status_string(int s) {
+  switch (s) {
+    case BFAST_OK: return "BFAST_OK";
+    case BFAST_EINVAL: return "BFAST_EINVAL";
+    case BFAST_EUNSUPPORTED: return "BFAST_EUNSUPPORTED";
+    case BFAST_ECUDA: return "BFAST_ECUDA";
+    case BFAST_ENOMEM: return "BFAST_ENOMEM";
+  }
+  return "unknown status";
+}
+
+void bfast_shard_range(int64_t P, int rank, int world, int64_t *begin, int64_t *end) {
+  if (world < 1 || rank < 0 || rank >= world || P <= 0) {
+    *begin = *end = 0;
+    return;
+  }
+  const int64_t tiles = (P + 127) / 128;
+  const int64_t b = tiles * rank / world, e = tiles * (rank + 1) / world;
+  *begin = std::min(P, b * 128);
+  *end = std::min(P, e * 128);
+}
+
+int bfast_plan_create(bfast_plan **out, int device, int64_t N, const double *dates, int32_t n_hist,
+                      int32_t k, float h, float lambda) {
+  if (!out) return fail(BFAST_EINVAL, "out is NULL");
+  *out = nullptr;
+  int rc = validate_scalar(N, dates, n_hist, k, h, lambda);
+  if (rc) return rc;
+  std::unique_ptr<bfast_plan> pl(new bfast_plan());
+  pl->device = device;
+  pl->N = N;
+  pl->n = n_hist;
+  pl->k = k;
+  pl->K = 2 + 2 * k;
+  pl->KP = (pl->K + 3) / 4 * 4;
+  pl->hf = h;
+  pl->lambda = lambda;
+  pl->dates.assign(dates, dates + N);
+  pl->tc = 0.5 * ((double)n_hist + 1.0);
+  pl->ts = n_hist > 1 ? 0.5 * ((double)n_hist - 1.0) : 1.0;
+  pl->hcap = std::max(1, host_window(n_hist, h));
+  if (simt_smem(*pl, 32) > (size_t)kMaxSmem)
+    return fail(BFAST_EUNSUPPORTED, "N=%lld with window %d exceeds shared memory", (long long)N,
+                pl->hcap);
+  if ((size_t)4 * (N + 1) * sizeof(double) > (size_t)kMaxSmem)
+    return fail(BFAST_EUNSUPPORTED, "N=%lld too large for the refit kernel", (long long)N);
+  std::vector<float> X;
+  std::vector<double> X64;
+  build_design(*pl, X, X64);
+  int prev = -1;
+  CUDA_TRY(cudaGetDevice(&prev));
+  CUDA_TRY(cudaSetDevice(device));
+  cudaError_t e = cudaMalloc(&pl->dX, X.size() * sizeof(float));
+  if (e == cudaSuccess) e = cudaMalloc(&pl->dX64, X64.size() * sizeof(double));
+  if (e == cudaSuccess) e = cudaMalloc(&pl->dcount, sizeof(int32_t));
+  if (e == cudaSuccess) e = cudaMemcpy(pl->dX, X.data(), X.size() * sizeof(float), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess)
+    e = cudaMemcpy(pl->dX64, X64.data(), X64.size() * sizeof(double), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemset(pl->dcount, 0, sizeof(int32_t));
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&pl->scratch_free, cudaEventDisableTiming);
+  cudaSetDevice(prev);
+  if (e != cudaSuccess)
+    return fail(e == cudaErrorMemoryAllocation ? BFAST_ENOMEM : BFAST_ECUDA, "plan: %s",
+                cudaGetErrorString(e));
+  *out = pl.release();
+  return BFAST_OK;
+}
+
+void bfast_plan_destroy(bfast_plan *plan) { delete plan; }
+
+int bfast_plan_execute(const bfast_plan *plan, const bfast_args *a) {
+  if (!plan) return fail(BFAST_EINVAL, "plan is NULL");
+  int rc = validate_args(a);
+  if (rc) return rc;
+  bfast_plan &pl = const_cast<bfast_plan &>(*plan);
+  if (!same_plan(pl, pl.device, a->N, a->dates, a->n_hist, a->k, a->h, a->lambda))
+    return fail(BFAST_EINVAL, "args do not match the plan");
+  std::lock_guard<std::mutex> g(pl.mu);
+  int prev = -1;
+  CUDA_TRY(cudaGetDevice(&prev));
+  if (prev != pl.device) CUDA_TRY(cudaSetDevice(pl.device));
+  rc = execute_range(pl, a, 0, a->P);
+  if (prev != pl.device) cudaSetDevice(prev);
+  return rc;
+}
+
+int bfast_monitor_ex(const bfast_args *a) {
+  int rc = validate_args(a);
+  if (rc) return rc;
+  int dev = 0;
+  CUDA_TRY(cudaGetDevice(&dev));
+  bfast_plan *pl = nullptr;
+  rc = cached_plan(dev, a->N, a->dates, a->n_hist, a->k, a->h, a->lambda, &pl);
+  if (rc) return rc;
+  std::lock_guard<std::mutex> g(pl->mu);
+  return execute_range(*pl, a, 0, a->P);
+}
+
+int bfast_monitor(const float *Y, int64_t N, int64_t P, const double *dates, int32_t n_hist,
+                  int32_t k, float h, float lambda, int32_t *out_break, float *out_magnitude) {
+  bfast_args a{};
+  a.Y = Y;
+  a.N = N;
+  a.P = P;
+  a.ldY = P;
+  a.dates = dates;
+  a.n_hist = n_hist;
+  a.k = k;
+  a.h = h;
+  a.lambda = lambda;
+  a.out_break = out_break;
+  a.out_magnitude = out_magnitude;
+  int rc = bfast_monitor_ex(&a);
+  if (rc) return rc;
+  CUDA_TRY(cudaStreamSynchronize(nullptr));
+  return BFAST_OK;
+}
+
+// End-to-end on host buffers: pixel slabs, double-buffered H2D on a copy
+// stream overlapping the kernel on the compute stream.
+int bfast_monitor_host(const float *Y_host, int64_t N, int64_t P, int64_t ldY, const double *dates,
+                       int32_t n_hist, int32_t k, float h, float lambda, int32_t *out_break_host,
+                       float *out_magnitude_host, int device) {
+  int rc = validate_scalar(N, dates, n_hist, k, h, lambda);
+  if (rc) return rc;
+  if (P < 0 || ldY < P) return fail(BFAST_EINVAL, "P < 0 or ldY < P");
+  if (P == 0) {
+    g_launches = 0;
+    return BFAST_OK;
+  }
+  if (!Y_host || !out_break_host || !out_magnitude_host) return fail(BFAST_EINVAL, "NULL pointer");
+  int prev = 0;
+  CUDA_TRY(cudaGetDevice(&prev));
+  const int dev = device < 0 ? prev : device;
+  CUDA_TRY(cudaSetDevice(dev));
+  bfast_plan *pl = nullptr;
+  rc = cached_plan(dev, N, dates, n_hist, k, h, lambda, &pl);
+  if (rc) {
+    cudaSetDevice(prev);
+    return rc;
+  }
+  // slab width: ~1 GiB of stack per buffer, multiple of 128 pixels
+  int64_t slab = std::max<int64_t>(128, ((int64_t)1 << 28) / N / 128 * 128);
+  slab = std::min<int64_t>(slab, (P + 127) / 128 * 128);
+  float *dY[2] = {nullptr, nullptr};
+  int32_t *dB[2] = {nullptr, nullptr};
+  float *dM[2] = {nullptr, nullptr};
+  cudaStream_t cs = nullptr, ks = nullptr;
+  cudaEvent_t loaded[2] = {nullptr, nullptr}, done[2] = {nullptr, nullptr};
+  int launches = 0;
+  cudaError_t e = cudaSuccess;
+  auto cleanup = [&]() {
+    for (int i = 0; i < 2; ++i) {
+      cudaFree(dY[i]);
+      cudaFree(dB[i]);
+      cudaFree(dM[i]);
+      if (loaded[i]) cudaEventDestroy(loaded[i]);
+      if (done[i]) cudaEventDestroy(done[i]);
+    }
+    if (cs) cudaStreamDestroy(cs);
+    if (ks) cudaStreamDestroy(ks);
+    cudaSetDevice(prev);
+  };
+  for (int i = 0; i < 2 && e == cudaSuccess; ++i) {
+    e = cudaMalloc(&dY[i], sizeof(float) * (size_t)N * slab);
+    if (e == cudaSuccess) e = cudaMalloc(&dB[i], sizeof(int32_t) * slab);
+    if (e == cudaSuccess) e = cudaMalloc(&dM[i], sizeof(float) * slab);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&loaded[i], cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&done[i], cudaEventDisableTiming);
+  }
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ks, cudaStreamNonBlocking);
+  if (e != cudaSuccess) {
+    cleanup();
+    return fail(e == cudaErrorMemoryAllocation ? BFAST_ENOMEM : BFAST_ECUDA, "host path: %s",
+                cudaGetErrorString(e));
+  }
+  std::lock_guard<std::mutex> g(pl->mu);
+  int slot = 0;
+  for (int64_t b0 = 0; b0 < P && rc == BFAST_OK; b0 += slab, slot ^= 1) {
+    const int64_t w = std::min(slab, P - b0);
+    // the buffer is free once the kernel that used it two slabs ago is done
+    e = cudaStreamWaitEvent(cs, done[slot], 0);
+    if (e == cudaSuccess)
+      e = cudaMemcpy2DAsync(dY[slot], sizeof(float) * w, Y_host + b0, sizeof(float) * ldY,
+                            sizeof(float) * w, N, cudaMemcpyHostToDevice, cs);
+    if (e == cudaSuccess) e = cudaEventRecord(loaded[slot], cs);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(ks, loaded[slot], 0);
+    if (e != cudaSuccess) break;
+    bfast_args a{};
+    a.Y = dY[slot];
+    a.N = N;
+    a.P = w;
+    a.ldY = w;
+    a.dates = dates;
+    a.n_hist = n_hist;
+    a.k = k;
+    a.h = h;
+    a.lambda = lambda;
+    a.out_break = dB[slot];
+    a.out_magnitude = dM[slot];
+    a.stream = ks;
+    rc = execute_range(*pl, &a, 0, w);
+    launches += g_launches;
+    if (rc) break;
+    e = cudaMemcpyAsync(out_break_host + b0, dB[slot], sizeof(int32_t) * w, cudaMemcpyDeviceToHost, ks);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(out_magnitude_host + b0, dM[slot], sizeof(float) * w, cudaMemcpyDeviceToHost, ks);
+    if (e == cudaSuccess) e = cudaEventRecord(done[slot], ks);
+    if (e != cudaSuccess) break;
+  }
+  if (e == cudaSuccess && rc == BFAST_OK) e = cudaStreamSynchronize(ks);
+  cleanup();
+  if (rc) return rc;
+  if (e != cudaSuccess) return fail(BFAST_ECUDA, "host path: %s", cudaGetErrorString(e));
+  g_launches = launches;
+  return BFAST_OK;
+}
+
+int bfast_monitor_multi(const float *Y_host, int64_t N, int64_t P, int64_t ldY, const double *dates,
+                        int32_t n_hist, int32_t k, float h, float lambda, const int *devices, int ndev,
+                        int32_t *out_break_host, float *out_magnitude_host) {
+  int rc = validate_scalar(N, dates, n_hist, k, h, lambda);
+  if (rc) return rc;
+  if (!devices || ndev < 1) return fail(BFAST_EINVAL, "no devices");
+  if (P < 0 || ldY < P) return fail(BFAST_EINVAL, "P < 0 or ldY < P");
+  if (P > 0 && (!Y_host || !out_break_host || !out_magnitude_host))
+    return fail(BFAST_EINVAL, "NULL pointer");
+  std::vector<int> status(ndev, BFAST_OK);
+  std::vector<std::string> errs(ndev);
+  std::vector<int> launches(ndev, 0);
+  std::vector<std::thread> th;
+  for (int r = 0; r < ndev; ++r) {
+    th.emplace_back([&, r]() {
+      int64_t b, e;
+      bfast_shard_range(P, r, ndev, &b, &e);
+      if (e > b)
+        status[r] = bfast_monitor_host(Y_host + b, N, e - b, ldY, dates, n_hist, k, h, lambda,
+                                       out_break_host + b, out_magnitude_host + b, devices[r]);
+      errs[r] = g_err;
+      launches[r] = g_launches;
+    });
+  }
+  for (auto &t : th) t.join();
+  int total = 0;
+  for (int r = 0; r < ndev; ++r) {
+    if (status[r]) return fail(status[r], "device %d: %s", devices[r], errs[r].c_str());
+    total += launches[r];
+  }
+  g_launches = total;
+  return BFAST_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,183 @@
+// refit_fp64.cuh -- fp64 recomputation of the pixels the fp32 pass flagged
+// as ill-conditioned (pivot ratio < kRefitRatio), one warp per pixel.
+//
+// Same definitions as the fused pass (Algorithm 1; Fig. 12
+// L478-L537), organised for a warp instead of a thread:
+//   - lanes take 32 consecutive dates; validity is a warp ballot and the
+//     order-preserving compaction of filterNaNsWKeys (L483-L490) is the
+//     popc-prefix of that ballot (the scan+scatter of Fig. 12 in one
+//     instruction pair);
+//   - the masked Gram / moment (Alg. 1 l.2, l.4) are accumulated per lane in
+//     fp64 and reduced with xor-shuffles;
+//   - every lane solves the same fp64 system (Cholesky, rank test on the
+//     unit-diagonal pivots as the oracle's reading R4 does);
+//   - compacted residuals go to a per-warp shared-memory array; the MOSUM
+//     windows (Eq. (4)) are prefix-sum differences; the first
+//     break is a ballot over j in order (the (bool, idx) reduce of
+//     L532-L534) and the mean a shuffle reduction.
+#pragma once
+#include "monitor_simt.cuh"
+
+namespace bfast {
+
+__device__ __forceinline__ double warp_sum(double v) {
+#pragma unroll
+  for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+template <int K>
+__global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
+  extern __shared__ double rbuf_all[];  // [warps][N + 1] compacted residual prefix sums
+  const int lane = threadIdx.x & 31;
+  const int wib = threadIdx.x >> 5;
+  const int wpb = blockDim.x >> 5;
+  double *S = rbuf_all + (size_t)wib * (p.N + 1);
+  const int count = *p.refit_count;
+  const int n = p.n, N = p.N;
+  const int64_t ldY = p.ldY;
+  const double qnan = __longlong_as_double(0x7ff8000000000000ll);
+
+  for (int item = blockIdx.x * wpb + wib; item < count; item += gridDim.x * wpb) {
+    const int64_t pix = p.p0 + p.refit_list[item];
+    const float *ycol = p.Y + pix;
+    // ---- history: offset, Gram, moment (fp64)
+    double A[Tri<K>::kN], b[K];
+#pragma unroll
+    for (int i = 0; i < Tri<K>::kN; ++i) A[i] = 0.0;
+#pragma unroll
+    for (int i = 0; i < K; ++i) b[i] = 0.0;
+    double c0 = 0.0;
+    bool have = false;
+    int nbar = 0;
+    double ymax = 0.0;
+    for (int t0 = 0; t0 < n; t0 += 32) {
+      const int t = t0 + lane;
+      const float yf = t < n ? ycol[(int64_t)t * ldY] : __int_as_float(0x7fc00000);
+      const bool v = (yf == yf);
+      const unsigned bal = __ballot_sync(0xffffffffu, v);
+      if (!bal) continue;
+      if (!have) {
+        c0 = (double)__shfl_sync(0xffffffffu, yf, __ffs(bal) - 1);
+        have = true;
+      }
+      nbar += __popc(bal);
+      if (v) {
+        const double y = (double)yf - c0;
+        ymax = fmax(ymax, fabs((double)yf));
+        const double *x = p.X64 + (size_t)t * K;
+        double xr[K];
+#pragma unroll
+        for (int i = 0; i < K; ++i) xr[i] = x[i];
+#pragma unroll
+        for (int i = 0; i < K; ++i) {
+#pragma unroll
+          for (int j = i; j < K; ++j) A[Tri<K>::idx(i, j)] = fma(xr[i], xr[j], A[Tri<K>::idx(i, j)]);
+          b[i] = fma(y, xr[i], b[i]);
+        }
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < Tri<K>::kN; ++i) A[i] = warp_sum(A[i]);
+#pragma unroll
+    for (int i = 0; i < K; ++i) b[i] = warp_sum(b[i]);
+#pragma unroll
+    for (int o = 16; o; o >>= 1) ymax = fmax(ymax, __shfl_xor_sync(0xffffffffu, ymax, o));
+
+    double beta[K];
+    const double minratio = chol_solve<K>(A, b, beta);
+    const int h = window_h(nbar, p.hf);
+    bool deg = !(minratio > 1e-9);  // rank test (reading R4)
+
+    // ---- residuals of all dates, compacted in order, as prefix sums S
+    double s2 = 0.0;
+    int cr = 0;
+    if (lane == 0) S[0] = 0.0;
+    for (int t0 = 0; t0 < N; t0 += 32) {
+      const int t = t0 + lane;
+      const float yf = t < N ? ycol[(int64_t)t * ldY] : __int_as_float(0x7fc00000);
+      const bool v = (yf == yf);
+      const unsigned bal = __ballot_sync(0xffffffffu, v);
+      double r = 0.0;
+      if (v) {
+        const double *x = p.X64 + (size_t)t * K;
+        double yhat = 0.0;
+#pragma unroll
+        for (int i = 0; i < K; ++i) yhat = fma(x[i], beta[i], yhat);
+        r = ((double)yf - c0) - yhat;
+      }
+      if (t < n) s2 += r * r;
+      // inclusive warp scan of r over valid lanes (invalid lanes carry 0)
+      double sc = r;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        double up = __shfl_up_sync(0xffffffffu, sc, o);
+        if (lane >= o) sc += up;
+      }
+      const double base = S[cr];
+      __syncwarp();
+      const int rank = cr + __popc(bal & ((1u << lane) - 1));
+      if (v) S[rank + 1] = base + sc;
+      cr += __popc(bal);
+      __syncwarp();
+    }
+    const int Nbar = cr;
+    s2 = warp_sum(s2);
+    const double sigma = sqrt(s2 / (double)(nbar - K));
+    if (!(sigma > 1e-4 * ymax)) deg = true;
+    // ---- MOSUM by prefix differences, first break, mean
+    const double scale = sigma * sqrt((double)nbar);
+    double msum = 0.0;
+    int jstar = -1;
+    const int J = Nbar - nbar;
+    for (int j0 = 0; j0 < J; j0 += 32) {
+      const int j = j0 + lane;
+      bool hit = false;
+      if (j < J) {
+        const double m = (S[nbar + j + 1] - S[nbar + j - h + 1]) / scale;
+        msum += m;
+        const double x = (double)(nbar + 1 + j) / (double)nbar;
+        const double B = (double)p.lambda * sqrt(fmax(1.0, log(x)));
+        hit = fabs(m) > B;
+      }
+      const unsigned hb = __ballot_sync(0xffffffffu, hit);
+      if (jstar < 0 && hb) jstar = j0 + __ffs(hb) - 1;
+    }
+    msum = warp_sum(msum);
+    // original date index of compacted rank nbar + jstar (REMAPINDICES)
+    int brk = -1;
+    if (jstar >= 0) {
+      int target = nbar + jstar, seen = 0;
+      for (int t0 = 0; t0 < N; t0 += 32) {
+        const int t = t0 + lane;
+        const float yf = t < N ? ycol[(int64_t)t * ldY] : __int_as_float(0x7fc00000);
+        const unsigned bal = __ballot_sync(0xffffffffu, yf == yf);
+        const int c = __popc(bal);
+        if (seen + c > target) {
+          unsigned bb = bal;
+          for (int q = 0; q < target - seen; ++q) bb &= bb - 1;
+          brk = t0 + __ffs(bb) - 1 - n;
+          break;
+        }
+        seen += c;
+      }
+    }
+    if (lane == 0) {
+      p.out_break[pix] = deg ? -2 : brk;
+      p.out_mag[pix] = deg ? (float)qnan : (float)(msum / (double)J);
+      if (p.out_sigma) p.out_sigma[pix] = (float)sigma;
+      if (p.out_flags) p.out_flags[pix] = (uint8_t)((deg ? 1u : 0u) | 2u);
+      if (p.out_beta) {
+        float *o = p.out_beta + pix * K;
+        const bool rank_def = !(minratio > 1e-9);
+        o[0] = rank_def ? (float)qnan : (float)(beta[0] - beta[1] * p.tc / p.ts + c0);
+        o[1] = rank_def ? (float)qnan : (float)(beta[1] / p.ts);
+#pragma unroll
+        for (int i = 2; i < K; ++i) o[i] = rank_def ? (float)qnan : (float)beta[i];
+      }
+    }
+    __syncwarp();
+  }
+}
+
+}  // namespace bfast
