@@ -49,7 +49,7 @@ constexpr int kMaxSmem = 227 * 1024;
 int validate_scalar(int64_t N, const double *dates, int32_t n_hist, int32_t k, float h,
                     float lambda) {
   if (N < 2) return fail(BFAST_EINVAL, "N=%lld < 2", (long long)N);
-  if (N > (int64_t)1 << 24) return fail(BFAST_EUNSUPPORTED, "N=%lld too large", (long long)N);
+  if (N > 32767) return fail(BFAST_EUNSUPPORTED, "N=%lld > 32767 dates", (long long)N);
   if (n_hist < 1 || n_hist > N - 1)
     return fail(BFAST_EINVAL, "n_hist=%d outside [1, N-1]", n_hist);
   if (k < 0) return fail(BFAST_EINVAL, "k=%d < 0", k);
@@ -128,7 +128,7 @@ void build_design(const bfast_plan &pl, std::vector<float> &X, std::vector<doubl
 }
 
 size_t simt_smem(const bfast_plan &pl, int bp) {
-  return (size_t)pl.N * pl.KP * sizeof(float) + (size_t)pl.hcap * bp * (sizeof(float) + sizeof(int));
+  return (size_t)pl.N * pl.KP * sizeof(float) + (size_t)pl.hcap * bp * (sizeof(float) + sizeof(int16_t));
 }
 
 template <int K>

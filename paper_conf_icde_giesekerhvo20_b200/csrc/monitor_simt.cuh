@@ -29,6 +29,7 @@
 // refit_fp64.cuh.
 #pragma once
 #include <cstdint>
+#include <type_traits>
 #include <cuda_runtime.h>
 
 namespace bfast {
@@ -89,55 +90,90 @@ struct Tri {
   }
 };
 
-// fp64 Cholesky solve of the packed SPD system (A, b) -> beta.  Returns the
-// smallest pivot ratio d_j / A_jj (1 - R^2 of column j on the previous
-// ones), a cheap conditioning proxy; <= 0 means not positive definite.
-template <int K>
-__device__ __forceinline__ double chol_solve(const double (&A)[Tri<K>::kN], const double (&b)[K],
-                                             double (&beta)[K]) {
-  double L[Tri<K>::kN];
-  double minratio = 1.0;
-#pragma unroll
-  for (int j = 0; j < K; ++j) {
-    double d = A[Tri<K>::idx(j, j)];
-#pragma unroll
-    for (int q = 0; q < j; ++q) d -= L[Tri<K>::idx(q, j)] * L[Tri<K>::idx(q, j)];
-    double ratio = d / A[Tri<K>::idx(j, j)];
-    minratio = fmin(minratio, ratio);
-    double ljj = sqrt(fmax(d, 1e-300));
-    double inv = 1.0 / ljj;
-    L[Tri<K>::idx(j, j)] = ljj;
-#pragma unroll
-    for (int i = j + 1; i < K; ++i) {
-      double s = A[Tri<K>::idx(j, i)];
-#pragma unroll
-      for (int q = 0; q < j; ++q) s -= L[Tri<K>::idx(q, i)] * L[Tri<K>::idx(q, j)];
-      L[Tri<K>::idx(j, i)] = s * inv;  // L stored transposed: L[q][i] = l_{iq}
+// Compile-time loop: f(std::integral_constant<int, I>) for I in [B, E), so
+// every register-array index below is a constant (no local memory).
+template <int B, int E>
+struct SFor {
+  template <class F>
+  __device__ __forceinline__ static void run(F &&f) {
+    if constexpr (B < E) {
+      f(std::integral_constant<int, B>{});
+      SFor<B + 1, E>::run(f);
     }
   }
-  double z[K];
-#pragma unroll
-  for (int i = 0; i < K; ++i) {
-    double s = b[i];
-#pragma unroll
-    for (int q = 0; q < i; ++q) s -= L[Tri<K>::idx(q, i)] * z[q];
-    z[i] = s / L[Tri<K>::idx(i, i)];
+};
+template <int B, int E>
+struct SForDown {  // I = E-1 down to B
+  template <class F>
+  __device__ __forceinline__ static void run(F &&f) {
+    if constexpr (B < E) {
+      f(std::integral_constant<int, E - 1>{});
+      SForDown<B, E - 1>::run(f);
+    }
   }
-#pragma unroll
-  for (int i = K - 1; i >= 0; --i) {
-    double s = z[i];
-#pragma unroll
-    for (int q = i + 1; q < K; ++q) s -= L[Tri<K>::idx(i, q)] * beta[q];
-    beta[i] = s / L[Tri<K>::idx(i, i)];
-  }
+};
+
+// Cholesky factorisation in place of the packed SPD matrix A (upper
+// triangle, row-major): on return A holds L^T (A[idx(q,i)] = l_iq).  Returns
+// the smallest pivot ratio d_j / A_jj (1 - R^2 of column j on the previous
+// ones), a cheap conditioning proxy; <= 0 means not positive definite.
+template <int K, typename T>
+__device__ __forceinline__ T chol_factor(T (&A)[Tri<K>::kN]) {
+  T minratio = T(1);
+  SFor<0, K>::run([&](auto jc) {
+    constexpr int j = decltype(jc)::value;
+    T d = A[Tri<K>::idx(j, j)];
+    SFor<0, j>::run([&](auto qc) {
+      constexpr int q = decltype(qc)::value;
+      d -= A[Tri<K>::idx(q, j)] * A[Tri<K>::idx(q, j)];
+    });
+    const T ratio = d / A[Tri<K>::idx(j, j)];
+    minratio = ratio < minratio ? ratio : minratio;
+    const T ljj = sqrt(d > T(1e-30) ? d : T(1e-30));
+    const T inv = T(1) / ljj;
+    A[Tri<K>::idx(j, j)] = ljj;
+    SFor<j + 1, K>::run([&](auto ic) {
+      constexpr int i = decltype(ic)::value;
+      T s = A[Tri<K>::idx(j, i)];
+      SFor<0, j>::run([&](auto qc) {
+        constexpr int q = decltype(qc)::value;
+        s -= A[Tri<K>::idx(q, i)] * A[Tri<K>::idx(q, j)];
+      });
+      A[Tri<K>::idx(j, i)] = s * inv;
+    });
+  });
   return minratio;
+}
+
+// Solve L L^T x = b with the factor of chol_factor.
+template <int K, typename T>
+__device__ __forceinline__ void chol_solve(const T (&L)[Tri<K>::kN], const T (&b)[K], T (&x)[K]) {
+  T z[K];
+  SFor<0, K>::run([&](auto ic) {
+    constexpr int i = decltype(ic)::value;
+    T s = b[i];
+    SFor<0, i>::run([&](auto qc) {
+      constexpr int q = decltype(qc)::value;
+      s -= L[Tri<K>::idx(q, i)] * z[q];
+    });
+    z[i] = s / L[Tri<K>::idx(i, i)];
+  });
+  SForDown<0, K>::run([&](auto ic) {
+    constexpr int i = decltype(ic)::value;
+    T s = z[i];
+    SFor<i + 1, K>::run([&](auto qc) {
+      constexpr int q = decltype(qc)::value;
+      s -= L[Tri<K>::idx(i, q)] * x[q];
+    });
+    x[i] = s / L[Tri<K>::idx(i, i)];
+  });
 }
 
 // Back-transform from the centred basis with offset c to the ABI basis
 // (1, t, sin, cos, ...), t 1-based.
-template <int K>
-__device__ __forceinline__ void store_beta(const MonitorParams &p, int64_t pix, const double (&beta)[K],
-                                           double c, bool valid) {
+template <int K, typename T>
+__device__ __forceinline__ void store_beta(const MonitorParams &p, int64_t pix, const T (&beta)[K],
+                                           T c, bool valid) {
   if (!p.out_beta) return;
   float *o = p.out_beta + pix * K;
   if (!valid) {
@@ -145,8 +181,8 @@ __device__ __forceinline__ void store_beta(const MonitorParams &p, int64_t pix, 
     for (int i = 0; i < K; ++i) o[i] = __int_as_float(0x7fc00000);
     return;
   }
-  o[0] = (float)(beta[0] - beta[1] * p.tc / p.ts + c);
-  o[1] = (float)(beta[1] / p.ts);
+  o[0] = (float)(beta[0] - beta[1] * (T)(p.tc / p.ts) + c);
+  o[1] = (float)(beta[1] / (T)p.ts);
 #pragma unroll
   for (int i = 2; i < K; ++i) o[i] = (float)beta[i];
 }
@@ -154,7 +190,7 @@ __device__ __forceinline__ void store_beta(const MonitorParams &p, int64_t pix, 
 constexpr int kUnroll = 8;
 
 template <int K>
-__global__ void __launch_bounds__(128) monitor_simt_kernel(MonitorParams p) {
+__global__ void __launch_bounds__(128, 4) monitor_simt_kernel(MonitorParams p) {
   extern __shared__ float4 smem4[];
   const int KP = p.KP;
   float *sX = reinterpret_cast<float *>(smem4);
@@ -222,27 +258,21 @@ __global__ void __launch_bounds__(128) monitor_simt_kernel(MonitorParams p) {
     }
   }
 
-  // ---------------- solve (Alg. 1 l.3-4), fp64 registers
+  // ---------------- solve (Alg. 1 l.3-4): Cholesky of the SPD Gram in
+  // fp32 registers; the factor is kept for the refinement step below
   const int h = window_h(nbar, p.hf);
   bool deg = (nbar < K + 1) || (h < 1);
-  double beta[K];
+  float beta[K];
   bool refit = false;
   {
-    double Ad[Tri<K>::kN], bd[K];
-#pragma unroll
-    for (int i = 0; i < Tri<K>::kN; ++i) Ad[i] = (double)A[i];
-#pragma unroll
-    for (int i = 0; i < K; ++i) bd[i] = (double)b[i];
-    double minratio = deg ? 1.0 : chol_solve<K>(Ad, bd, beta);
+    const float minratio = chol_factor<K, float>(A);
+    chol_solve<K, float>(A, b, beta);
+    if (!deg && !(minratio >= (float)kRefitRatio)) refit = true;
     if (deg) {
 #pragma unroll
-      for (int i = 0; i < K; ++i) beta[i] = 0.0;
+      for (int i = 0; i < K; ++i) beta[i] = 0.f;
     }
-    if (!deg && !(minratio >= kRefitRatio)) refit = true;
   }
-  float bf[K];
-#pragma unroll
-  for (int i = 0; i < K; ++i) bf[i] = (float)beta[i];
 
   // ---------------- pass 2a: history residuals r0 = y' - x'beta0, their
   // moment db = sum v r0 x (one step of iterative refinement of the fp32
@@ -251,7 +281,7 @@ __global__ void __launch_bounds__(128) monitor_simt_kernel(MonitorParams p) {
   const int hh = deg ? 1 : h;
   const int hcap = p.hcap;
   float *myring = ring + tid;
-  int *mydate = reinterpret_cast<int *>(ring + (size_t)hcap * BP) + tid;
+  int16_t *mydate = reinterpret_cast<int16_t *>(ring + (size_t)hcap * BP) + tid;
   float s2 = 0.f;
   float db[K];
 #pragma unroll
@@ -279,7 +309,7 @@ __global__ void __launch_bounds__(128) monitor_simt_kernel(MonitorParams p) {
       }
       float yhat = 0.f;
 #pragma unroll
-      for (int i = 0; i < K; ++i) yhat = fmaf(bf[i], x[i], yhat);
+      for (int i = 0; i < K; ++i) yhat = fmaf(beta[i], x[i], yhat);
       const bool v = (y == y);
       const float r = v ? (y - c0) - yhat : 0.f;
 #pragma unroll
@@ -287,45 +317,26 @@ __global__ void __launch_bounds__(128) monitor_simt_kernel(MonitorParams p) {
       s2 = fmaf(r, r, s2);
       if (v) {
         myring[ws * BP] = r;
-        mydate[ws * BP] = t;
+        mydate[ws * BP] = (int16_t)t;
         ws = (ws + 1 == hcap) ? 0 : ws + 1;
         ++cr;
       }
     }
   }
-  // refined fit beta = beta0 + A^-1 db; sigma-hat from the refined
-  // residuals: sum (r0 - x'dbeta)^2 = s2 - 2 dbeta.db + dbeta' A dbeta
+  // refined fit beta = beta0 + A^-1 db (same factor); sigma-hat of the
+  // refined residuals: sum (r0 - x'dbeta)^2 = s2 - dbeta.db (A dbeta = db)
   float sigma;
   float dbf[K];
   {
-    double Ad[Tri<K>::kN], bd[K], dbeta[K];
-#pragma unroll
-    for (int i = 0; i < Tri<K>::kN; ++i) Ad[i] = (double)A[i];
-#pragma unroll
-    for (int i = 0; i < K; ++i) bd[i] = (double)db[i];
-    if (!deg) {
-      chol_solve<K>(Ad, bd, dbeta);
-    } else {
-#pragma unroll
-      for (int i = 0; i < K; ++i) dbeta[i] = 0.0;
-    }
-    double quad = 0.0, lin = 0.0;
+    chol_solve<K, float>(A, db, dbf);
+    float lin = 0.f;
 #pragma unroll
     for (int i = 0; i < K; ++i) {
-      lin += dbeta[i] * bd[i];
-      double Ai = 0.0;
-#pragma unroll
-      for (int j = 0; j < K; ++j) Ai += Ad[i <= j ? Tri<K>::idx(i, j) : Tri<K>::idx(j, i)] * dbeta[j];
-      quad += dbeta[i] * Ai;
+      if (deg) dbf[i] = 0.f;
+      lin = fmaf(dbf[i], db[i], lin);
+      beta[i] += dbf[i];
     }
-    const double ss = fmax((double)s2 - 2.0 * lin + quad, 0.0);
-    sigma = (float)sqrt(ss / (double)(nbar - K));
-#pragma unroll
-    for (int i = 0; i < K; ++i) {
-      beta[i] += dbeta[i];
-      bf[i] = (float)beta[i];
-      dbf[i] = (float)dbeta[i];
-    }
+    sigma = sqrtf(fmaxf(s2 - lin, 0.f) / (float)(nbar - K));
   }
   if (!deg && !(sigma > 1e-4f * ymax)) deg = true;
   const float inv_scale = 1.0f / (sigma * sqrtf((float)nbar));
@@ -376,8 +387,8 @@ __global__ void __launch_bounds__(128) monitor_simt_kernel(MonitorParams p) {
 #pragma unroll
       for (int i = 0; i < K; i += 2) {
         float2 xx = *reinterpret_cast<const float2 *>(xr + i);
-        yhat = fmaf(bf[i], xx.x, yhat);
-        yhat = fmaf(bf[i + 1], xx.y, yhat);
+        yhat = fmaf(beta[i], xx.x, yhat);
+        yhat = fmaf(beta[i + 1], xx.y, yhat);
       }
       const float r = (y - c0) - yhat;
       if (y == y) {
@@ -411,7 +422,7 @@ __global__ void __launch_bounds__(128) monitor_simt_kernel(MonitorParams p) {
   if (p.out_sigma) p.out_sigma[pix] = fit_ok ? sigma : qnan;
   if (p.out_nbar) p.out_nbar[pix] = nbar;
   if (p.out_flags) p.out_flags[pix] = deg ? 1u : 0u;
-  store_beta<K>(p, pix, beta, (double)c0, fit_ok);
+  store_beta<K, float>(p, pix, beta, c0, fit_ok);
   if ((refit || tie) && fit_ok && !(nbar < K + 1)) {
     // warp-aggregated append to the fp64 refit list
     const unsigned mask = __activemask();

@@ -85,7 +85,8 @@ __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
     for (int o = 16; o; o >>= 1) ymax = fmax(ymax, __shfl_xor_sync(0xffffffffu, ymax, o));
 
     double beta[K];
-    const double minratio = chol_solve<K>(A, b, beta);
+    const double minratio = chol_factor<K, double>(A);
+    chol_solve<K, double>(A, b, beta);
     const int h = window_h(nbar, p.hf);
     bool deg = !(minratio > 1e-9);  // rank test (reading R4)
 
