@@ -1,0 +1,19 @@
+"""Hardware check of the tcgen05 / TMEM / bulk-copy primitives (csrc/sm100.cuh)
+by a standalone probe: every MMA shape the tensor-core kernel uses is
+compared with a host fp64 GEMM of the same bf16 operands."""
+import os
+import subprocess
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+HERE = os.path.dirname(os.path.abspath(__file__))
+
+
+def test_umma_probe(tmp_path):
+    exe = str(tmp_path / "umma_probe")
+    subprocess.run(["nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O2", "-std=c++17",
+                    os.path.join(HERE, "native", "umma_probe.cu"), "-o", exe], check=True)
+    r = subprocess.run([exe], capture_output=True, text=True, timeout=120)
+    print(r.stdout)
+    assert r.returncode == 0 and "ALL OK" in r.stdout, r.stdout + r.stderr
