@@ -294,7 +294,7 @@ def main():
     workload_key = f"{args.config}:P={P}:N={N}:k={rspec.k}"
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": achieved / peak, "traffic": ncu_traffic(workload_key),
-                "kernel": "monitor_simt_kernel<8>", "kernel_ms_avg": k_avg,
+                "kernel": "monitor_tc_kernel<8> (+SIMT tail)", "kernel_ms_avg": k_avg,
                 "kernel_share_of_step": k_avg / ms_step if ms_step else None,
                 "alg_bytes_per_launch": alg_bytes, "peak_source": peak_src}
 

@@ -8,6 +8,7 @@
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <memory>
 #include <mutex>
@@ -17,6 +18,7 @@
 
 #include "../../include/bfast.h"
 #include "monitor_simt.cuh"
+#include "monitor_tc.cuh"
 #include "refit_fp64.cuh"
 
 namespace {
@@ -88,6 +90,11 @@ struct bfast_plan {
   int32_t *dlist = nullptr;
   int64_t list_cap = 0;
   cudaEvent_t scratch_free = nullptr;  // orders executions sharing the refit scratch
+  // tensor-core path: per-chunk B-operand tables (monitor_tc.cuh)
+  uint8_t *dtab = nullptr;
+  size_t tab2_off = 0, tab3_off = 0;
+  int nch = 0, ncm = 0;
+  int mode = 0;  // 0 auto, 1 force SIMT, 2 force tensor cores (BFAST_KERNEL env at plan creation)
   std::mutex mu;
   ~bfast_plan() {
     int prev = -1;
@@ -97,6 +104,7 @@ struct bfast_plan {
     cudaFree(dX64);
     cudaFree(dcount);
     cudaFree(dlist);
+    cudaFree(dtab);
     if (scratch_free) cudaEventDestroy(scratch_free);
     if (prev >= 0) cudaSetDevice(prev);
   }
@@ -127,12 +135,154 @@ void build_design(const bfast_plan &pl, std::vector<float> &X, std::vector<doubl
   }
 }
 
+uint16_t bf16_rne(double v) {
+  float f = (float)v;
+  uint32_t u;
+  std::memcpy(&u, &f, 4);
+  if ((u & 0x7f800000u) == 0x7f800000u) return (uint16_t)(u >> 16);
+  u += 0x7fffu + ((u >> 16) & 1u);
+  return (uint16_t)(u >> 16);
+}
+double bf16_val(uint16_t h) {
+  uint32_t u = (uint32_t)h << 16;
+  float f;
+  std::memcpy(&f, &u, 4);
+  return (double)f;
+}
+void split2(double v, uint16_t &h, uint16_t &l) {
+  h = bf16_rne(v);
+  l = bf16_rne(v - bf16_val(h));
+}
+void split3(double v, uint16_t &h, uint16_t &m, uint16_t &l) {
+  h = bf16_rne(v);
+  m = bf16_rne(v - bf16_val(h));
+  l = bf16_rne(v - bf16_val(h) - bf16_val(m));
+}
+inline size_t kmaj(int row, int k, int rows) { return sm100::kmajor_off(row, k, rows) / 2; }
+
+// Chunk tables of the tensor-core kernel (monitor_tc.cuh): B operands in the
+// canonical K-major layout, fp64 values split into bf16 parts.
+template <int K>
+void build_tc_tables(const bfast_plan &pl, std::vector<uint16_t> &tab, size_t &off2, size_t &off3) {
+  using C = bfast::TcCfg<K>;
+  const int k = pl.k, n = pl.n, N = (int)pl.N, DC = C::DC;
+  const int nch = (n + DC - 1) / DC, ncm = (N - n + DC - 1) / DC;
+  const double two_pi = 6.283185307179586476925286766559;
+  auto xrow = [&](int t, double *x) {
+    const double tau = ((double)(t + 1) - pl.tc) / pl.ts, th = two_pi * pl.dates[t];
+    x[0] = 1.0;
+    x[1] = tau;
+    for (int j = 1; j <= k; ++j) {
+      x[2 * j] = std::sin(j * th);
+      x[2 * j + 1] = std::cos(j * th);
+    }
+  };
+  auto frow = [&](int t, double *f) {  // tau, tau^2, tau sin_j, tau cos_j, sin_m, cos_m
+    const double tau = ((double)(t + 1) - pl.tc) / pl.ts, th = two_pi * pl.dates[t];
+    f[0] = tau;
+    f[1] = tau * tau;
+    for (int j = 1; j <= k; ++j) {
+      f[2 + 2 * (j - 1)] = tau * std::sin(j * th);
+      f[3 + 2 * (j - 1)] = tau * std::cos(j * th);
+    }
+    for (int m = 1; m <= 2 * k; ++m) {
+      f[2 + 2 * k + 2 * (m - 1)] = std::sin(m * th);
+      f[3 + 2 * k + 2 * (m - 1)] = std::cos(m * th);
+    }
+  };
+  const size_t T1 = C::TAB1 / 2, T2 = C::TAB2 / 2, T3 = C::TAB3 / 2;
+  tab.assign((size_t)nch * T1 + (size_t)nch * T2 + (size_t)ncm * T3, 0);
+  off2 = (size_t)nch * T1;
+  off3 = off2 + (size_t)nch * T2;
+  double x[2 + 2 * BFAST_K_MAX_HARMONICS], f[2 + 6 * BFAST_K_MAX_HARMONICS];
+  auto put_b2 = [&](uint16_t *b2, int d, const double *xv) {  // [KB x 32], k = 2d + {yhi, ylo}
+    for (int i = 0; i < K; ++i) {
+      uint16_t h, l;
+      split2(xv[i], h, l);
+      b2[kmaj(i, 2 * d, C::KB)] = h;
+      b2[kmaj(i, 2 * d + 1, C::KB)] = h;
+      b2[kmaj(K + i, 2 * d, C::KB)] = l;
+    }
+  };
+  auto put_br = [&](uint16_t *br, int d, const double *xv) {  // [KB3 x 48], k = 3d + e
+    for (int i = 0; i < K; ++i) {
+      uint16_t h, m, l;
+      split3(xv[i], h, m, l);
+      const uint16_t blk[3] = {h, m, l};
+      for (int b = 0; b < 3; ++b)
+        for (int e = 0; e < 3; ++e) br[kmaj(b * K + i, 3 * d + e, C::KB3)] = blk[b];
+    }
+  };
+  auto put_b3 = [&](uint16_t *b3, int d, const double *xv) {  // [16 x KY]: xh|xm|xl|xh|xm|xh
+    for (int i = 0; i < K; ++i) {
+      uint16_t h, m, l;
+      split3(xv[i], h, m, l);
+      const uint16_t blk[6] = {h, m, l, h, m, h};
+      for (int b = 0; b < 6; ++b) b3[kmaj(d, b * K + i, C::DC)] = blk[b];
+    }
+  };
+  for (int c = 0; c < nch; ++c) {
+    uint16_t *b1 = tab.data() + (size_t)c * T1;
+    uint16_t *b2 = b1 + C::B1_BYTES / 2;
+    uint16_t *c2 = tab.data() + off2 + (size_t)c * T2;
+    uint16_t *c3 = c2 + C::BR_BYTES / 2;
+    for (int d = 0; d < DC; ++d) {
+      const int t = c * DC + d;
+      if (t >= n) continue;
+      xrow(t, x);
+      frow(t, f);
+      for (int q = 0; q < C::NF; ++q) {
+        uint16_t h, m, l;
+        split3(f[q], h, m, l);
+        b1[kmaj(q, d, C::NGp)] = h;
+        b1[kmaj(C::NF + q, d, C::NGp)] = m;
+        b1[kmaj(2 * C::NF + q, d, C::NGp)] = l;
+      }
+      put_b2(b2, d, x);
+      put_br(c2, d, x);
+      put_b3(c3, d, x);
+    }
+  }
+  for (int c = 0; c < ncm; ++c) {
+    uint16_t *b3 = tab.data() + off3 + (size_t)c * T3;
+    for (int d = 0; d < DC; ++d) {
+      const int t = n + c * DC + d;
+      if (t >= N) continue;
+      xrow(t, x);
+      put_b3(b3, d, x);
+    }
+  }
+}
+
+int build_tc(bfast_plan &pl) {
+  std::vector<uint16_t> tab;
+  size_t o2 = 0, o3 = 0;
+  switch (pl.k) {
+    case 0: build_tc_tables<2>(pl, tab, o2, o3); break;
+    case 1: build_tc_tables<4>(pl, tab, o2, o3); break;
+    case 2: build_tc_tables<6>(pl, tab, o2, o3); break;
+    case 3: build_tc_tables<8>(pl, tab, o2, o3); break;
+    case 4: build_tc_tables<10>(pl, tab, o2, o3); break;
+    case 5: build_tc_tables<12>(pl, tab, o2, o3); break;
+    case 6: build_tc_tables<14>(pl, tab, o2, o3); break;
+    default: return BFAST_EUNSUPPORTED;
+  }
+  pl.nch = (pl.n + 15) / 16;
+  pl.ncm = ((int)pl.N - pl.n + 15) / 16;
+  pl.tab2_off = o2 * 2;
+  pl.tab3_off = o3 * 2;
+  CUDA_TRY(cudaMalloc(&pl.dtab, tab.size() * 2));
+  CUDA_TRY(cudaMemcpy(pl.dtab, tab.data(), tab.size() * 2, cudaMemcpyHostToDevice));
+  return BFAST_OK;
+}
+
 size_t simt_smem(const bfast_plan &pl, int bp) {
   return (size_t)pl.N * pl.KP * sizeof(float) + (size_t)pl.hcap * bp * (sizeof(float) + sizeof(int16_t));
 }
 
 template <int K>
 int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t st) {
+  using TC = bfast::TcCfg<K>;
   static thread_local int configured_dev = -1;
   int bp = 128;
   while (bp > 32 && simt_smem(pl, bp) > (size_t)kMaxSmem) bp >>= 1;
@@ -143,10 +293,22 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
                                   cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmem));
     CUDA_TRY(cudaFuncSetAttribute(bfast::refit_fp64_kernel<K>,
                                   cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmem));
+    {
+      cudaFuncAttributes fa{};
+      CUDA_TRY(cudaFuncGetAttributes(&fa, bfast::monitor_tc_kernel<K>));
+      CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_tc_kernel<K>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    kMaxSmem - (int)fa.sharedSizeBytes));
+    }
     configured_dev = pl.device;
   }
-  const int64_t blocks = (prm.P + bp - 1) / bp;
-  if (blocks > 0x7fffffff) return fail(BFAST_EUNSUPPORTED, "P too large");
+  int sms = 148;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, pl.device);
+  // tensor-core path on the full 128-pixel tiles when the stack rows allow
+  // 16-byte bulk copies; SIMT kernel on the ragged tail (or everything)
+  const size_t tc_smem = TC::smem_bytes(pl.hcap);
+  const bool tc_ok = pl.dtab && pl.mode != 1 && (prm.ldY % 4) == 0 &&
+                     ((uintptr_t)(prm.Y + prm.p0) % 16) == 0 && tc_smem + 1024 <= (size_t)kMaxSmem;
+  const int64_t ntiles = tc_ok ? prm.P / 128 : 0;
   // the refit list/counter are plan scratch: order executions on any stream
   CUDA_TRY(cudaStreamWaitEvent(st, pl.scratch_free, 0));
   CUDA_TRY(cudaMemsetAsync(prm.refit_count, 0, sizeof(int32_t), st));
@@ -156,8 +318,33 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
     CUDA_TRY(cudaEventCreate(&e1));
     CUDA_TRY(cudaEventRecord(e0, st));
   }
-  bfast::monitor_simt_kernel<K><<<(unsigned)blocks, bp, smem, st>>>(prm);
-  CUDA_TRY(cudaGetLastError());
+  int launches = 0;
+  if (ntiles > 0) {
+    bfast::TcTables tb;
+    tb.tab1 = pl.dtab;
+    tb.tab2 = pl.dtab + pl.tab2_off;
+    tb.tab3 = pl.dtab + pl.tab3_off;
+    tb.nch = pl.nch;
+    tb.ncm = pl.ncm;
+    tb.ntiles = ntiles;
+    const int per_sm = (tc_smem + 1024) * 2 + 2048 <= (size_t)kMaxSmem ? 2 : 1;
+    const int64_t grid = std::min<int64_t>(ntiles, (int64_t)sms * per_sm);
+    bfast::MonitorParams q = prm;
+    bfast::monitor_tc_kernel<K><<<(unsigned)grid, 160, tc_smem, st>>>(q, tb);
+    CUDA_TRY(cudaGetLastError());
+    ++launches;
+  }
+  const int64_t rest = prm.P - ntiles * 128;
+  if (rest > 0) {
+    bfast::MonitorParams q = prm;
+    q.p0 = prm.p0 + ntiles * 128;
+    q.P = rest;
+    const int64_t blocks = (rest + bp - 1) / bp;
+    if (blocks > 0x7fffffff) return fail(BFAST_EUNSUPPORTED, "P too large");
+    bfast::monitor_simt_kernel<K><<<(unsigned)blocks, bp, smem, st>>>(q);
+    CUDA_TRY(cudaGetLastError());
+    ++launches;
+  }
   if (g_prof_on) {
     CUDA_TRY(cudaEventRecord(e1, st));
     g_prof.emplace_back(e0, e1);
@@ -166,12 +353,10 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
   const int rwarps = 4;
   const size_t rsmem = (size_t)rwarps * (pl.N + 1) * sizeof(double);
   if (rsmem > (size_t)kMaxSmem) return fail(BFAST_EUNSUPPORTED, "refit smem too large");
-  int sms = 148;
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, pl.device);
   bfast::refit_fp64_kernel<K><<<sms * 4, rwarps * 32, rsmem, st>>>(prm);
   CUDA_TRY(cudaGetLastError());
   CUDA_TRY(cudaEventRecord(pl.scratch_free, st));
-  g_launches = 2;
+  g_launches = launches + 1;
   return BFAST_OK;
 }
 
@@ -192,6 +377,11 @@ int launch(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t s
 std::mutex g_cache_mu;
 std::vector<std::unique_ptr<bfast_plan>> g_cache;
 
+int env_mode() {
+  const char *m = std::getenv("BFAST_KERNEL");
+  return !m ? 0 : (std::strcmp(m, "simt") == 0 ? 1 : std::strcmp(m, "tc") == 0 ? 2 : 0);
+}
+
 bool same_plan(const bfast_plan &pl, int dev, int64_t N, const double *dates, int32_t n, int32_t k,
                float h, float lambda) {
   return pl.device == dev && pl.N == N && pl.n == n && pl.k == k && pl.hf == h &&
@@ -202,7 +392,7 @@ int cached_plan(int dev, int64_t N, const double *dates, int32_t n, int32_t k, f
                 bfast_plan **out) {
   std::lock_guard<std::mutex> g(g_cache_mu);
   for (auto &p : g_cache)
-    if (same_plan(*p, dev, N, dates, n, k, h, lambda)) {
+    if (same_plan(*p, dev, N, dates, n, k, h, lambda) && p->mode == env_mode()) {
       *out = p.get();
       return BFAST_OK;
     }
@@ -356,6 +546,10 @@ int bfast_plan_create(bfast_plan **out, int device, int64_t N, const double *dat
                 pl->hcap);
   if ((size_t)4 * (N + 1) * sizeof(double) > (size_t)kMaxSmem)
     return fail(BFAST_EUNSUPPORTED, "N=%lld too large for the refit kernel", (long long)N);
+  {
+    const char *mode = std::getenv("BFAST_KERNEL");
+    pl->mode = !mode ? 0 : (std::strcmp(mode, "simt") == 0 ? 1 : std::strcmp(mode, "tc") == 0 ? 2 : 0);
+  }
   std::vector<float> X;
   std::vector<double> X64;
   build_design(*pl, X, X64);
@@ -370,7 +564,10 @@ int bfast_plan_create(bfast_plan **out, int device, int64_t N, const double *dat
     e = cudaMemcpy(pl->dX64, X64.data(), X64.size() * sizeof(double), cudaMemcpyHostToDevice);
   if (e == cudaSuccess) e = cudaMemset(pl->dcount, 0, sizeof(int32_t));
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&pl->scratch_free, cudaEventDisableTiming);
+  int trc = BFAST_OK;
+  if (e == cudaSuccess && pl->mode != 1 && N <= 32767) trc = build_tc(*pl);
   cudaSetDevice(prev);
+  if (trc != BFAST_OK) return trc;
   if (e != cudaSuccess)
     return fail(e == cudaErrorMemoryAllocation ? BFAST_ENOMEM : BFAST_ECUDA, "plan: %s",
                 cudaGetErrorString(e));

@@ -431,7 +431,7 @@ __global__ void __launch_bounds__(128, 4) monitor_simt_kernel(MonitorParams p) {
     int base = 0;
     if (lane == leader) base = atomicAdd(p.refit_count, __popc(mask));
     base = __shfl_sync(mask, base, leader);
-    p.refit_list[base + __popc(mask & ((1u << lane) - 1))] = (int32_t)(pix - p.p0);
+    p.refit_list[base + __popc(mask & ((1u << lane) - 1))] = (int32_t)pix;
   }
 }
 

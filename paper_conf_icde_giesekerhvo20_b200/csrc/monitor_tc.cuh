@@ -1,0 +1,567 @@
+// monitor_tc.cuh -- BFAST-Monitor hot path on the 5th-generation tensor cores.
+//
+// Same algorithm and numerics contract as monitor_simt.cuh (Algorithm 1,
+// PAPER.md L134; Fig. 12), re-mapped so that every contraction
+// shared by a 128-pixel tile runs as a tcgen05.mma with fp32 accumulators
+// in Tensor Memory, and the CUDA cores only do per-(pixel, date) scalar
+// work:
+//
+//   masked Gram  A = sum_t v_t x_t x_t^T  (Alg. 1 l.2, Fig. 4)
+//       The K(K+1)/2 entries are linear in NF = 2+6k masked moments
+//       sum_t v_t f_q(t) of the functions f = {tau, tau^2, tau sin_j,
+//       tau cos_j, sin_m, cos_m (m <= 2k)} (product-to-sum identities), so
+//       the tile's Gram is ONE bf16 GEMM: D_G[128 x 3NF] += V[128 x 16] *
+//       F[16 x 3NF] per 16 dates, with V the exact 0/1 mask and F split in
+//       hi+mid+lo bf16 (24-bit mantissa: the products are exact, so the
+//       Gram carries fp32 accumulation error only).
+//   moment b = sum_t v_t y'_t x_t  (Alg. 1 l.4): D_b += [y'hi y'lo] * [xhi xlo]
+//   yhat = X beta (Fig. 12 ker 6): D_y[128 x 16 dates] = [beta hi/mid/lo] *
+//       [x hi/mid/lo] with the 6 cross terms of a 3-way bf16 split
+//       (~24-bit accuracy, fp32 accumulate).
+//   refinement db = sum_t v_t r0_t x_t, r0 = y' - x beta0: a sum with heavy
+//       cancellation (db -> 0 as beta0 -> beta), so both r0 and x are split
+//       3-way (24-bit): D_db[128 x 3K] += [r0 hi,mid,lo per date] * [x hi|mid|lo].
+//   Because the refinement step re-solves with the residual moment, the
+//   16-bit moment only sets beta0; the final beta carries fp32-level error
+//   (DESIGN.md "Numerics").
+//
+// Roles (160 threads): warps 0-3 own one pixel per thread (TMEM lane =
+// pixel row); warp 4 is the producer, streaming 16-date chunks of the
+// time-major stack (one 512-byte bulk copy per date row) plus the chunk's
+// B-operand tables into a 3-stage ring.  Thread 0 issues the MMAs after a
+// named barrier and signals completion with tcgen05.commit on mbarriers.
+// Per tile the chunk sequence is: history (Gram+moment), history again
+// (residuals, sigma, refinement moment, MOSUM ring), monitoring (MOSUM,
+// boundary, first break, mean).  Full 128-pixel tiles only; the host runs
+// the SIMT kernel on the ragged tail.
+#pragma once
+#include "monitor_simt.cuh"
+#include "sm100.cuh"
+
+namespace bfast {
+
+template <int K>
+struct TcCfg {
+  static constexpr int k = (K - 2) / 2;
+  static constexpr int NF = 2 + 6 * k;                     // masked moment functions
+  static constexpr int NGp = ((3 * NF + 15) / 16) * 16;    // Gram GEMM N (hi, mid, lo)
+  static constexpr int KB = ((2 * K + 15) / 16) * 16;      // moment GEMM N
+  static constexpr int KY = ((6 * K + 15) / 16) * 16;      // yhat GEMM K
+  static constexpr int KB3 = ((3 * K + 15) / 16) * 16;     // refinement GEMM N (x hi|mid|lo)
+  static constexpr int DC = 16;                            // dates per chunk
+  static constexpr int COL_G = 0, COL_B = NGp, COL_DB = NGp + KB, COL_Y = NGp + KB + KB3;
+  static constexpr int COLS_USED = COL_Y + 2 * DC;
+  static constexpr int TMEM_COLS = COLS_USED <= 32 ? 32 : COLS_USED <= 64 ? 64 : COLS_USED <= 128 ? 128
+                                   : COLS_USED <= 256 ? 256 : 512;
+  static constexpr int B1_BYTES = NGp * DC * 2;            // [NGp x 16] bf16
+  static constexpr int B2_BYTES = KB * 2 * DC * 2;         // [KB x 32] bf16
+  static constexpr int B3_BYTES = DC * KY * 2;             // [16 x KY] bf16
+  static constexpr int BR_BYTES = KB3 * 3 * DC * 2;        // [KB3 x 48] bf16 (refinement)
+  static constexpr int TAB1 = B1_BYTES + B2_BYTES;         // pass 1 chunk tables
+  static constexpr int TAB2 = BR_BYTES + B3_BYTES;         // pass 2a
+  static constexpr int TAB3 = B3_BYTES;                    // pass 2b
+  static constexpr int TABMAX = TAB1 > TAB2 ? TAB1 : TAB2;
+  static constexpr int YBYTES = DC * 128 * 4;
+  static constexpr int STAGE = ((YBYTES + TABMAX + 127) / 128) * 128;
+  static constexpr int S = 3;                              // ring stages
+  static constexpr int A1_BYTES = 128 * DC * 2;
+  static constexpr int A2_BYTES = 128 * 2 * DC * 2;
+  static constexpr int A4_BYTES = 128 * 3 * DC * 2;        // r0 hi|mid|lo per date
+  static constexpr int OPBUF = A1_BYTES + A2_BYTES > A4_BYTES ? A1_BYTES + A2_BYTES : A4_BYTES;
+  static constexpr int A3_BYTES = 128 * KY * 2;
+  static constexpr size_t smem_fixed() { return (size_t)S * STAGE + 2 * OPBUF + A3_BYTES; }
+  static constexpr size_t smem_bytes(int hcap) { return smem_fixed() + (size_t)hcap * 128 * 6; }
+};
+
+struct TcTables {
+  const uint8_t *tab1, *tab2, *tab3;  // per-chunk B operands, canonical K-major layout
+  int nch, ncm;                       // history / monitoring chunks of 16 dates
+  int64_t ntiles;                     // full 128-pixel tiles
+};
+
+__device__ __forceinline__ void named_bar_sync_128() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
+
+// y split into hi and lo bf16 halves packed {lo16: hi part, hi16: lo part}
+__device__ __forceinline__ uint32_t split2_bf16(float v) {
+  const uint32_t w1 = sm100::pack_bf16x2(v, 0.f);
+  const float hi = __uint_as_float(w1 << 16);
+  return sm100::pack_bf16x2(v, v - hi);
+}
+__device__ __forceinline__ float bf16_round(float v) {
+  return __uint_as_float(sm100::pack_bf16x2(v, 0.f) << 16);
+}
+
+template <int K>
+__global__ void __launch_bounds__(160, 2) monitor_tc_kernel(MonitorParams p, TcTables tb) {
+  using C = TcCfg<K>;
+  extern __shared__ __align__(1024) uint8_t smem[];
+  __shared__ __align__(8) uint64_t full[C::S], empty[C::S], opfree[2], yfull[2], accready;
+  __shared__ uint32_t tmem_base_s;
+  uint8_t *stages = smem;
+  uint8_t *opb = stages + C::S * C::STAGE;
+  uint8_t *a3 = opb + 2 * C::OPBUF;
+  const int hcap = p.hcap;
+  float *ring = reinterpret_cast<float *>(a3 + C::A3_BYTES);
+  int16_t *rdate = reinterpret_cast<int16_t *>(ring + (size_t)hcap * 128);
+
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  if (tid == 0) {
+    for (int i = 0; i < C::S; ++i) {
+      sm100::mbar_init(&full[i], 1);
+      sm100::mbar_init(&empty[i], 1);
+    }
+    sm100::mbar_init(&opfree[0], 1);
+    sm100::mbar_init(&opfree[1], 1);
+    sm100::mbar_init(&yfull[0], 1);
+    sm100::mbar_init(&yfull[1], 1);
+    sm100::mbar_init(&accready, 1);
+    sm100::fence_mbar_init();
+  }
+  if (warp == 0) sm100::tmem_alloc(&tmem_base_s, C::TMEM_COLS);
+  sm100::tc_fence_before();
+  __syncthreads();
+  sm100::tc_fence_after();
+  const uint32_t tbase = tmem_base_s;
+  const int n = p.n, N = p.N, nch = tb.nch, ncm = tb.ncm;
+  const int64_t ldY = p.ldY;
+
+  if (warp == 4) {
+    // ------------------------------------------------------------ producer
+    if (lane == 0) {
+      const uint64_t pol_first = sm100::policy_evict_first();
+      int s = 0;
+      uint32_t ph = 0;
+      for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
+        const float *ybase = p.Y + p.p0 + tile * 128;
+        for (int phase = 0; phase < 3; ++phase) {
+          const int nc = phase < 2 ? nch : ncm;
+          const int tbeg = phase < 2 ? 0 : n, tend = phase < 2 ? n : N;
+          const uint32_t tabbytes = phase == 0 ? C::TAB1 : phase == 1 ? C::TAB2 : C::TAB3;
+          const uint8_t *tabsrc = phase == 0 ? tb.tab1 : phase == 1 ? tb.tab2 : tb.tab3;
+          for (int c = 0; c < nc; ++c) {
+            sm100::mbar_wait(&empty[s], ph ^ 1);
+            uint8_t *st = stages + s * C::STAGE;
+            const int t0 = tbeg + c * C::DC;
+            const int rows = min(C::DC, tend - t0);
+            sm100::mbar_arrive_expect_tx(&full[s], rows * 512 + tabbytes);
+            for (int d = 0; d < rows; ++d) {
+              const float *src = ybase + (int64_t)(t0 + d) * ldY;
+              if (phase == 0)
+                sm100::bulk_g2s(st + d * 512, src, 512, &full[s]);          // re-read in pass 2a
+              else
+                sm100::bulk_g2s_stream(st + d * 512, src, 512, &full[s], pol_first);  // last use
+            }
+            sm100::bulk_g2s(st + C::YBYTES, tabsrc + (size_t)c * tabbytes, tabbytes, &full[s]);
+            if (++s == C::S) {
+              s = 0;
+              ph ^= 1;
+            }
+          }
+        }
+      }
+    }
+  } else {
+    // ------------------------------------------------------------ consumers
+    const uint32_t lanebase = tbase + ((uint32_t)(32 * warp) << 16);
+    const uint32_t idG = sm100::idesc_bf16_f32(128, C::NGp);
+    const uint32_t idB = sm100::idesc_bf16_f32(128, C::KB);
+    const uint32_t idY = sm100::idesc_bf16_f32(128, C::DC);
+    const uint32_t idR = sm100::idesc_bf16_f32(128, C::KB3);
+    const float qnan = __int_as_float(0x7fc00000);
+    const uint32_t aop = sm100::smem_u32(opb), a3s = sm100::smem_u32(a3), sts = sm100::smem_u32(stages);
+    int cs = 0;
+    uint32_t cph = 0;
+    uint32_t opcnt = 0, yissue = 0, yuse = 0, acnt = 0;
+
+    auto stage_ahead = [&](int ahead, uint32_t &par) {
+      int s = cs + ahead;
+      par = cph;
+      while (s >= C::S) {
+        s -= C::S;
+        par ^= 1;
+      }
+      return s;
+    };
+    auto advance = [&]() {
+      if (++cs == C::S) {
+        cs = 0;
+        cph ^= 1;
+      }
+    };
+    // thread 0: yhat MMA for the chunk `ahead` stages ahead (table offset in stage)
+    auto issue_yhat = [&](int ahead, uint32_t tab_off) {
+      uint32_t par;
+      const int s = stage_ahead(ahead, par);
+      sm100::mbar_wait(&full[s], par);
+      sm100::tc_fence_after();
+      const uint32_t slot = yissue & 1;
+      const uint32_t b3 = sts + s * C::STAGE + C::YBYTES + tab_off;
+#pragma unroll
+      for (int q = 0; q < C::KY / 16; ++q)
+        sm100::umma_bf16(tbase + C::COL_Y + slot * C::DC, sm100::smem_desc(a3s + q * 2 * 2048, 2048, 128),
+                         sm100::smem_desc(b3 + q * 2 * 256, 256, 128), idY, q > 0);
+      sm100::umma_commit(&yfull[slot]);
+      ++yissue;
+    };
+    auto write_beta_operand = [&](const float (&bt)[K]) {
+      // A3 row = [bh | bh | bh | bm | bm | bl | 0...] (6 blocks of K, KY cols)
+      float h[K], m[K], l[K];
+#pragma unroll
+      for (int i = 0; i < K; ++i) {
+        h[i] = bf16_round(bt[i]);
+        m[i] = bf16_round(bt[i] - h[i]);
+        l[i] = bt[i] - h[i] - m[i];
+      }
+      uint32_t w[C::KY / 2];
+#pragma unroll
+      for (int j = 0; j < C::KY / 2; ++j) {
+        float e[2];
+#pragma unroll
+        for (int u = 0; u < 2; ++u) {
+          const int col = 2 * j + u, blk = col / K, i = col % K;
+          e[u] = col >= 6 * K ? 0.f : (blk < 3 ? h[i] : blk < 5 ? m[i] : l[i]);
+        }
+        w[j] = sm100::pack_bf16x2(e[0], e[1]);
+      }
+#pragma unroll
+      for (int q = 0; q < C::KY / 8; ++q)
+        *reinterpret_cast<uint4 *>(a3 + sm100::kmajor_off(tid, 8 * q, 128)) =
+            make_uint4(w[4 * q], w[4 * q + 1], w[4 * q + 2], w[4 * q + 3]);
+    };
+
+    for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
+      const int64_t pix = p.p0 + tile * 128 + tid;
+      // ================= pass 1: masked Gram + moment on the tensor cores
+      int nbar = 0;
+      float c0 = 0.f, ymax = 0.f;
+      bool have = false;
+      for (int c = 0; c < nch; ++c) {
+        sm100::mbar_wait(&full[cs], cph);
+        const uint32_t ob = opcnt & 1;
+        sm100::mbar_wait(&opfree[ob], ((opcnt >> 1) & 1) ^ 1);
+        const float *Ys = reinterpret_cast<const float *>(stages + cs * C::STAGE);
+        uint32_t mw[C::DC / 2], yw[C::DC];
+#pragma unroll
+        for (int d = 0; d < C::DC; ++d) {
+          const int t = c * C::DC + d;
+          const float y = t < n ? Ys[d * 128 + tid] : qnan;
+          const bool v = (y == y);
+          if (v && !have) {
+            c0 = y;
+            have = true;
+          }
+          ymax = v ? fmaxf(ymax, fabsf(y)) : ymax;
+          nbar += v ? 1 : 0;
+          const float yp = v ? y - c0 : 0.f;
+          yw[d] = split2_bf16(yp);
+          const uint32_t mb = v ? 0x3F80u : 0u;
+          if (d & 1)
+            mw[d >> 1] |= mb << 16;
+          else
+            mw[d >> 1] = mb;
+        }
+        uint8_t *A1 = opb + ob * C::OPBUF;
+        uint8_t *A2 = A1 + C::A1_BYTES;
+        *reinterpret_cast<uint4 *>(A1 + sm100::kmajor_off(tid, 0, 128)) = make_uint4(mw[0], mw[1], mw[2], mw[3]);
+        *reinterpret_cast<uint4 *>(A1 + sm100::kmajor_off(tid, 8, 128)) = make_uint4(mw[4], mw[5], mw[6], mw[7]);
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          *reinterpret_cast<uint4 *>(A2 + sm100::kmajor_off(tid, 8 * q, 128)) =
+              make_uint4(yw[4 * q], yw[4 * q + 1], yw[4 * q + 2], yw[4 * q + 3]);
+        sm100::fence_proxy_async_smem();
+        named_bar_sync_128();
+        if (tid == 0) {
+          sm100::tc_fence_after();
+          const uint32_t a1 = aop + ob * C::OPBUF, a2 = a1 + C::A1_BYTES;
+          const uint32_t b1 = sts + cs * C::STAGE + C::YBYTES, b2 = b1 + C::B1_BYTES;
+          sm100::umma_bf16(tbase + C::COL_G, sm100::smem_desc(a1, 2048, 128),
+                           sm100::smem_desc(b1, C::NGp * 16, 128), idG, c > 0);
+#pragma unroll
+          for (int q = 0; q < 2; ++q)
+            sm100::umma_bf16(tbase + C::COL_B, sm100::smem_desc(a2 + q * 2 * 2048, 2048, 128),
+                             sm100::smem_desc(b2 + q * 2 * C::KB * 16, C::KB * 16, 128), idB, (c > 0 || q > 0));
+          sm100::umma_commit(&opfree[ob]);
+          sm100::umma_commit(&empty[cs]);
+          if (c == nch - 1) sm100::umma_commit(&accready);
+        }
+        ++opcnt;
+        advance();
+      }
+      sm100::mbar_wait(&accready, acnt & 1);
+      ++acnt;
+      sm100::tc_fence_after();
+
+      // ================= solve (Alg. 1 l.3-4): Gram from the masked moments
+      float A[Tri<K>::kN], b[K];
+      {
+        float F[C::NGp];
+#pragma unroll
+        for (int q = 0; q < C::NGp / 16; ++q) {
+          float v16[16];
+          sm100::tmem_ld16(lanebase + C::COL_G + 16 * q, v16);
+          sm100::tmem_ld_wait();
+#pragma unroll
+          for (int i = 0; i < 16; ++i)
+            F[16 * q + i] = v16[i];
+        }
+        float Bm[C::KB];
+#pragma unroll
+        for (int q = 0; q < C::KB / 16; ++q) {
+          float v16[16];
+          sm100::tmem_ld16(lanebase + C::COL_B + 16 * q, v16);
+          sm100::tmem_ld_wait();
+#pragma unroll
+          for (int i = 0; i < 16; ++i) Bm[16 * q + i] = v16[i];
+        }
+        float G[C::NF];
+#pragma unroll
+        for (int q = 0; q < C::NF; ++q) G[q] = F[q] + F[C::NF + q] + F[2 * C::NF + q];
+#pragma unroll
+        for (int i = 0; i < K; ++i) b[i] = Bm[i] + Bm[K + i];
+        const float nb = (float)nbar;
+        auto Cf = [&](int m) -> float { return m == 0 ? nb : G[2 + 2 * C::k + 2 * ((m < 0 ? -m : m) - 1) + 1]; };
+        auto Sf = [&](int m) -> float {
+          return m == 0 ? 0.f : (m < 0 ? -G[2 + 2 * C::k + 2 * (-m - 1)] : G[2 + 2 * C::k + 2 * (m - 1)]);
+        };
+        A[Tri<K>::idx(0, 0)] = nb;
+        A[Tri<K>::idx(0, 1)] = G[0];
+        A[Tri<K>::idx(1, 1)] = G[1];
+#pragma unroll
+        for (int j = 1; j <= C::k; ++j) {
+          A[Tri<K>::idx(0, 2 * j)] = Sf(j);
+          A[Tri<K>::idx(0, 2 * j + 1)] = Cf(j);
+          A[Tri<K>::idx(1, 2 * j)] = G[2 + 2 * (j - 1)];
+          A[Tri<K>::idx(1, 2 * j + 1)] = G[3 + 2 * (j - 1)];
+#pragma unroll
+          for (int jb = j; jb <= C::k; ++jb) {
+            A[Tri<K>::idx(2 * j, 2 * jb)] = 0.5f * (Cf(j - jb) - Cf(j + jb));          // s_j s_jb
+            A[Tri<K>::idx(2 * j + 1, 2 * jb + 1)] = 0.5f * (Cf(j - jb) + Cf(j + jb));  // c_j c_jb
+            A[Tri<K>::idx(2 * j, 2 * jb + 1)] = 0.5f * (Sf(j + jb) + Sf(j - jb));      // s_j c_jb
+            if (jb > j) A[Tri<K>::idx(2 * j + 1, 2 * jb)] = 0.5f * (Sf(jb + j) + Sf(jb - j));  // c_j s_jb
+          }
+        }
+      }
+      const int h = window_h(nbar, p.hf);
+      bool deg = (nbar < K + 1) || (h < 1);
+      float beta[K];
+      bool refit = false;
+      {
+        const float minratio = chol_factor<K, float>(A);
+        chol_solve<K, float>(A, b, beta);
+        if (!deg && !(minratio >= (float)kRefitRatio)) refit = true;
+        if (deg) {
+#pragma unroll
+          for (int i = 0; i < K; ++i) beta[i] = 0.f;
+        }
+      }
+      write_beta_operand(beta);
+      sm100::fence_proxy_async_smem();
+      sm100::tc_fence_before();
+      named_bar_sync_128();
+      if (tid == 0) {
+        sm100::tc_fence_after();
+        for (int a = 0; a < 2 && a < nch; ++a) issue_yhat(a, C::BR_BYTES);
+      }
+
+      // ================= pass 2a: residuals r0, sigma, refinement moment, ring
+      const int hh = deg ? 1 : h;
+      float s2 = 0.f;
+      int cr = 0, ws = 0;
+      for (int c = 0; c < nch; ++c) {
+        sm100::mbar_wait(&full[cs], cph);
+        sm100::mbar_wait(&yfull[yuse & 1], (yuse >> 1) & 1);
+        sm100::tc_fence_after();
+        float yh[16];
+        sm100::tmem_ld16(lanebase + C::COL_Y + (yuse & 1) * C::DC, yh);
+        sm100::tmem_ld_wait();
+        ++yuse;
+        const uint32_t ob = opcnt & 1;
+        sm100::mbar_wait(&opfree[ob], ((opcnt >> 1) & 1) ^ 1);
+        const float *Ys = reinterpret_cast<const float *>(stages + cs * C::STAGE);
+        float rs3[3 * C::DC];
+#pragma unroll
+        for (int d = 0; d < C::DC; ++d) {
+          const int t = c * C::DC + d;
+          const float y = t < n ? Ys[d * 128 + tid] : qnan;
+          const bool v = (y == y);
+          const float r = v ? (y - c0) - yh[d] : 0.f;
+          s2 = fmaf(r, r, s2);
+          const float rh = bf16_round(r), rm = bf16_round(r - rh);
+          rs3[3 * d] = rh;
+          rs3[3 * d + 1] = rm;
+          rs3[3 * d + 2] = (r - rh) - rm;
+          if (v) {
+            ring[ws * 128 + tid] = r;
+            rdate[ws * 128 + tid] = (int16_t)t;
+            ws = (ws + 1 == hcap) ? 0 : ws + 1;
+            ++cr;
+          }
+        }
+        uint8_t *A4 = opb + ob * C::OPBUF;
+#pragma unroll
+        for (int q = 0; q < 3 * C::DC / 8; ++q) {
+          uint32_t w[4];
+#pragma unroll
+          for (int u = 0; u < 4; ++u) w[u] = sm100::pack_bf16x2(rs3[8 * q + 2 * u], rs3[8 * q + 2 * u + 1]);
+          *reinterpret_cast<uint4 *>(A4 + sm100::kmajor_off(tid, 8 * q, 128)) = make_uint4(w[0], w[1], w[2], w[3]);
+        }
+        sm100::fence_proxy_async_smem();
+        sm100::tc_fence_before();
+        named_bar_sync_128();
+        if (tid == 0) {
+          sm100::tc_fence_after();
+          const uint32_t a4 = aop + ob * C::OPBUF;
+          const uint32_t br = sts + cs * C::STAGE + C::YBYTES;
+#pragma unroll
+          for (int q = 0; q < 3; ++q)
+            sm100::umma_bf16(tbase + C::COL_DB, sm100::smem_desc(a4 + q * 2 * 2048, 2048, 128),
+                             sm100::smem_desc(br + q * 2 * C::KB3 * 16, C::KB3 * 16, 128), idR, (c > 0 || q > 0));
+          sm100::umma_commit(&opfree[ob]);
+          if (c + 2 < nch) issue_yhat(2, C::BR_BYTES);
+          sm100::umma_commit(&empty[cs]);
+          if (c == nch - 1) sm100::umma_commit(&accready);
+        }
+        ++opcnt;
+        advance();
+      }
+      sm100::mbar_wait(&accready, acnt & 1);
+      ++acnt;
+      sm100::tc_fence_after();
+
+      // ================= refinement: beta = beta0 + A^-1 db; sigma-hat
+      float sigma, dbf[K];
+      {
+        float db[K], Dd[C::KB3];
+#pragma unroll
+        for (int q = 0; q < C::KB3 / 16; ++q) {
+          float v16[16];
+          sm100::tmem_ld16(lanebase + C::COL_DB + 16 * q, v16);
+          sm100::tmem_ld_wait();
+#pragma unroll
+          for (int i = 0; i < 16; ++i) Dd[16 * q + i] = v16[i];
+        }
+#pragma unroll
+        for (int i = 0; i < K; ++i) db[i] = Dd[i] + Dd[K + i] + Dd[2 * K + i];
+        chol_solve<K, float>(A, db, dbf);
+        float lin = 0.f;
+#pragma unroll
+        for (int i = 0; i < K; ++i) {
+          if (deg) dbf[i] = 0.f;
+          lin = fmaf(dbf[i], db[i], lin);
+          beta[i] += dbf[i];
+        }
+        sigma = sqrtf(fmaxf(s2 - lin, 0.f) / (float)(nbar - K));
+      }
+      if (!deg && !(sigma > 1e-4f * ymax)) deg = true;
+      const float inv_scale = 1.0f / (sigma * sqrtf((float)nbar));
+      write_beta_operand(beta);
+      sm100::fence_proxy_async_smem();
+      sm100::tc_fence_before();
+      named_bar_sync_128();
+      if (tid == 0) {
+        sm100::tc_fence_after();
+        for (int a = 0; a < 2 && a < ncm; ++a) issue_yhat(a, 0);
+      }
+      // MOSUM seed (m^fst, L518): the last h-1 history residuals, corrected
+      // to the refined fit
+      float W = 0.f;
+      {
+        const int nseed = deg ? 0 : hh - 1;
+        int slot = ws - nseed;
+        slot += (slot < 0) ? hcap : 0;
+        for (int q = 0; q < nseed; ++q) {
+          const int t = rdate[slot * 128 + tid];
+          const float *xr = p.X + (size_t)t * p.KP;
+          float corr = 0.f;
+#pragma unroll
+          for (int i = 0; i < K; i += 2) {
+            const float2 xx = __ldg(reinterpret_cast<const float2 *>(xr + i));
+            corr = fmaf(dbf[i], xx.x, corr);
+            corr = fmaf(dbf[i + 1], xx.y, corr);
+          }
+          const float r = ring[slot * 128 + tid] - corr;
+          ring[slot * 128 + tid] = r;
+          W += r;
+          slot = (slot + 1 == hcap) ? 0 : slot + 1;
+        }
+      }
+
+      // ================= pass 2b: monitoring (Alg. 1 l.6-12, Fig. 12 ker 9-10)
+      float msum = 0.f;
+      int brk = -1;
+      bool tie = false;
+      const float lam = p.lambda, lam_lo = lam * (1.0f - kTieTol);
+      for (int c = 0; c < ncm; ++c) {
+        sm100::mbar_wait(&full[cs], cph);
+        sm100::mbar_wait(&yfull[yuse & 1], (yuse >> 1) & 1);
+        sm100::tc_fence_after();
+        float yh[16];
+        sm100::tmem_ld16(lanebase + C::COL_Y + (yuse & 1) * C::DC, yh);
+        sm100::tmem_ld_wait();
+        ++yuse;
+        const float *Ys = reinterpret_cast<const float *>(stages + cs * C::STAGE);
+#pragma unroll
+        for (int d = 0; d < C::DC; ++d) {
+          const int t = n + c * C::DC + d;
+          const float y = t < N ? Ys[d * 128 + tid] : qnan;
+          if (y == y) {
+            const float r = (y - c0) - yh[d];
+            if (cr > nbar) {  // j >= 1: the window drops rank cr - h
+              int rs = ws - hh;
+              rs += (rs < 0) ? hcap : 0;
+              W -= ring[rs * 128 + tid];
+            }
+            W += r;
+            ring[ws * 128 + tid] = r;
+            ws = (ws + 1 == hcap) ? 0 : ws + 1;
+            const float m = W * inv_scale;
+            msum += m;
+            if (brk < 0 && fabsf(m) > lam_lo) {
+              const float B = boundary_f32(lam, cr + 1, nbar);
+              const float am = fabsf(m);
+              tie |= fabsf(am - B) <= kTieTol * B;
+              if (am > B) brk = t - n;
+            }
+            ++cr;
+          }
+        }
+        sm100::tc_fence_before();
+        named_bar_sync_128();
+        if (tid == 0) {
+          sm100::tc_fence_after();
+          if (c + 2 < ncm) issue_yhat(2, 0);
+          sm100::mbar_arrive(&empty[cs]);
+        }
+        advance();
+      }
+      const int Nbar = cr;
+      if (Nbar - nbar < 1) deg = true;
+
+      // ================= epilogue
+      const bool fit_ok = !((nbar < K + 1) || (h < 1) || (Nbar - nbar < 1));
+      p.out_break[pix] = deg ? -2 : brk;
+      p.out_mag[pix] = deg ? qnan : msum / (float)(Nbar - nbar);
+      if (p.out_sigma) p.out_sigma[pix] = fit_ok ? sigma : qnan;
+      if (p.out_nbar) p.out_nbar[pix] = nbar;
+      if (p.out_flags) p.out_flags[pix] = deg ? 1u : 0u;
+      store_beta<K, float>(p, pix, beta, c0, fit_ok);
+      const bool want = (refit || tie) && fit_ok;
+      const unsigned mask = __ballot_sync(0xffffffffu, want);
+      if (want) {
+        const int leader = __ffs(mask) - 1;
+        int base = 0;
+        if (lane == leader) base = atomicAdd(p.refit_count, __popc(mask));
+        base = __shfl_sync(mask, base, leader);
+        p.refit_list[base + __popc(mask & ((1u << lane) - 1))] = (int32_t)pix;
+      }
+    }
+  }
+  sm100::tc_fence_before();
+  __syncthreads();
+  if (warp == 0) {
+    sm100::tc_fence_after();
+    sm100::tmem_dealloc(tbase, C::TMEM_COLS);
+  }
+}
+
+}  // namespace bfast

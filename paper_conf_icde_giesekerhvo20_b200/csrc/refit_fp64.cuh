@@ -39,7 +39,7 @@ __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
   const double qnan = __longlong_as_double(0x7ff8000000000000ll);
 
   for (int item = blockIdx.x * wpb + wib; item < count; item += gridDim.x * wpb) {
-    const int64_t pix = p.p0 + p.refit_list[item];
+    const int64_t pix = p.refit_list[item];  // absolute pixel index
     const float *ycol = p.Y + pix;
     // ---- history: offset, Gram, moment (fp64)
     double A[Tri<K>::kN], b[K];

@@ -21,6 +21,14 @@ pytestmark = pytest.mark.gpu
 DEV = "cuda:0"
 
 
+@pytest.fixture(params=["tc", "simt"])
+def mode(request, monkeypatch):
+    """Run the test on the tensor-core path (full 128-pixel tiles; the SIMT
+    kernel takes the ragged tail) and on the SIMT-only path."""
+    monkeypatch.setenv("BFAST_KERNEL", request.param)
+    return request.param
+
+
 def _run_both(Y, dates, n, k, hf, lam, P=None):
     out = binding.bfast_monitor_ex(Y, dates, n, k, hf, lam, P=P, diagnostics=True)
     torch.cuda.synchronize()
@@ -39,7 +47,7 @@ def _assert_parity(gpu, orc, dates, n, k, **kw):
     return rep
 
 
-def test_tiny_config_full_parity():
+def test_tiny_config_full_parity(mode):
     spec = synth.CONFIGS["tiny"]
     Y, dates = synth.generate(spec, DEV)
     gpu, orc = _run_both(Y, dates, spec.n_hist, spec.k, spec.hf, spec.lam)
@@ -49,8 +57,8 @@ def test_tiny_config_full_parity():
     np.testing.assert_allclose(gpu["sigma"][ok], orc["sigma"][ok], rtol=1e-4)
 
 
-@pytest.mark.parametrize("P,ldY", [(1000, 1000), (1000, 1003), (129, 132), (1, 1), (31, 64)])
-def test_ragged_tails_and_leading_dimension(P, ldY):
+@pytest.mark.parametrize("P,ldY", [(1000, 1000), (1000, 1003), (1000, 1004), (129, 132), (1, 1), (31, 64), (384, 384)])
+def test_ragged_tails_and_leading_dimension(P, ldY, mode):
     spec = synth.StackSpec(P=P, N=150, n_hist=75, miss=0.45, seed=11 + P)
     Y, dates = synth.generate(spec, DEV, ldY=ldY)
     gpu, orc = _run_both(Y, dates, spec.n_hist, spec.k, spec.hf, spec.lam, P=P)
@@ -58,7 +66,7 @@ def test_ragged_tails_and_leading_dimension(P, ldY):
 
 
 @pytest.mark.parametrize("k", [0, 1, 2, 3, 4, 5, 6])
-def test_all_harmonic_orders(k):
+def test_all_harmonic_orders(k, mode):
     spec = synth.StackSpec(P=2048, N=240, n_hist=120, k=k, miss=0.4, seed=20 + k)
     Y, dates = synth.generate(spec, DEV)
     gpu, orc = _run_both(Y, dates, spec.n_hist, k, spec.hf, spec.lam)
@@ -66,7 +74,7 @@ def test_all_harmonic_orders(k):
 
 
 @pytest.mark.parametrize("hf,lam", [(1.0, 1.65), (0.7, 1.0), (0.05, 3.0), (0.5, 0.25)])
-def test_window_and_boundary_variants(hf, lam):
+def test_window_and_boundary_variants(hf, lam, mode):
     spec = synth.StackSpec(P=2048, N=200, n_hist=60, miss=0.3, seed=31)
     Y, dates = synth.generate(spec, DEV)
     gpu, orc = _run_both(Y, dates, spec.n_hist, spec.k, hf, lam)
@@ -76,7 +84,7 @@ def test_window_and_boundary_variants(hf, lam):
 @pytest.mark.parametrize("N", [100, 250, 500, 1000])
 @pytest.mark.parametrize("miss", [0.1, 0.5, 0.9])
 @pytest.mark.parametrize("k", [1, 3, 5])
-def test_sweep_shapes(N, miss, k):
+def test_sweep_shapes(N, miss, k, mode):
     """configs[2] shapes at a reduced pixel count (full size: sampled test below)."""
     idx = [100, 250, 500, 1000].index(N) * 9 + [0.1, 0.5, 0.9].index(miss) * 3 + [1, 3, 5].index(k)
     spec = synth.sweep_spec(N, miss, k, P=4096, index=idx)
@@ -85,7 +93,7 @@ def test_sweep_shapes(N, miss, k):
     _assert_parity(gpu, orc, dates, spec.n_hist, k)
 
 
-def test_edge_cases_degenerate_pixels():
+def test_edge_cases_degenerate_pixels(mode):
     N, n, k = 92, 46, 1
     dates = synth.make_dates(N)
     rng = np.random.default_rng(5)
@@ -99,7 +107,7 @@ def test_edge_cases_degenerate_pixels():
     cols.append(base.copy())                                    # no NaN at all
     cols.append(np.full(N, 0.25, np.float32))                   # constant: sigma = 0
     y = base.copy(); y[n:] -= 1.0; cols.append(y)               # break at the first date
-    Y = torch.tensor(np.stack(cols, 1), device=DEV).contiguous()
+    Y = torch.tensor(np.stack(cols * 32, 1), device=DEV).contiguous()   # 256 px: two full tiles
     gpu, orc = _run_both(Y, dates, n, k, 0.25, 1.65)
     _assert_parity(gpu, orc, dates, n, k)
     assert list(gpu["break"][:4]) == [-2, -2, gpu["break"][2], -2]
@@ -145,7 +153,7 @@ def test_host_path_and_multi_match_device_path():
     np.testing.assert_array_equal(m2, m)
 
 
-def test_plan_execute_is_deterministic_and_stream_ordered():
+def test_plan_execute_is_deterministic_and_stream_ordered(mode):
     spec = synth.StackSpec(P=50_000, N=200, n_hist=100, miss=0.6, mask="cloud", seed=51)
     Y, dates = synth.generate(spec, DEV)
     plan = binding.Plan(0, spec.N, dates, spec.n_hist, spec.k, spec.hf, spec.lam)
@@ -160,7 +168,7 @@ def test_plan_execute_is_deterministic_and_stream_ordered():
 
 
 @pytest.mark.slow
-def test_landsat_full_size_sampled_parity():
+def test_landsat_full_size_sampled_parity(mode):
     """configs[1] at full size (P = 4096^2, N = 400, 60% cloud-masked), in the
     launch configuration bench.py times (Plan.execute on one stream), with
     2^16 sampled pixels checked against the oracle and all-pixel properties."""
@@ -183,3 +191,22 @@ def test_landsat_full_size_sampled_parity():
     assert rep["breaks_oracle"] > 0.05 * len(idx)
     del Y
     torch.cuda.empty_cache()
+
+
+def test_tc_and_simt_paths_agree_closely(monkeypatch):
+    """The two kernels compute the same definitions with different fp32
+    contraction orders: breaks equal up to near ties, magnitudes within the
+    parity tolerance of each other."""
+    spec = synth.StackSpec(P=8192, N=300, n_hist=150, miss=0.5, seed=61)
+    Y, dates = synth.generate(spec, DEV)
+    outs = {}
+    for m in ("tc", "simt"):
+        monkeypatch.setenv("BFAST_KERNEL", m)
+        o = binding.bfast_monitor_ex(Y, dates, spec.n_hist, spec.k, spec.hf, spec.lam, diagnostics=True)
+        torch.cuda.synchronize()
+        outs[m] = {key: v.cpu().numpy() for key, v in o.items() if hasattr(v, "cpu")}
+    a, b = outs["tc"], outs["simt"]
+    assert (a["break"] != b["break"]).mean() < 1e-3
+    ok = (a["break"] != -2) & (b["break"] != -2)
+    d = np.abs(a["magnitude"][ok] - b["magnitude"][ok]) / np.maximum(1, np.abs(b["magnitude"][ok]))
+    assert d.max() < 1e-4
