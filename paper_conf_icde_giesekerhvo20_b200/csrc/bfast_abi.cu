@@ -2,6 +2,7 @@
 // (design matrix in fp64 -> fp32 device constants), kernel launches, the
 // host-buffer (end-to-end) path and the multi-device shard driver.
 // Declarations and contracts: include/bfast.h.
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -133,6 +134,38 @@ void build_design(const bfast_plan &pl, std::vector<float> &X, std::vector<doubl
       X64[(size_t)t * pl.K + i] = row[i];
     }
   }
+}
+
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no
+// link-time dependency on libcuda).
+typedef CUresult (*PFN_encodeTiled)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                    const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                                    CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+PFN_encodeTiled get_encode() {
+  static PFN_encodeTiled fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, []() {
+    void *f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = (PFN_encodeTiled)f;
+  });
+  return fn;
+}
+
+// Tensor map of the stack range [p0, p0+P) x [0, N): box 128 px x 16 dates,
+// out-of-bounds elements read as NaN (= missing).
+bool make_stack_map(CUtensorMap *m, const float *Y, int64_t ldY, int64_t P, int64_t N) {
+  PFN_encodeTiled enc = get_encode();
+  if (!enc) return false;
+  cuuint64_t dims[2] = {(cuuint64_t)P, (cuuint64_t)N};
+  cuuint64_t strides[1] = {(cuuint64_t)ldY * sizeof(float)};
+  cuuint32_t box[2] = {128, 16};
+  cuuint32_t es[2] = {1, 1};
+  return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void *)Y, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+             CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NAN_REQUEST_ZERO_FMA) == CUDA_SUCCESS;
 }
 
 uint16_t bf16_rne(double v) {
@@ -308,7 +341,9 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
   const size_t tc_smem = TC::smem_bytes(pl.hcap);
   const bool tc_ok = pl.dtab && pl.mode != 1 && (prm.ldY % 4) == 0 &&
                      ((uintptr_t)(prm.Y + prm.p0) % 16) == 0 && tc_smem + 1024 <= (size_t)kMaxSmem;
-  const int64_t ntiles = tc_ok ? prm.P / 128 : 0;
+  CUtensorMap ymap;
+  const bool tma_ok = tc_ok && make_stack_map(&ymap, prm.Y + prm.p0, prm.ldY, prm.P, pl.N);
+  const int64_t ntiles = tma_ok ? (prm.P + 127) / 128 : 0;
   // the refit list/counter are plan scratch: order executions on any stream
   CUDA_TRY(cudaStreamWaitEvent(st, pl.scratch_free, 0));
   CUDA_TRY(cudaMemsetAsync(prm.refit_count, 0, sizeof(int32_t), st));
@@ -330,11 +365,11 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
     const int per_sm = (tc_smem + 1024) * 2 + 2048 <= (size_t)kMaxSmem ? 2 : 1;
     const int64_t grid = std::min<int64_t>(ntiles, (int64_t)sms * per_sm);
     bfast::MonitorParams q = prm;
-    bfast::monitor_tc_kernel<K><<<(unsigned)grid, 160, tc_smem, st>>>(q, tb);
+    bfast::monitor_tc_kernel<K><<<(unsigned)grid, 160, tc_smem, st>>>(q, tb, ymap);
     CUDA_TRY(cudaGetLastError());
     ++launches;
   }
-  const int64_t rest = prm.P - ntiles * 128;
+  const int64_t rest = ntiles > 0 ? 0 : prm.P;
   if (rest > 0) {
     bfast::MonitorParams q = prm;
     q.p0 = prm.p0 + ntiles * 128;

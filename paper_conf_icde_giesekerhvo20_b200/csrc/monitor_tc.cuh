@@ -26,17 +26,21 @@
 //   (DESIGN.md "Numerics").
 //
 // Roles (160 threads): warps 0-3 own one pixel per thread (TMEM lane =
-// pixel row); warp 4 is the producer, streaming 16-date chunks of the
-// time-major stack (one 512-byte bulk copy per date row) plus the chunk's
-// B-operand tables into a 3-stage ring.  Thread 0 issues the MMAs after a
+// pixel row); warp 4 is the producer, streaming 16-date x 128-pixel boxes of
+// the time-major stack (one 2-D TMA copy each) into a 4-stage ring that the
+// consumers release as soon as they have read a box, and the chunk's
+// B-operand tables (one 1-D bulk copy each, L2-resident) into a 3-stage ring
+// released by tcgen05.commit of the MMAs that read them.  Thread 0 issues the MMAs after a
 // named barrier and signals completion with tcgen05.commit on mbarriers.
 // Per tile the chunk sequence is: history (Gram+moment), history again
 // (residuals, sigma, refinement moment, MOSUM ring), monitoring (MOSUM,
-// boundary, first break, mean).  Full 128-pixel tiles only; the host runs
-// the SIMT kernel on the ragged tail.
+// boundary, first break, mean).  The stack is read through a 2-D TMA tensor
+// map whose out-of-bounds fill is NaN, so a ragged last tile needs no
+// special case (its missing pixels are "all missing").
 #pragma once
 #include "monitor_simt.cuh"
 #include "sm100.cuh"
+#include <cuda.h>
 
 namespace bfast {
 
@@ -61,25 +65,55 @@ struct TcCfg {
   static constexpr int TAB2 = BR_BYTES + B3_BYTES;         // pass 2a
   static constexpr int TAB3 = B3_BYTES;                    // pass 2b
   static constexpr int TABMAX = TAB1 > TAB2 ? TAB1 : TAB2;
-  static constexpr int YBYTES = DC * 128 * 4;
-  static constexpr int STAGE = ((YBYTES + TABMAX + 127) / 128) * 128;
-  static constexpr int S = 3;                              // ring stages
+  static constexpr int YBYTES = DC * 128 * 4;             // one [16 dates x 128 px] box
+  static constexpr int TSTAGE = ((TABMAX + 127) / 128) * 128;
+  static constexpr int SY = 4;                             // stack ring stages (released on read)
+  static constexpr int ST = 3;                             // table ring stages (released by MMA commit)
   static constexpr int A1_BYTES = 128 * DC * 2;
   static constexpr int A2_BYTES = 128 * 2 * DC * 2;
   static constexpr int A4_BYTES = 128 * 3 * DC * 2;        // r0 hi|mid|lo per date
   static constexpr int OPBUF = A1_BYTES + A2_BYTES > A4_BYTES ? A1_BYTES + A2_BYTES : A4_BYTES;
   static constexpr int A3_BYTES = 128 * KY * 2;
-  static constexpr size_t smem_fixed() { return (size_t)S * STAGE + 2 * OPBUF + A3_BYTES; }
-  static constexpr size_t smem_bytes(int hcap) { return smem_fixed() + (size_t)hcap * 128 * 6; }
+  static constexpr int RSLOT = 128 * 4 + 128 * 2;         // ring slot: 128 residuals + 128 dates
+  static constexpr size_t smem_fixed() { return (size_t)SY * YBYTES + (size_t)ST * TSTAGE + OPBUF + A3_BYTES; }
+  static constexpr size_t smem_bytes(int hcap) { return smem_fixed() + (size_t)hcap * RSLOT; }
 };
 
 struct TcTables {
   const uint8_t *tab1, *tab2, *tab3;  // per-chunk B operands, canonical K-major layout
   int nch, ncm;                       // history / monitoring chunks of 16 dates
-  int64_t ntiles;                     // full 128-pixel tiles
+  int64_t ntiles;                     // 128-pixel tiles (the last may be ragged)
 };
 
 __device__ __forceinline__ void named_bar_sync_128() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
+__device__ __forceinline__ void sts_f32(uint32_t a, float v) {
+  asm volatile("st.shared.f32 [%0], %1;" ::"r"(a), "f"(v) : "memory");
+}
+__device__ __forceinline__ void sts_u16(uint32_t a, uint16_t v) {
+  asm volatile("st.shared.u16 [%0], %1;" ::"r"(a), "h"(v) : "memory");
+}
+__device__ __forceinline__ float lds_f32(uint32_t a) {
+  float v;
+  asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ int lds_u16(uint32_t a) {
+  uint16_t v;
+  asm volatile("ld.shared.u16 %0, [%1];" : "=h"(v) : "r"(a) : "memory");
+  return v;
+}
+// producer-side wait with back-off so a waiting producer does not steal
+// issue slots from the consumer warps of its SM sub-partition
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t *bar, uint32_t parity) {
+  while (!sm100::mbar_try_wait(bar, parity)) __nanosleep(64);
+}
+// the rare branch of the boundary test (Alg. 1 l.10-12), kept out of line
+__device__ __noinline__ void boundary_rare(float m, int rank1, int nbar, float lam, int off, int &brk, int &tie) {
+  const float B = boundary_f32(lam, rank1, nbar);
+  const float am = fabsf(m);
+  tie |= fabsf(am - B) <= kTieTol * B;
+  if (am > B) brk = off;
+}
 
 // y split into hi and lo bf16 halves packed {lo16: hi part, hi16: lo part}
 __device__ __forceinline__ uint32_t split2_bf16(float v) {
@@ -92,28 +126,33 @@ __device__ __forceinline__ float bf16_round(float v) {
 }
 
 template <int K>
-__global__ void __launch_bounds__(160, 2) monitor_tc_kernel(MonitorParams p, TcTables tb) {
+__global__ void __launch_bounds__(160, 2)
+    monitor_tc_kernel(MonitorParams p, TcTables tb, const __grid_constant__ CUtensorMap ymap) {
   using C = TcCfg<K>;
   extern __shared__ __align__(1024) uint8_t smem[];
-  __shared__ __align__(8) uint64_t full[C::S], empty[C::S], opfree[2], yfull[2], accready;
+  __shared__ __align__(8) uint64_t yfull[C::SY], yempty[C::SY], tfull[C::ST], tempty[C::ST], opfree, yhfull[2],
+      accready;
   __shared__ uint32_t tmem_base_s;
-  uint8_t *stages = smem;
-  uint8_t *opb = stages + C::S * C::STAGE;
-  uint8_t *a3 = opb + 2 * C::OPBUF;
+  uint8_t *ystages = smem;
+  uint8_t *tstages = ystages + C::SY * C::YBYTES;
+  uint8_t *opb = tstages + C::ST * C::TSTAGE;
+  uint8_t *a3 = opb + C::OPBUF;
+  uint8_t *ring = a3 + C::A3_BYTES;
   const int hcap = p.hcap;
-  float *ring = reinterpret_cast<float *>(a3 + C::A3_BYTES);
-  int16_t *rdate = reinterpret_cast<int16_t *>(ring + (size_t)hcap * 128);
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (tid == 0) {
-    for (int i = 0; i < C::S; ++i) {
-      sm100::mbar_init(&full[i], 1);
-      sm100::mbar_init(&empty[i], 1);
+    for (int i = 0; i < C::SY; ++i) {
+      sm100::mbar_init(&yfull[i], 1);
+      sm100::mbar_init(&yempty[i], 1);
     }
-    sm100::mbar_init(&opfree[0], 1);
-    sm100::mbar_init(&opfree[1], 1);
-    sm100::mbar_init(&yfull[0], 1);
-    sm100::mbar_init(&yfull[1], 1);
+    for (int i = 0; i < C::ST; ++i) {
+      sm100::mbar_init(&tfull[i], 1);
+      sm100::mbar_init(&tempty[i], 1);
+    }
+    sm100::mbar_init(&opfree, 1);
+    sm100::mbar_init(&yhfull[0], 1);
+    sm100::mbar_init(&yhfull[1], 1);
     sm100::mbar_init(&accready, 1);
     sm100::fence_mbar_init();
   }
@@ -123,38 +162,41 @@ __global__ void __launch_bounds__(160, 2) monitor_tc_kernel(MonitorParams p, TcT
   sm100::tc_fence_after();
   const uint32_t tbase = tmem_base_s;
   const int n = p.n, N = p.N, nch = tb.nch, ncm = tb.ncm;
-  const int64_t ldY = p.ldY;
 
   if (warp == 4) {
     // ------------------------------------------------------------ producer
     if (lane == 0) {
+      // one 2-D TMA box [16 dates x 128 px] per chunk (OOB -> NaN = missing)
+      sm100::prefetch_tmap(&ymap);
       const uint64_t pol_first = sm100::policy_evict_first();
-      int s = 0;
-      uint32_t ph = 0;
+      int ys = 0, ts = 0;
+      uint32_t yph = 0, tph = 0;
       for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
-        const float *ybase = p.Y + p.p0 + tile * 128;
+        const int x0 = (int)(tile * 128);
         for (int phase = 0; phase < 3; ++phase) {
           const int nc = phase < 2 ? nch : ncm;
-          const int tbeg = phase < 2 ? 0 : n, tend = phase < 2 ? n : N;
+          const int tbeg = phase < 2 ? 0 : n;
           const uint32_t tabbytes = phase == 0 ? C::TAB1 : phase == 1 ? C::TAB2 : C::TAB3;
           const uint8_t *tabsrc = phase == 0 ? tb.tab1 : phase == 1 ? tb.tab2 : tb.tab3;
           for (int c = 0; c < nc; ++c) {
-            sm100::mbar_wait(&empty[s], ph ^ 1);
-            uint8_t *st = stages + s * C::STAGE;
-            const int t0 = tbeg + c * C::DC;
-            const int rows = min(C::DC, tend - t0);
-            sm100::mbar_arrive_expect_tx(&full[s], rows * 512 + tabbytes);
-            for (int d = 0; d < rows; ++d) {
-              const float *src = ybase + (int64_t)(t0 + d) * ldY;
-              if (phase == 0)
-                sm100::bulk_g2s(st + d * 512, src, 512, &full[s]);          // re-read in pass 2a
-              else
-                sm100::bulk_g2s_stream(st + d * 512, src, 512, &full[s], pol_first);  // last use
+            mbar_wait_sleep(&yempty[ys], yph ^ 1);
+            uint8_t *yst = ystages + ys * C::YBYTES;
+            sm100::mbar_arrive_expect_tx(&yfull[ys], C::YBYTES);
+            if (phase == 0)
+              sm100::tma_load_2d(yst, &ymap, x0, tbeg + c * C::DC, &yfull[ys]);  // re-read in pass 2a (L2)
+            else
+              sm100::tma_load_2d_hint(yst, &ymap, x0, tbeg + c * C::DC, &yfull[ys], pol_first);  // last use
+            if (++ys == C::SY) {
+              ys = 0;
+              yph ^= 1;
             }
-            sm100::bulk_g2s(st + C::YBYTES, tabsrc + (size_t)c * tabbytes, tabbytes, &full[s]);
-            if (++s == C::S) {
-              s = 0;
-              ph ^= 1;
+            mbar_wait_sleep(&tempty[ts], tph ^ 1);
+            uint8_t *tst = tstages + ts * C::TSTAGE;
+            sm100::mbar_arrive_expect_tx(&tfull[ts], tabbytes);
+            sm100::bulk_g2s(tst, tabsrc + (size_t)c * tabbytes, tabbytes, &tfull[ts]);
+            if (++ts == C::ST) {
+              ts = 0;
+              tph ^= 1;
             }
           }
         }
@@ -168,39 +210,42 @@ __global__ void __launch_bounds__(160, 2) monitor_tc_kernel(MonitorParams p, TcT
     const uint32_t idY = sm100::idesc_bf16_f32(128, C::DC);
     const uint32_t idR = sm100::idesc_bf16_f32(128, C::KB3);
     const float qnan = __int_as_float(0x7fc00000);
-    const uint32_t aop = sm100::smem_u32(opb), a3s = sm100::smem_u32(a3), sts = sm100::smem_u32(stages);
-    int cs = 0;
-    uint32_t cph = 0;
-    uint32_t opcnt = 0, yissue = 0, yuse = 0, acnt = 0;
+    const uint32_t aop = sm100::smem_u32(opb), a3s = sm100::smem_u32(a3), tss = sm100::smem_u32(tstages);
+    // ring: slot s = [128 residuals f32][128 date indices u16]; this thread's
+    // residual of slot s at rbase + s*RSLOT, its date at +dofs
+    const uint32_t rbase = sm100::smem_u32(ring) + 4 * tid;
+    const uint32_t rend = rbase + hcap * C::RSLOT;
+    const uint32_t dofs = 512 - 2 * tid;
+    int ys = 0, ts = 0;
+    uint32_t yph = 0, tph = 0, opcnt = 0, yissue = 0, yuse = 0, acnt = 0;
 
-    auto stage_ahead = [&](int ahead, uint32_t &par) {
-      int s = cs + ahead;
-      par = cph;
-      while (s >= C::S) {
-        s -= C::S;
+    auto advance = [&]() {
+      if (++ys == C::SY) {
+        ys = 0;
+        yph ^= 1;
+      }
+      if (++ts == C::ST) {
+        ts = 0;
+        tph ^= 1;
+      }
+    };
+    // thread 0: yhat MMA for the chunk `ahead` chunks after the current one
+    auto issue_yhat = [&](int ahead, uint32_t tab_off) {
+      int s = ts + ahead;
+      uint32_t par = tph;
+      while (s >= C::ST) {
+        s -= C::ST;
         par ^= 1;
       }
-      return s;
-    };
-    auto advance = [&]() {
-      if (++cs == C::S) {
-        cs = 0;
-        cph ^= 1;
-      }
-    };
-    // thread 0: yhat MMA for the chunk `ahead` stages ahead (table offset in stage)
-    auto issue_yhat = [&](int ahead, uint32_t tab_off) {
-      uint32_t par;
-      const int s = stage_ahead(ahead, par);
-      sm100::mbar_wait(&full[s], par);
+      sm100::mbar_wait(&tfull[s], par);
       sm100::tc_fence_after();
       const uint32_t slot = yissue & 1;
-      const uint32_t b3 = sts + s * C::STAGE + C::YBYTES + tab_off;
+      const uint32_t b3 = tss + s * C::TSTAGE + tab_off;
 #pragma unroll
       for (int q = 0; q < C::KY / 16; ++q)
         sm100::umma_bf16(tbase + C::COL_Y + slot * C::DC, sm100::smem_desc(a3s + q * 2 * 2048, 2048, 128),
                          sm100::smem_desc(b3 + q * 2 * 256, 256, 128), idY, q > 0);
-      sm100::umma_commit(&yfull[slot]);
+      sm100::umma_commit(&yhfull[slot]);
       ++yissue;
     };
     auto write_beta_operand = [&](const float (&bt)[K]) {
@@ -228,39 +273,39 @@ __global__ void __launch_bounds__(160, 2) monitor_tc_kernel(MonitorParams p, TcT
         *reinterpret_cast<uint4 *>(a3 + sm100::kmajor_off(tid, 8 * q, 128)) =
             make_uint4(w[4 * q], w[4 * q + 1], w[4 * q + 2], w[4 * q + 3]);
     };
+    auto wait_yhat = [&](float (&yh)[16]) {
+      sm100::mbar_wait(&yhfull[yuse & 1], (yuse >> 1) & 1);
+      sm100::tc_fence_after();
+      sm100::tmem_ld16(lanebase + C::COL_Y + (yuse & 1) * C::DC, yh);
+      sm100::tmem_ld_wait();
+      ++yuse;
+    };
 
     for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
       const int64_t pix = p.p0 + tile * 128 + tid;
       // ================= pass 1: masked Gram + moment on the tensor cores
       int nbar = 0;
-      float c0 = 0.f, ymax = 0.f;
+      float c0 = qnan, ymax = 0.f;
       bool have = false;
       for (int c = 0; c < nch; ++c) {
-        sm100::mbar_wait(&full[cs], cph);
-        const uint32_t ob = opcnt & 1;
-        sm100::mbar_wait(&opfree[ob], ((opcnt >> 1) & 1) ^ 1);
-        const float *Ys = reinterpret_cast<const float *>(stages + cs * C::STAGE);
+        sm100::mbar_wait(&yfull[ys], yph);
+        const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
         uint32_t mw[C::DC / 2], yw[C::DC];
 #pragma unroll
         for (int d = 0; d < C::DC; ++d) {
-          const int t = c * C::DC + d;
-          const float y = t < n ? Ys[d * 128 + tid] : qnan;
+          float y = Ys[d * 128 + tid];
+          y = (c * C::DC + d < n) ? y : qnan;
           const bool v = (y == y);
-          if (v && !have) {
-            c0 = y;
-            have = true;
-          }
-          ymax = v ? fmaxf(ymax, fabsf(y)) : ymax;
-          nbar += v ? 1 : 0;
-          const float yp = v ? y - c0 : 0.f;
-          yw[d] = split2_bf16(yp);
+          c0 = have ? c0 : y;
+          have = have || v;
+          ymax = fmaxf(ymax, fabsf(y));  // NaN ignored
+          nbar += v;
+          yw[d] = split2_bf16(v ? y - c0 : 0.f);
           const uint32_t mb = v ? 0x3F80u : 0u;
-          if (d & 1)
-            mw[d >> 1] |= mb << 16;
-          else
-            mw[d >> 1] = mb;
+          mw[d >> 1] = (d & 1) ? (mw[d >> 1] | (mb << 16)) : mb;
         }
-        uint8_t *A1 = opb + ob * C::OPBUF;
+        sm100::mbar_wait(&opfree, (opcnt & 1) ^ 1);
+        uint8_t *A1 = opb;
         uint8_t *A2 = A1 + C::A1_BYTES;
         *reinterpret_cast<uint4 *>(A1 + sm100::kmajor_off(tid, 0, 128)) = make_uint4(mw[0], mw[1], mw[2], mw[3]);
         *reinterpret_cast<uint4 *>(A1 + sm100::kmajor_off(tid, 8, 128)) = make_uint4(mw[4], mw[5], mw[6], mw[7]);
@@ -271,17 +316,19 @@ __global__ void __launch_bounds__(160, 2) monitor_tc_kernel(MonitorParams p, TcT
         sm100::fence_proxy_async_smem();
         named_bar_sync_128();
         if (tid == 0) {
+          sm100::mbar_arrive(&yempty[ys]);
+          sm100::mbar_wait(&tfull[ts], tph);
           sm100::tc_fence_after();
-          const uint32_t a1 = aop + ob * C::OPBUF, a2 = a1 + C::A1_BYTES;
-          const uint32_t b1 = sts + cs * C::STAGE + C::YBYTES, b2 = b1 + C::B1_BYTES;
+          const uint32_t a1 = aop, a2 = a1 + C::A1_BYTES;
+          const uint32_t b1 = tss + ts * C::TSTAGE, b2 = b1 + C::B1_BYTES;
           sm100::umma_bf16(tbase + C::COL_G, sm100::smem_desc(a1, 2048, 128),
                            sm100::smem_desc(b1, C::NGp * 16, 128), idG, c > 0);
 #pragma unroll
           for (int q = 0; q < 2; ++q)
             sm100::umma_bf16(tbase + C::COL_B, sm100::smem_desc(a2 + q * 2 * 2048, 2048, 128),
                              sm100::smem_desc(b2 + q * 2 * C::KB * 16, C::KB * 16, 128), idB, (c > 0 || q > 0));
-          sm100::umma_commit(&opfree[ob]);
-          sm100::umma_commit(&empty[cs]);
+          sm100::umma_commit(&opfree);
+          sm100::umma_commit(&tempty[ts]);
           if (c == nch - 1) sm100::umma_commit(&accready);
         }
         ++opcnt;
@@ -301,8 +348,7 @@ __global__ void __launch_bounds__(160, 2) monitor_tc_kernel(MonitorParams p, TcT
           sm100::tmem_ld16(lanebase + C::COL_G + 16 * q, v16);
           sm100::tmem_ld_wait();
 #pragma unroll
-          for (int i = 0; i < 16; ++i)
-            F[16 * q + i] = v16[i];
+          for (int i = 0; i < 16; ++i) F[16 * q + i] = v16[i];
         }
         float Bm[C::KB];
 #pragma unroll
@@ -366,23 +412,19 @@ __global__ void __launch_bounds__(160, 2) monitor_tc_kernel(MonitorParams p, TcT
       // ================= pass 2a: residuals r0, sigma, refinement moment, ring
       const int hh = deg ? 1 : h;
       float s2 = 0.f;
-      int cr = 0, ws = 0;
+      int cr = 0;
+      uint32_t wa = rbase;  // ring write address (slot of rank cr)
       for (int c = 0; c < nch; ++c) {
-        sm100::mbar_wait(&full[cs], cph);
-        sm100::mbar_wait(&yfull[yuse & 1], (yuse >> 1) & 1);
-        sm100::tc_fence_after();
+        sm100::mbar_wait(&yfull[ys], yph);
         float yh[16];
-        sm100::tmem_ld16(lanebase + C::COL_Y + (yuse & 1) * C::DC, yh);
-        sm100::tmem_ld_wait();
-        ++yuse;
-        const uint32_t ob = opcnt & 1;
-        sm100::mbar_wait(&opfree[ob], ((opcnt >> 1) & 1) ^ 1);
-        const float *Ys = reinterpret_cast<const float *>(stages + cs * C::STAGE);
+        wait_yhat(yh);
+        const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
         float rs3[3 * C::DC];
 #pragma unroll
         for (int d = 0; d < C::DC; ++d) {
           const int t = c * C::DC + d;
-          const float y = t < n ? Ys[d * 128 + tid] : qnan;
+          float y = Ys[d * 128 + tid];
+          y = (t < n) ? y : qnan;
           const bool v = (y == y);
           const float r = v ? (y - c0) - yh[d] : 0.f;
           s2 = fmaf(r, r, s2);
@@ -391,13 +433,15 @@ __global__ void __launch_bounds__(160, 2) monitor_tc_kernel(MonitorParams p, TcT
           rs3[3 * d + 1] = rm;
           rs3[3 * d + 2] = (r - rh) - rm;
           if (v) {
-            ring[ws * 128 + tid] = r;
-            rdate[ws * 128 + tid] = (int16_t)t;
-            ws = (ws + 1 == hcap) ? 0 : ws + 1;
-            ++cr;
+            sts_f32(wa, r);
+            sts_u16(wa + dofs, (uint16_t)t);
           }
+          const uint32_t wn = wa + C::RSLOT;
+          wa = v ? (wn == rend ? rbase : wn) : wa;
+          cr += v;
         }
-        uint8_t *A4 = opb + ob * C::OPBUF;
+        sm100::mbar_wait(&opfree, (opcnt & 1) ^ 1);
+        uint8_t *A4 = opb;
 #pragma unroll
         for (int q = 0; q < 3 * C::DC / 8; ++q) {
           uint32_t w[4];
@@ -409,16 +453,17 @@ __global__ void __launch_bounds__(160, 2) monitor_tc_kernel(MonitorParams p, TcT
         sm100::tc_fence_before();
         named_bar_sync_128();
         if (tid == 0) {
+          sm100::mbar_arrive(&yempty[ys]);
+          sm100::mbar_wait(&tfull[ts], tph);
           sm100::tc_fence_after();
-          const uint32_t a4 = aop + ob * C::OPBUF;
-          const uint32_t br = sts + cs * C::STAGE + C::YBYTES;
+          const uint32_t br = tss + ts * C::TSTAGE;
 #pragma unroll
           for (int q = 0; q < 3; ++q)
-            sm100::umma_bf16(tbase + C::COL_DB, sm100::smem_desc(a4 + q * 2 * 2048, 2048, 128),
+            sm100::umma_bf16(tbase + C::COL_DB, sm100::smem_desc(aop + q * 2 * 2048, 2048, 128),
                              sm100::smem_desc(br + q * 2 * C::KB3 * 16, C::KB3 * 16, 128), idR, (c > 0 || q > 0));
-          sm100::umma_commit(&opfree[ob]);
+          sm100::umma_commit(&opfree);
           if (c + 2 < nch) issue_yhat(2, C::BR_BYTES);
-          sm100::umma_commit(&empty[cs]);
+          sm100::umma_commit(&tempty[ts]);
           if (c == nch - 1) sm100::umma_commit(&accready);
         }
         ++opcnt;
@@ -463,14 +508,16 @@ __global__ void __launch_bounds__(160, 2) monitor_tc_kernel(MonitorParams p, TcT
         for (int a = 0; a < 2 && a < ncm; ++a) issue_yhat(a, 0);
       }
       // MOSUM seed (m^fst, L518): the last h-1 history residuals, corrected
-      // to the refined fit
+      // to the refined fit; ra = slot of rank cr - hh (the next one to drop)
       float W = 0.f;
+      uint32_t ra;
       {
         const int nseed = deg ? 0 : hh - 1;
-        int slot = ws - nseed;
-        slot += (slot < 0) ? hcap : 0;
+        uint32_t a = wa;
+        for (int q = 0; q < nseed; ++q) a = (a == rbase ? rend : a) - C::RSLOT;  // back nseed slots
+        ra = (a == rbase ? rend : a) - C::RSLOT;                                 // rank cr - hh
         for (int q = 0; q < nseed; ++q) {
-          const int t = rdate[slot * 128 + tid];
+          const int t = lds_u16(a + dofs);
           const float *xr = p.X + (size_t)t * p.KP;
           float corr = 0.f;
 #pragma unroll
@@ -479,58 +526,49 @@ __global__ void __launch_bounds__(160, 2) monitor_tc_kernel(MonitorParams p, TcT
             corr = fmaf(dbf[i], xx.x, corr);
             corr = fmaf(dbf[i + 1], xx.y, corr);
           }
-          const float r = ring[slot * 128 + tid] - corr;
-          ring[slot * 128 + tid] = r;
+          const float r = lds_f32(a) - corr;
+          sts_f32(a, r);
           W += r;
-          slot = (slot + 1 == hcap) ? 0 : slot + 1;
+          a += C::RSLOT;
+          a = (a == rend) ? rbase : a;
         }
+        if (deg) ra = wa;
       }
 
       // ================= pass 2b: monitoring (Alg. 1 l.6-12, Fig. 12 ker 9-10)
       float msum = 0.f;
-      int brk = -1;
-      bool tie = false;
+      int brk = -1, tie = 0;
       const float lam = p.lambda, lam_lo = lam * (1.0f - kTieTol);
       for (int c = 0; c < ncm; ++c) {
-        sm100::mbar_wait(&full[cs], cph);
-        sm100::mbar_wait(&yfull[yuse & 1], (yuse >> 1) & 1);
-        sm100::tc_fence_after();
+        sm100::mbar_wait(&yfull[ys], yph);
         float yh[16];
-        sm100::tmem_ld16(lanebase + C::COL_Y + (yuse & 1) * C::DC, yh);
-        sm100::tmem_ld_wait();
-        ++yuse;
-        const float *Ys = reinterpret_cast<const float *>(stages + cs * C::STAGE);
+        wait_yhat(yh);
+        const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
 #pragma unroll
         for (int d = 0; d < C::DC; ++d) {
-          const int t = n + c * C::DC + d;
-          const float y = t < N ? Ys[d * 128 + tid] : qnan;
-          if (y == y) {
-            const float r = (y - c0) - yh[d];
-            if (cr > nbar) {  // j >= 1: the window drops rank cr - h
-              int rs = ws - hh;
-              rs += (rs < 0) ? hcap : 0;
-              W -= ring[rs * 128 + tid];
-            }
-            W += r;
-            ring[ws * 128 + tid] = r;
-            ws = (ws + 1 == hcap) ? 0 : ws + 1;
-            const float m = W * inv_scale;
-            msum += m;
-            if (brk < 0 && fabsf(m) > lam_lo) {
-              const float B = boundary_f32(lam, cr + 1, nbar);
-              const float am = fabsf(m);
-              tie |= fabsf(am - B) <= kTieTol * B;
-              if (am > B) brk = t - n;
-            }
-            ++cr;
-          }
+          const float y = Ys[d * 128 + tid];  // dates >= N read as NaN (TMA OOB fill)
+          const bool v = (y == y);
+          const float r = (y - c0) - yh[d];
+          const float old = lds_f32(ra);
+          const bool drop = cr > nbar;  // j >= 1: the window drops rank cr - h
+          const float Wn = W + (r - (drop ? old : 0.f));
+          W = v ? Wn : W;
+          if (v) sts_f32(wa, r);
+          const uint32_t wn = wa + C::RSLOT, rn = ra + C::RSLOT;  // ra tracks slot(cr - h)
+          wa = v ? (wn == rend ? rbase : wn) : wa;
+          ra = v ? (rn == rend ? rbase : rn) : ra;
+          const float m = W * inv_scale;
+          msum += v ? m : 0.f;
+          if (v && brk < 0 && fabsf(m) > lam_lo) boundary_rare(m, cr + 1, nbar, lam, c * C::DC + d, brk, tie);
+          cr += v;
         }
         sm100::tc_fence_before();
         named_bar_sync_128();
         if (tid == 0) {
+          sm100::mbar_arrive(&yempty[ys]);
           sm100::tc_fence_after();
           if (c + 2 < ncm) issue_yhat(2, 0);
-          sm100::mbar_arrive(&empty[cs]);
+          sm100::mbar_arrive(&tempty[ts]);
         }
         advance();
       }
@@ -539,13 +577,16 @@ __global__ void __launch_bounds__(160, 2) monitor_tc_kernel(MonitorParams p, TcT
 
       // ================= epilogue
       const bool fit_ok = !((nbar < K + 1) || (h < 1) || (Nbar - nbar < 1));
-      p.out_break[pix] = deg ? -2 : brk;
-      p.out_mag[pix] = deg ? qnan : msum / (float)(Nbar - nbar);
-      if (p.out_sigma) p.out_sigma[pix] = fit_ok ? sigma : qnan;
-      if (p.out_nbar) p.out_nbar[pix] = nbar;
-      if (p.out_flags) p.out_flags[pix] = deg ? 1u : 0u;
-      store_beta<K, float>(p, pix, beta, c0, fit_ok);
-      const bool want = (refit || tie) && fit_ok;
+      const bool inside = pix < p.p0 + p.P;  // the last tile may be ragged
+      if (inside) {
+        p.out_break[pix] = deg ? -2 : brk;
+        p.out_mag[pix] = deg ? qnan : msum / (float)(Nbar - nbar);
+        if (p.out_sigma) p.out_sigma[pix] = fit_ok ? sigma : qnan;
+        if (p.out_nbar) p.out_nbar[pix] = nbar;
+        if (p.out_flags) p.out_flags[pix] = deg ? 1u : 0u;
+        store_beta<K, float>(p, pix, beta, c0, fit_ok);
+      }
+      const bool want = (refit || tie) && fit_ok && inside;
       const unsigned mask = __ballot_sync(0xffffffffu, want);
       if (want) {
         const int leader = __ffs(mask) - 1;
