@@ -338,11 +338,13 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, pl.device);
   // tensor-core path on the full 128-pixel tiles when the stack rows allow
   // 16-byte bulk copies; SIMT kernel on the ragged tail (or everything)
-  const size_t tc_smem = TC::smem_bytes(pl.hcap);
+  const int tc_hcap = pl.hcap;
+  const size_t tc_smem = TC::smem_bytes(tc_hcap);
   const bool tc_ok = pl.dtab && pl.mode != 1 && (prm.ldY % 4) == 0 &&
                      ((uintptr_t)(prm.Y + prm.p0) % 16) == 0 && tc_smem + 1024 <= (size_t)kMaxSmem;
-  CUtensorMap ymap;
-  const bool tma_ok = tc_ok && make_stack_map(&ymap, prm.Y + prm.p0, prm.ldY, prm.P, pl.N);
+  CUtensorMap ymap, hmap;  // full stack; history only (dates >= n out of bounds)
+  const bool tma_ok = tc_ok && make_stack_map(&ymap, prm.Y + prm.p0, prm.ldY, prm.P, pl.N) &&
+                      make_stack_map(&hmap, prm.Y + prm.p0, prm.ldY, prm.P, pl.n);
   const int64_t ntiles = tma_ok ? (prm.P + 127) / 128 : 0;
   // the refit list/counter are plan scratch: order executions on any stream
   CUDA_TRY(cudaStreamWaitEvent(st, pl.scratch_free, 0));
@@ -365,7 +367,8 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
     const int per_sm = (tc_smem + 1024) * 2 + 2048 <= (size_t)kMaxSmem ? 2 : 1;
     const int64_t grid = std::min<int64_t>(ntiles, (int64_t)sms * per_sm);
     bfast::MonitorParams q = prm;
-    bfast::monitor_tc_kernel<K><<<(unsigned)grid, 160, tc_smem, st>>>(q, tb, ymap);
+    q.hcap = tc_hcap;
+    bfast::monitor_tc_kernel<K><<<(unsigned)grid, 224, tc_smem, st>>>(q, tb, ymap, hmap);
     CUDA_TRY(cudaGetLastError());
     ++launches;
   }

@@ -26,11 +26,13 @@
 //   (DESIGN.md "Numerics").
 //
 // Roles (160 threads): warps 0-3 own one pixel per thread (TMEM lane =
-// pixel row); warp 4 is the producer, streaming 16-date x 128-pixel boxes of
-// the time-major stack (one 2-D TMA copy each) into a 4-stage ring that the
-// consumers release as soon as they have read a box, and the chunk's
+// pixel row); warp 4 streams 16-date x 128-pixel boxes of the time-major
+// stack (one 2-D TMA copy each) into a 4-stage ring that the consumer warps
+// release as soon as they have read a box; warp 5 streams the chunk's
 // B-operand tables (one 1-D bulk copy each, L2-resident) into a 3-stage ring
-// released by tcgen05.commit of the MMAs that read them.  Thread 0 issues the MMAs after a
+// released by tcgen05.commit of the MMAs that read them; warp 6 issues every
+// tcgen05.mma.  All hand-offs are mbarriers (per-warp arrivals), so no warp
+// ever waits at a CTA-wide barrier inside the date loops.  Thread 0 issues the MMAs after a
 // named barrier and signals completion with tcgen05.commit on mbarriers.
 // Per tile the chunk sequence is: history (Gram+moment), history again
 // (residuals, sigma, refinement moment, MOSUM ring), monitoring (MOSUM,
@@ -92,6 +94,16 @@ __device__ __forceinline__ void sts_f32(uint32_t a, float v) {
 __device__ __forceinline__ void sts_u16(uint32_t a, uint16_t v) {
   asm volatile("st.shared.u16 [%0], %1;" ::"r"(a), "h"(v) : "memory");
 }
+__device__ __forceinline__ void sts_f32_if(uint32_t a, float v, bool pred) {
+  asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.shared.f32 [%0], %1;\n\t}" ::"r"(a), "f"(v),
+               "r"((uint32_t)pred)
+               : "memory");
+}
+__device__ __forceinline__ void sts_u16_if(uint32_t a, uint16_t v, bool pred) {
+  asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.shared.u16 [%0], %1;\n\t}" ::"r"(a), "h"(v),
+               "r"((uint32_t)pred)
+               : "memory");
+}
 __device__ __forceinline__ float lds_f32(uint32_t a) {
   float v;
   asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(a) : "memory");
@@ -105,14 +117,15 @@ __device__ __forceinline__ int lds_u16(uint32_t a) {
 // producer-side wait with back-off so a waiting producer does not steal
 // issue slots from the consumer warps of its SM sub-partition
 __device__ __forceinline__ void mbar_wait_sleep(uint64_t *bar, uint32_t parity) {
-  while (!sm100::mbar_try_wait(bar, parity)) __nanosleep(64);
+  while (!sm100::mbar_try_wait_suspend(bar, parity, 1000000u)) {
+  }
 }
 // the rare branch of the boundary test (Alg. 1 l.10-12), kept out of line
-__device__ __noinline__ void boundary_rare(float m, int rank1, int nbar, float lam, int off, int &brk, int &tie) {
+// returns bit 0: |m| > B (a break), bit 1: |m|/B within kTieTol of 1
+__device__ __noinline__ int boundary_rare(float m, int rank1, int nbar, float lam) {
   const float B = boundary_f32(lam, rank1, nbar);
   const float am = fabsf(m);
-  tie |= fabsf(am - B) <= kTieTol * B;
-  if (am > B) brk = off;
+  return (am > B ? 1 : 0) | (fabsf(am - B) <= kTieTol * B ? 2 : 0);
 }
 
 // y split into hi and lo bf16 halves packed {lo16: hi part, hi16: lo part}
@@ -126,12 +139,13 @@ __device__ __forceinline__ float bf16_round(float v) {
 }
 
 template <int K>
-__global__ void __launch_bounds__(160, 2)
-    monitor_tc_kernel(MonitorParams p, TcTables tb, const __grid_constant__ CUtensorMap ymap) {
+__global__ void __launch_bounds__(224, 2)
+    monitor_tc_kernel(MonitorParams p, TcTables tb, const __grid_constant__ CUtensorMap ymap,
+                      const __grid_constant__ CUtensorMap hmap) {
   using C = TcCfg<K>;
   extern __shared__ __align__(1024) uint8_t smem[];
-  __shared__ __align__(8) uint64_t yfull[C::SY], yempty[C::SY], tfull[C::ST], tempty[C::ST], opfree, yhfull[2],
-      accready;
+  __shared__ __align__(8) uint64_t yfull[C::SY], yempty[C::SY], tfull[C::ST], tempty[C::ST], opfull, opfree,
+      yhfull[2], yhfree[2], accready, betaready;
   __shared__ uint32_t tmem_base_s;
   uint8_t *ystages = smem;
   uint8_t *tstages = ystages + C::SY * C::YBYTES;
@@ -139,21 +153,26 @@ __global__ void __launch_bounds__(160, 2)
   uint8_t *a3 = opb + C::OPBUF;
   uint8_t *ring = a3 + C::A3_BYTES;
   const int hcap = p.hcap;
+  constexpr int NCW = 4;  // consumer warps
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (tid == 0) {
     for (int i = 0; i < C::SY; ++i) {
       sm100::mbar_init(&yfull[i], 1);
-      sm100::mbar_init(&yempty[i], 1);
+      sm100::mbar_init(&yempty[i], NCW);
     }
     for (int i = 0; i < C::ST; ++i) {
       sm100::mbar_init(&tfull[i], 1);
       sm100::mbar_init(&tempty[i], 1);
     }
+    sm100::mbar_init(&opfull, NCW);
     sm100::mbar_init(&opfree, 1);
-    sm100::mbar_init(&yhfull[0], 1);
-    sm100::mbar_init(&yhfull[1], 1);
+    for (int i = 0; i < 2; ++i) {
+      sm100::mbar_init(&yhfull[i], 1);
+      sm100::mbar_init(&yhfree[i], NCW);
+    }
     sm100::mbar_init(&accready, 1);
+    sm100::mbar_init(&betaready, NCW);
     sm100::fence_mbar_init();
   }
   if (warp == 0) sm100::tmem_alloc(&tmem_base_s, C::TMEM_COLS);
@@ -164,32 +183,49 @@ __global__ void __launch_bounds__(160, 2)
   const int n = p.n, N = p.N, nch = tb.nch, ncm = tb.ncm;
 
   if (warp == 4) {
-    // ------------------------------------------------------------ producer
+    // ------------------------------------------------------------ stack producer
     if (lane == 0) {
-      // one 2-D TMA box [16 dates x 128 px] per chunk (OOB -> NaN = missing)
+      // one 2-D TMA box [16 dates x 128 px] per chunk.  History chunks read
+      // through `hmap` (dates >= n are out of bounds), monitoring chunks
+      // through `ymap`; out-of-bounds elements arrive as NaN = missing.
       sm100::prefetch_tmap(&ymap);
+      sm100::prefetch_tmap(&hmap);
       const uint64_t pol_first = sm100::policy_evict_first();
-      int ys = 0, ts = 0;
-      uint32_t yph = 0, tph = 0;
+      int ys = 0;
+      uint32_t yph = 0;
       for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
         const int x0 = (int)(tile * 128);
         for (int phase = 0; phase < 3; ++phase) {
           const int nc = phase < 2 ? nch : ncm;
           const int tbeg = phase < 2 ? 0 : n;
-          const uint32_t tabbytes = phase == 0 ? C::TAB1 : phase == 1 ? C::TAB2 : C::TAB3;
-          const uint8_t *tabsrc = phase == 0 ? tb.tab1 : phase == 1 ? tb.tab2 : tb.tab3;
           for (int c = 0; c < nc; ++c) {
             mbar_wait_sleep(&yempty[ys], yph ^ 1);
             uint8_t *yst = ystages + ys * C::YBYTES;
             sm100::mbar_arrive_expect_tx(&yfull[ys], C::YBYTES);
             if (phase == 0)
-              sm100::tma_load_2d(yst, &ymap, x0, tbeg + c * C::DC, &yfull[ys]);  // re-read in pass 2a (L2)
+              sm100::tma_load_2d(yst, &hmap, x0, c * C::DC, &yfull[ys]);  // re-read in pass 2a (L2)
             else
-              sm100::tma_load_2d_hint(yst, &ymap, x0, tbeg + c * C::DC, &yfull[ys], pol_first);  // last use
+              sm100::tma_load_2d_hint(yst, phase == 1 ? &hmap : &ymap, x0, tbeg + c * C::DC, &yfull[ys],
+                                      pol_first);  // last use
             if (++ys == C::SY) {
               ys = 0;
               yph ^= 1;
             }
+          }
+        }
+      }
+    }
+  } else if (warp == 5) {
+    // ------------------------------------------------------------ table producer
+    if (lane == 0) {
+      int ts = 0;
+      uint32_t tph = 0;
+      for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
+        for (int phase = 0; phase < 3; ++phase) {
+          const int nc = phase < 2 ? nch : ncm;
+          const uint32_t tabbytes = phase == 0 ? C::TAB1 : phase == 1 ? C::TAB2 : C::TAB3;
+          const uint8_t *tabsrc = phase == 0 ? tb.tab1 : phase == 1 ? tb.tab2 : tb.tab3;
+          for (int c = 0; c < nc; ++c) {
             mbar_wait_sleep(&tempty[ts], tph ^ 1);
             uint8_t *tst = tstages + ts * C::TSTAGE;
             sm100::mbar_arrive_expect_tx(&tfull[ts], tabbytes);
@@ -202,51 +238,119 @@ __global__ void __launch_bounds__(160, 2)
         }
       }
     }
+  } else if (warp == 6) {
+    // ------------------------------------------------------------ MMA issuer
+    if (lane == 0) {
+      const uint32_t idG = sm100::idesc_bf16_f32(128, C::NGp);
+      const uint32_t idB = sm100::idesc_bf16_f32(128, C::KB);
+      const uint32_t idY = sm100::idesc_bf16_f32(128, C::DC);
+      const uint32_t idR = sm100::idesc_bf16_f32(128, C::KB3);
+      const uint32_t aop = sm100::smem_u32(opb), a3s = sm100::smem_u32(a3), tss = sm100::smem_u32(tstages);
+      int ts = 0;
+      uint32_t tph = 0, opcnt = 0, yissue = 0, bcnt = 0;
+      auto tslot = [&](int ahead, uint32_t &par) {
+        int s = ts + ahead;
+        par = tph;
+        while (s >= C::ST) {
+          s -= C::ST;
+          par ^= 1;
+        }
+        return s;
+      };
+      auto tadvance = [&]() {
+        if (++ts == C::ST) {
+          ts = 0;
+          tph ^= 1;
+        }
+      };
+      // yhat of the chunk `ahead` chunks after the current one (table offset)
+      auto issue_yhat = [&](int ahead, uint32_t tab_off) {
+        uint32_t par;
+        const int s = tslot(ahead, par);
+        const uint32_t slot = yissue & 1;
+        mbar_wait_sleep(&yhfree[slot], ((yissue >> 1) & 1) ^ 1);  // consumers done with the slot
+        mbar_wait_sleep(&tfull[s], par);
+        sm100::tc_fence_after();
+        const uint32_t b3 = tss + s * C::TSTAGE + tab_off;
+#pragma unroll
+        for (int q = 0; q < C::KY / 16; ++q)
+          sm100::umma_bf16(tbase + C::COL_Y + slot * C::DC, sm100::smem_desc(a3s + q * 2 * 2048, 2048, 128),
+                           sm100::smem_desc(b3 + q * 2 * 256, 256, 128), idY, q > 0);
+        sm100::umma_commit(&yhfull[slot]);
+        ++yissue;
+      };
+      for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
+        // pass 1: Gram + moment per chunk
+        for (int c = 0; c < nch; ++c) {
+          mbar_wait_sleep(&opfull, opcnt & 1);
+          mbar_wait_sleep(&tfull[ts], tph);
+          sm100::tc_fence_after();
+          const uint32_t a1 = aop, a2 = a1 + C::A1_BYTES;
+          const uint32_t b1 = tss + ts * C::TSTAGE, b2 = b1 + C::B1_BYTES;
+          sm100::umma_bf16(tbase + C::COL_G, sm100::smem_desc(a1, 2048, 128),
+                           sm100::smem_desc(b1, C::NGp * 16, 128), idG, c > 0);
+#pragma unroll
+          for (int q = 0; q < 2; ++q)
+            sm100::umma_bf16(tbase + C::COL_B, sm100::smem_desc(a2 + q * 2 * 2048, 2048, 128),
+                             sm100::smem_desc(b2 + q * 2 * C::KB * 16, C::KB * 16, 128), idB, (c > 0 || q > 0));
+          sm100::umma_commit(&opfree);
+          sm100::umma_commit(&tempty[ts]);
+          if (c == nch - 1) sm100::umma_commit(&accready);
+          ++opcnt;
+          tadvance();
+        }
+        // pass 2a: yhat0 two chunks ahead, refinement moment per chunk
+        mbar_wait_sleep(&betaready, bcnt & 1);
+        ++bcnt;
+        for (int a = 0; a < 2 && a < nch; ++a) issue_yhat(a, C::BR_BYTES);
+        for (int c = 0; c < nch; ++c) {
+          mbar_wait_sleep(&opfull, opcnt & 1);
+          mbar_wait_sleep(&tfull[ts], tph);
+          sm100::tc_fence_after();
+          const uint32_t br = tss + ts * C::TSTAGE;
+#pragma unroll
+          for (int q = 0; q < 3; ++q)
+            sm100::umma_bf16(tbase + C::COL_DB, sm100::smem_desc(aop + q * 2 * 2048, 2048, 128),
+                             sm100::smem_desc(br + q * 2 * C::KB3 * 16, C::KB3 * 16, 128), idR, (c > 0 || q > 0));
+          sm100::umma_commit(&opfree);
+          if (c + 2 < nch) issue_yhat(2, C::BR_BYTES);
+          sm100::umma_commit(&tempty[ts]);
+          if (c == nch - 1) sm100::umma_commit(&accready);
+          ++opcnt;
+          tadvance();
+        }
+        // pass 2b: yhat with the refined beta, two chunks ahead
+        mbar_wait_sleep(&betaready, bcnt & 1);
+        ++bcnt;
+        for (int a = 0; a < 2 && a < ncm; ++a) issue_yhat(a, 0);
+        for (int c = 0; c < ncm; ++c) {
+          if (c + 2 < ncm) issue_yhat(2, 0);
+          sm100::umma_commit(&tempty[ts]);  // chunk c's table was read by its yhat MMA
+          tadvance();
+        }
+      }
+    }
   } else {
     // ------------------------------------------------------------ consumers
     const uint32_t lanebase = tbase + ((uint32_t)(32 * warp) << 16);
-    const uint32_t idG = sm100::idesc_bf16_f32(128, C::NGp);
-    const uint32_t idB = sm100::idesc_bf16_f32(128, C::KB);
-    const uint32_t idY = sm100::idesc_bf16_f32(128, C::DC);
-    const uint32_t idR = sm100::idesc_bf16_f32(128, C::KB3);
     const float qnan = __int_as_float(0x7fc00000);
-    const uint32_t aop = sm100::smem_u32(opb), a3s = sm100::smem_u32(a3), tss = sm100::smem_u32(tstages);
     // ring: slot s = [128 residuals f32][128 date indices u16]; this thread's
     // residual of slot s at rbase + s*RSLOT, its date at +dofs
     const uint32_t rbase = sm100::smem_u32(ring) + 4 * tid;
     const uint32_t rend = rbase + hcap * C::RSLOT;
     const uint32_t dofs = 512 - 2 * tid;
-    int ys = 0, ts = 0;
-    uint32_t yph = 0, tph = 0, opcnt = 0, yissue = 0, yuse = 0, acnt = 0;
+    int ys = 0;
+    uint32_t yph = 0, opcnt = 0, yuse = 0, acnt = 0;
 
-    auto advance = [&]() {
+    auto yadvance = [&]() {
       if (++ys == C::SY) {
         ys = 0;
         yph ^= 1;
       }
-      if (++ts == C::ST) {
-        ts = 0;
-        tph ^= 1;
-      }
     };
-    // thread 0: yhat MMA for the chunk `ahead` chunks after the current one
-    auto issue_yhat = [&](int ahead, uint32_t tab_off) {
-      int s = ts + ahead;
-      uint32_t par = tph;
-      while (s >= C::ST) {
-        s -= C::ST;
-        par ^= 1;
-      }
-      sm100::mbar_wait(&tfull[s], par);
-      sm100::tc_fence_after();
-      const uint32_t slot = yissue & 1;
-      const uint32_t b3 = tss + s * C::TSTAGE + tab_off;
-#pragma unroll
-      for (int q = 0; q < C::KY / 16; ++q)
-        sm100::umma_bf16(tbase + C::COL_Y + slot * C::DC, sm100::smem_desc(a3s + q * 2 * 2048, 2048, 128),
-                         sm100::smem_desc(b3 + q * 2 * 256, 256, 128), idY, q > 0);
-      sm100::umma_commit(&yhfull[slot]);
-      ++yissue;
+    auto warp_arrive = [&](uint64_t *bar) {
+      __syncwarp();
+      if (lane == 0) sm100::mbar_arrive(bar);
     };
     auto write_beta_operand = [&](const float (&bt)[K]) {
       // A3 row = [bh | bh | bh | bm | bm | bl | 0...] (6 blocks of K, KY cols)
@@ -272,12 +376,16 @@ __global__ void __launch_bounds__(160, 2)
       for (int q = 0; q < C::KY / 8; ++q)
         *reinterpret_cast<uint4 *>(a3 + sm100::kmajor_off(tid, 8 * q, 128)) =
             make_uint4(w[4 * q], w[4 * q + 1], w[4 * q + 2], w[4 * q + 3]);
+      sm100::fence_proxy_async_smem();
+      warp_arrive(&betaready);
     };
-    auto wait_yhat = [&](float (&yh)[16]) {
+    auto read_yhat = [&](float (&yh)[16]) {
       sm100::mbar_wait(&yhfull[yuse & 1], (yuse >> 1) & 1);
       sm100::tc_fence_after();
       sm100::tmem_ld16(lanebase + C::COL_Y + (yuse & 1) * C::DC, yh);
       sm100::tmem_ld_wait();
+      sm100::tc_fence_before();
+      warp_arrive(&yhfree[yuse & 1]);
       ++yuse;
     };
 
@@ -290,11 +398,13 @@ __global__ void __launch_bounds__(160, 2)
       for (int c = 0; c < nch; ++c) {
         sm100::mbar_wait(&yfull[ys], yph);
         const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
+        float yv[C::DC];
+#pragma unroll
+        for (int d = 0; d < C::DC; ++d) yv[d] = Ys[d * 128 + tid];  // dates >= n read as NaN (hmap OOB)
         uint32_t mw[C::DC / 2], yw[C::DC];
 #pragma unroll
         for (int d = 0; d < C::DC; ++d) {
-          float y = Ys[d * 128 + tid];
-          y = (c * C::DC + d < n) ? y : qnan;
+          const float y = yv[d];
           const bool v = (y == y);
           c0 = have ? c0 : y;
           have = have || v;
@@ -304,6 +414,7 @@ __global__ void __launch_bounds__(160, 2)
           const uint32_t mb = v ? 0x3F80u : 0u;
           mw[d >> 1] = (d & 1) ? (mw[d >> 1] | (mb << 16)) : mb;
         }
+        warp_arrive(&yempty[ys]);  // every loaded value has been consumed
         sm100::mbar_wait(&opfree, (opcnt & 1) ^ 1);
         uint8_t *A1 = opb;
         uint8_t *A2 = A1 + C::A1_BYTES;
@@ -314,25 +425,9 @@ __global__ void __launch_bounds__(160, 2)
           *reinterpret_cast<uint4 *>(A2 + sm100::kmajor_off(tid, 8 * q, 128)) =
               make_uint4(yw[4 * q], yw[4 * q + 1], yw[4 * q + 2], yw[4 * q + 3]);
         sm100::fence_proxy_async_smem();
-        named_bar_sync_128();
-        if (tid == 0) {
-          sm100::mbar_arrive(&yempty[ys]);
-          sm100::mbar_wait(&tfull[ts], tph);
-          sm100::tc_fence_after();
-          const uint32_t a1 = aop, a2 = a1 + C::A1_BYTES;
-          const uint32_t b1 = tss + ts * C::TSTAGE, b2 = b1 + C::B1_BYTES;
-          sm100::umma_bf16(tbase + C::COL_G, sm100::smem_desc(a1, 2048, 128),
-                           sm100::smem_desc(b1, C::NGp * 16, 128), idG, c > 0);
-#pragma unroll
-          for (int q = 0; q < 2; ++q)
-            sm100::umma_bf16(tbase + C::COL_B, sm100::smem_desc(a2 + q * 2 * 2048, 2048, 128),
-                             sm100::smem_desc(b2 + q * 2 * C::KB * 16, C::KB * 16, 128), idB, (c > 0 || q > 0));
-          sm100::umma_commit(&opfree);
-          sm100::umma_commit(&tempty[ts]);
-          if (c == nch - 1) sm100::umma_commit(&accready);
-        }
+        warp_arrive(&opfull);
         ++opcnt;
-        advance();
+        yadvance();
       }
       sm100::mbar_wait(&accready, acnt & 1);
       ++acnt;
@@ -400,14 +495,8 @@ __global__ void __launch_bounds__(160, 2)
           for (int i = 0; i < K; ++i) beta[i] = 0.f;
         }
       }
-      write_beta_operand(beta);
-      sm100::fence_proxy_async_smem();
       sm100::tc_fence_before();
-      named_bar_sync_128();
-      if (tid == 0) {
-        sm100::tc_fence_after();
-        for (int a = 0; a < 2 && a < nch; ++a) issue_yhat(a, C::BR_BYTES);
-      }
+      write_beta_operand(beta);
 
       // ================= pass 2a: residuals r0, sigma, refinement moment, ring
       const int hh = deg ? 1 : h;
@@ -417,14 +506,15 @@ __global__ void __launch_bounds__(160, 2)
       for (int c = 0; c < nch; ++c) {
         sm100::mbar_wait(&yfull[ys], yph);
         float yh[16];
-        wait_yhat(yh);
+        read_yhat(yh);
         const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
+        float yv[C::DC];
+#pragma unroll
+        for (int d = 0; d < C::DC; ++d) yv[d] = Ys[d * 128 + tid];  // dates >= n read as NaN (hmap OOB)
         float rs3[3 * C::DC];
 #pragma unroll
         for (int d = 0; d < C::DC; ++d) {
-          const int t = c * C::DC + d;
-          float y = Ys[d * 128 + tid];
-          y = (t < n) ? y : qnan;
+          const float y = yv[d];
           const bool v = (y == y);
           const float r = v ? (y - c0) - yh[d] : 0.f;
           s2 = fmaf(r, r, s2);
@@ -432,14 +522,13 @@ __global__ void __launch_bounds__(160, 2)
           rs3[3 * d] = rh;
           rs3[3 * d + 1] = rm;
           rs3[3 * d + 2] = (r - rh) - rm;
-          if (v) {
-            sts_f32(wa, r);
-            sts_u16(wa + dofs, (uint16_t)t);
-          }
+          sts_f32_if(wa, r, v);
+          sts_u16_if(wa + dofs, (uint16_t)(c * C::DC + d), v);
           const uint32_t wn = wa + C::RSLOT;
           wa = v ? (wn == rend ? rbase : wn) : wa;
           cr += v;
         }
+        warp_arrive(&yempty[ys]);  // every loaded value has been consumed
         sm100::mbar_wait(&opfree, (opcnt & 1) ^ 1);
         uint8_t *A4 = opb;
 #pragma unroll
@@ -450,24 +539,9 @@ __global__ void __launch_bounds__(160, 2)
           *reinterpret_cast<uint4 *>(A4 + sm100::kmajor_off(tid, 8 * q, 128)) = make_uint4(w[0], w[1], w[2], w[3]);
         }
         sm100::fence_proxy_async_smem();
-        sm100::tc_fence_before();
-        named_bar_sync_128();
-        if (tid == 0) {
-          sm100::mbar_arrive(&yempty[ys]);
-          sm100::mbar_wait(&tfull[ts], tph);
-          sm100::tc_fence_after();
-          const uint32_t br = tss + ts * C::TSTAGE;
-#pragma unroll
-          for (int q = 0; q < 3; ++q)
-            sm100::umma_bf16(tbase + C::COL_DB, sm100::smem_desc(aop + q * 2 * 2048, 2048, 128),
-                             sm100::smem_desc(br + q * 2 * C::KB3 * 16, C::KB3 * 16, 128), idR, (c > 0 || q > 0));
-          sm100::umma_commit(&opfree);
-          if (c + 2 < nch) issue_yhat(2, C::BR_BYTES);
-          sm100::umma_commit(&tempty[ts]);
-          if (c == nch - 1) sm100::umma_commit(&accready);
-        }
+        warp_arrive(&opfull);
         ++opcnt;
-        advance();
+        yadvance();
       }
       sm100::mbar_wait(&accready, acnt & 1);
       ++acnt;
@@ -499,16 +573,10 @@ __global__ void __launch_bounds__(160, 2)
       }
       if (!deg && !(sigma > 1e-4f * ymax)) deg = true;
       const float inv_scale = 1.0f / (sigma * sqrtf((float)nbar));
-      write_beta_operand(beta);
-      sm100::fence_proxy_async_smem();
       sm100::tc_fence_before();
-      named_bar_sync_128();
-      if (tid == 0) {
-        sm100::tc_fence_after();
-        for (int a = 0; a < 2 && a < ncm; ++a) issue_yhat(a, 0);
-      }
+      write_beta_operand(beta);
       // MOSUM seed (m^fst, L518): the last h-1 history residuals, corrected
-      // to the refined fit; ra = slot of rank cr - hh (the next one to drop)
+      // to the refined fit.  ra = slot of rank cr - hh (the next to drop).
       float W = 0.f;
       uint32_t ra;
       {
@@ -533,44 +601,70 @@ __global__ void __launch_bounds__(160, 2)
           a = (a == rend) ? rbase : a;
         }
         if (deg) ra = wa;
+        // the window of j = 0 drops nothing: the slot of rank nbar - h (or
+        // the write slot for invalid pixels) reads as 0 at the first step
+        sts_f32(ra, 0.f);
       }
 
       // ================= pass 2b: monitoring (Alg. 1 l.6-12, Fig. 12 ker 9-10)
       float msum = 0.f;
-      int brk = -1, tie = 0;
-      const float lam = p.lambda, lam_lo = lam * (1.0f - kTieTol);
+      int brk = -1;
+      bool tie = false;
+      const float lam = p.lambda, lam_lo = lam * (1.0f - kTieTol), lam_hi = lam * (1.0f + kTieTol);
+      // B_j == lambda for every reachable rank (t/nbar <= e): warp-uniform
+      // fast path without the out-of-line boundary evaluation
+      const bool fast = __all_sync(0xffffffffu, deg || boundary_f32(lam, nbar + (N - n), nbar) == lam);
       for (int c = 0; c < ncm; ++c) {
         sm100::mbar_wait(&yfull[ys], yph);
         float yh[16];
-        wait_yhat(yh);
+        read_yhat(yh);
         const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
+        float yv[C::DC];
 #pragma unroll
-        for (int d = 0; d < C::DC; ++d) {
-          const float y = Ys[d * 128 + tid];  // dates >= N read as NaN (TMA OOB fill)
-          const bool v = (y == y);
-          const float r = (y - c0) - yh[d];
-          const float old = lds_f32(ra);
-          const bool drop = cr > nbar;  // j >= 1: the window drops rank cr - h
-          const float Wn = W + (r - (drop ? old : 0.f));
-          W = v ? Wn : W;
-          if (v) sts_f32(wa, r);
-          const uint32_t wn = wa + C::RSLOT, rn = ra + C::RSLOT;  // ra tracks slot(cr - h)
-          wa = v ? (wn == rend ? rbase : wn) : wa;
-          ra = v ? (rn == rend ? rbase : rn) : ra;
-          const float m = W * inv_scale;
-          msum += v ? m : 0.f;
-          if (v && brk < 0 && fabsf(m) > lam_lo) boundary_rare(m, cr + 1, nbar, lam, c * C::DC + d, brk, tie);
-          cr += v;
+        for (int d = 0; d < C::DC; ++d) yv[d] = Ys[d * 128 + tid];  // dates >= N read as NaN (TMA OOB)
+        if (fast) {
+#pragma unroll
+          for (int d = 0; d < C::DC; ++d) {
+            const float y = yv[d];
+            const bool v = (y == y);
+            const float r = (y - c0) - yh[d];
+            const float old = lds_f32(ra);  // rank cr - h (zeroed phantom at j = 0)
+            sts_f32_if(wa, r, v);
+            const uint32_t wn = wa + C::RSLOT, rn = ra + C::RSLOT;
+            wa = v ? (wn == rend ? rbase : wn) : wa;
+            ra = v ? (rn == rend ? rbase : rn) : ra;
+            W = v ? W + (r - old) : W;
+            const float m = W * inv_scale, am = fabsf(m);
+            msum += v ? m : 0.f;
+            const bool cand = v && brk < 0 && am > lam_lo;
+            tie = tie || (cand && am <= lam_hi);
+            brk = (cand && am > lam) ? c * C::DC + d : brk;
+            cr += v;
+          }
+        } else {
+#pragma unroll
+          for (int d = 0; d < C::DC; ++d) {
+            const float y = yv[d];
+            const bool v = (y == y);
+            const float r = (y - c0) - yh[d];
+            const float old = lds_f32(ra);
+            sts_f32_if(wa, r, v);
+            const uint32_t wn = wa + C::RSLOT, rn = ra + C::RSLOT;
+            wa = v ? (wn == rend ? rbase : wn) : wa;
+            ra = v ? (rn == rend ? rbase : rn) : ra;
+            W = v ? W + (r - old) : W;
+            const float m = W * inv_scale;
+            msum += v ? m : 0.f;
+            if (v && brk < 0 && fabsf(m) > lam_lo) {
+              const int code = boundary_rare(m, cr + 1, nbar, lam);
+              tie = tie || (code >> 1);
+              brk = (code & 1) ? c * C::DC + d : brk;
+            }
+            cr += v;
+          }
         }
-        sm100::tc_fence_before();
-        named_bar_sync_128();
-        if (tid == 0) {
-          sm100::mbar_arrive(&yempty[ys]);
-          sm100::tc_fence_after();
-          if (c + 2 < ncm) issue_yhat(2, 0);
-          sm100::mbar_arrive(&tempty[ts]);
-        }
-        advance();
+        warp_arrive(&yempty[ys]);  // every loaded value has been consumed
+        yadvance();
       }
       const int Nbar = cr;
       if (Nbar - nbar < 1) deg = true;

@@ -210,3 +210,19 @@ def test_tc_and_simt_paths_agree_closely(monkeypatch):
     ok = (a["break"] != -2) & (b["break"] != -2)
     d = np.abs(a["magnitude"][ok] - b["magnitude"][ok]) / np.maximum(1, np.abs(b["magnitude"][ok]))
     assert d.max() < 1e-4
+
+
+def test_tc_path_is_deterministic_at_scale(monkeypatch):
+    """Race detector for the warp-specialised pipeline: many persistent tiles
+    per CTA, repeated runs must agree bit for bit."""
+    monkeypatch.setenv("BFAST_KERNEL", "tc")
+    spec = synth.StackSpec(P=1 << 21, N=400, n_hist=200, miss=0.6, mask="cloud", seed=71)
+    Y, dates = synth.generate(spec, DEV)
+    plan = binding.Plan(0, spec.N, dates, spec.n_hist, spec.k, spec.hf, spec.lam)
+    ref = plan.execute(Y, diagnostics=True)
+    ref = {key: v.clone() for key, v in ref.items()}
+    for _ in range(4):
+        o = plan.execute(Y, diagnostics=True)
+        for key in ("break", "magnitude", "sigma", "beta"):
+            assert torch.equal(o[key].nan_to_num(), ref[key].nan_to_num()), key
+    plan.close()
