@@ -379,11 +379,15 @@ __global__ void __launch_bounds__(224, 2)
       sm100::fence_proxy_async_smem();
       warp_arrive(&betaready);
     };
-    auto read_yhat = [&](float (&yh)[16]) {
+    auto wait_yhat = [&]() {
       sm100::mbar_wait(&yhfull[yuse & 1], (yuse >> 1) & 1);
       sm100::tc_fence_after();
-      sm100::tmem_ld16(lanebase + C::COL_Y + (yuse & 1) * C::DC, yh);
+    };
+    auto load_yhat8 = [&](int half, float (&yh)[8]) {
+      sm100::tmem_ld8(lanebase + C::COL_Y + (yuse & 1) * C::DC + 8 * half, yh);
       sm100::tmem_ld_wait();
+    };
+    auto release_yhat = [&]() {
       sm100::tc_fence_before();
       warp_arrive(&yhfree[yuse & 1]);
       ++yuse;
@@ -398,32 +402,32 @@ __global__ void __launch_bounds__(224, 2)
       for (int c = 0; c < nch; ++c) {
         sm100::mbar_wait(&yfull[ys], yph);
         const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
-        float yv[C::DC];
+        sm100::mbar_wait(&opfree, (opcnt & 1) ^ 1);
+#pragma unroll 1
+        for (int hf = 0; hf < 2; ++hf) {  // two halves of 8 dates: half the hot code
+          float yv[8];
 #pragma unroll
-        for (int d = 0; d < C::DC; ++d) yv[d] = Ys[d * 128 + tid];  // dates >= n read as NaN (hmap OOB)
-        uint32_t mw[C::DC / 2], yw[C::DC];
+          for (int d = 0; d < 8; ++d) yv[d] = Ys[(8 * hf + d) * 128 + tid];  // dates >= n read as NaN (hmap)
+          uint32_t mw[4], yw[8];
 #pragma unroll
-        for (int d = 0; d < C::DC; ++d) {
-          const float y = yv[d];
-          const bool v = (y == y);
-          c0 = have ? c0 : y;
-          have = have || v;
-          ymax = fmaxf(ymax, fabsf(y));  // NaN ignored
-          nbar += v;
-          yw[d] = split2_bf16(v ? y - c0 : 0.f);
-          const uint32_t mb = v ? 0x3F80u : 0u;
-          mw[d >> 1] = (d & 1) ? (mw[d >> 1] | (mb << 16)) : mb;
+          for (int d = 0; d < 8; ++d) {
+            const float y = yv[d];
+            const bool v = (y == y);
+            c0 = have ? c0 : y;
+            have = have || v;
+            ymax = fmaxf(ymax, fabsf(y));  // NaN ignored
+            nbar += v;
+            yw[d] = split2_bf16(v ? y - c0 : 0.f);
+            const uint32_t mb = v ? 0x3F80u : 0u;
+            mw[d >> 1] = (d & 1) ? (mw[d >> 1] | (mb << 16)) : mb;
+          }
+          *reinterpret_cast<uint4 *>(opb + sm100::kmajor_off(tid, 8 * hf, 128)) = make_uint4(mw[0], mw[1], mw[2], mw[3]);
+#pragma unroll
+          for (int q = 0; q < 2; ++q)
+            *reinterpret_cast<uint4 *>(opb + C::A1_BYTES + sm100::kmajor_off(tid, 16 * hf + 8 * q, 128)) =
+                make_uint4(yw[4 * q], yw[4 * q + 1], yw[4 * q + 2], yw[4 * q + 3]);
         }
         warp_arrive(&yempty[ys]);  // every loaded value has been consumed
-        sm100::mbar_wait(&opfree, (opcnt & 1) ^ 1);
-        uint8_t *A1 = opb;
-        uint8_t *A2 = A1 + C::A1_BYTES;
-        *reinterpret_cast<uint4 *>(A1 + sm100::kmajor_off(tid, 0, 128)) = make_uint4(mw[0], mw[1], mw[2], mw[3]);
-        *reinterpret_cast<uint4 *>(A1 + sm100::kmajor_off(tid, 8, 128)) = make_uint4(mw[4], mw[5], mw[6], mw[7]);
-#pragma unroll
-        for (int q = 0; q < 4; ++q)
-          *reinterpret_cast<uint4 *>(A2 + sm100::kmajor_off(tid, 8 * q, 128)) =
-              make_uint4(yw[4 * q], yw[4 * q + 1], yw[4 * q + 2], yw[4 * q + 3]);
         sm100::fence_proxy_async_smem();
         warp_arrive(&opfull);
         ++opcnt;
@@ -505,39 +509,43 @@ __global__ void __launch_bounds__(224, 2)
       uint32_t wa = rbase;  // ring write address (slot of rank cr)
       for (int c = 0; c < nch; ++c) {
         sm100::mbar_wait(&yfull[ys], yph);
-        float yh[16];
-        read_yhat(yh);
+        wait_yhat();
         const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
-        float yv[C::DC];
-#pragma unroll
-        for (int d = 0; d < C::DC; ++d) yv[d] = Ys[d * 128 + tid];  // dates >= n read as NaN (hmap OOB)
-        float rs3[3 * C::DC];
-#pragma unroll
-        for (int d = 0; d < C::DC; ++d) {
-          const float y = yv[d];
-          const bool v = (y == y);
-          const float r = v ? (y - c0) - yh[d] : 0.f;
-          s2 = fmaf(r, r, s2);
-          const float rh = bf16_round(r), rm = bf16_round(r - rh);
-          rs3[3 * d] = rh;
-          rs3[3 * d + 1] = rm;
-          rs3[3 * d + 2] = (r - rh) - rm;
-          sts_f32_if(wa, r, v);
-          sts_u16_if(wa + dofs, (uint16_t)(c * C::DC + d), v);
-          const uint32_t wn = wa + C::RSLOT;
-          wa = v ? (wn == rend ? rbase : wn) : wa;
-          cr += v;
-        }
-        warp_arrive(&yempty[ys]);  // every loaded value has been consumed
         sm100::mbar_wait(&opfree, (opcnt & 1) ^ 1);
-        uint8_t *A4 = opb;
+#pragma unroll 1
+        for (int hf = 0; hf < 2; ++hf) {
+          float yh[8], yv[8];
+          load_yhat8(hf, yh);
 #pragma unroll
-        for (int q = 0; q < 3 * C::DC / 8; ++q) {
-          uint32_t w[4];
+          for (int d = 0; d < 8; ++d) yv[d] = Ys[(8 * hf + d) * 128 + tid];  // dates >= n read as NaN (hmap)
+          float rs3[24];
 #pragma unroll
-          for (int u = 0; u < 4; ++u) w[u] = sm100::pack_bf16x2(rs3[8 * q + 2 * u], rs3[8 * q + 2 * u + 1]);
-          *reinterpret_cast<uint4 *>(A4 + sm100::kmajor_off(tid, 8 * q, 128)) = make_uint4(w[0], w[1], w[2], w[3]);
+          for (int d = 0; d < 8; ++d) {
+            const float y = yv[d];
+            const bool v = (y == y);
+            const float r = v ? (y - c0) - yh[d] : 0.f;
+            s2 = fmaf(r, r, s2);
+            const float rh = bf16_round(r), rm = bf16_round(r - rh);
+            rs3[3 * d] = rh;
+            rs3[3 * d + 1] = rm;
+            rs3[3 * d + 2] = (r - rh) - rm;
+            sts_f32_if(wa, r, v);
+            sts_u16_if(wa + dofs, (uint16_t)(c * C::DC + 8 * hf + d), v);
+            const uint32_t wn = wa + C::RSLOT;
+            wa = v ? (wn == rend ? rbase : wn) : wa;
+            cr += v;
+          }
+#pragma unroll
+          for (int q = 0; q < 3; ++q) {
+            uint32_t w[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) w[u] = sm100::pack_bf16x2(rs3[8 * q + 2 * u], rs3[8 * q + 2 * u + 1]);
+            *reinterpret_cast<uint4 *>(opb + sm100::kmajor_off(tid, 24 * hf + 8 * q, 128)) =
+                make_uint4(w[0], w[1], w[2], w[3]);
+          }
         }
+        release_yhat();
+        warp_arrive(&yempty[ys]);  // every loaded value has been consumed
         sm100::fence_proxy_async_smem();
         warp_arrive(&opfull);
         ++opcnt;
@@ -611,58 +619,62 @@ __global__ void __launch_bounds__(224, 2)
       int brk = -1;
       bool tie = false;
       const float lam = p.lambda, lam_lo = lam * (1.0f - kTieTol), lam_hi = lam * (1.0f + kTieTol);
-      // B_j == lambda for every reachable rank (t/nbar <= e): warp-uniform
-      // fast path without the out-of-line boundary evaluation
-      const bool fast = __all_sync(0xffffffffu, deg || boundary_f32(lam, nbar + (N - n), nbar) == lam);
       for (int c = 0; c < ncm; ++c) {
         sm100::mbar_wait(&yfull[ys], yph);
-        float yh[16];
-        read_yhat(yh);
+        wait_yhat();
         const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
-        float yv[C::DC];
+        // B_j == lambda for every rank this chunk can reach (rank/nbar <= e):
+        // warp-uniform fast path without the out-of-line boundary evaluation
+        const bool fast = __all_sync(0xffffffffu, deg || boundary_f32(lam, cr + C::DC, nbar) == lam);
+#pragma unroll 1
+        for (int hf = 0; hf < 2; ++hf) {
+          float yh[8], yv[8];
+          load_yhat8(hf, yh);
 #pragma unroll
-        for (int d = 0; d < C::DC; ++d) yv[d] = Ys[d * 128 + tid];  // dates >= N read as NaN (TMA OOB)
-        if (fast) {
+          for (int d = 0; d < 8; ++d) yv[d] = Ys[(8 * hf + d) * 128 + tid];  // dates >= N read as NaN (TMA OOB)
+          if (fast) {
 #pragma unroll
-          for (int d = 0; d < C::DC; ++d) {
-            const float y = yv[d];
-            const bool v = (y == y);
-            const float r = (y - c0) - yh[d];
-            const float old = lds_f32(ra);  // rank cr - h (zeroed phantom at j = 0)
-            sts_f32_if(wa, r, v);
-            const uint32_t wn = wa + C::RSLOT, rn = ra + C::RSLOT;
-            wa = v ? (wn == rend ? rbase : wn) : wa;
-            ra = v ? (rn == rend ? rbase : rn) : ra;
-            W = v ? W + (r - old) : W;
-            const float m = W * inv_scale, am = fabsf(m);
-            msum += v ? m : 0.f;
-            const bool cand = v && brk < 0 && am > lam_lo;
-            tie = tie || (cand && am <= lam_hi);
-            brk = (cand && am > lam) ? c * C::DC + d : brk;
-            cr += v;
-          }
-        } else {
-#pragma unroll
-          for (int d = 0; d < C::DC; ++d) {
-            const float y = yv[d];
-            const bool v = (y == y);
-            const float r = (y - c0) - yh[d];
-            const float old = lds_f32(ra);
-            sts_f32_if(wa, r, v);
-            const uint32_t wn = wa + C::RSLOT, rn = ra + C::RSLOT;
-            wa = v ? (wn == rend ? rbase : wn) : wa;
-            ra = v ? (rn == rend ? rbase : rn) : ra;
-            W = v ? W + (r - old) : W;
-            const float m = W * inv_scale;
-            msum += v ? m : 0.f;
-            if (v && brk < 0 && fabsf(m) > lam_lo) {
-              const int code = boundary_rare(m, cr + 1, nbar, lam);
-              tie = tie || (code >> 1);
-              brk = (code & 1) ? c * C::DC + d : brk;
+            for (int d = 0; d < 8; ++d) {
+              const float y = yv[d];
+              const bool v = (y == y);
+              const float r = (y - c0) - yh[d];
+              const float old = lds_f32(ra);  // rank cr - h (zeroed phantom at j = 0)
+              sts_f32_if(wa, r, v);
+              const uint32_t wn = wa + C::RSLOT, rn = ra + C::RSLOT;
+              wa = v ? (wn == rend ? rbase : wn) : wa;
+              ra = v ? (rn == rend ? rbase : rn) : ra;
+              W = v ? W + (r - old) : W;
+              const float m = W * inv_scale, am = fabsf(m);
+              msum += v ? m : 0.f;
+              const bool cand = v && brk < 0 && am > lam_lo;
+              tie = tie || (cand && am <= lam_hi);
+              brk = (cand && am > lam) ? c * C::DC + 8 * hf + d : brk;
+              cr += v;
             }
-            cr += v;
+          } else {
+#pragma unroll
+            for (int d = 0; d < 8; ++d) {
+              const float y = yv[d];
+              const bool v = (y == y);
+              const float r = (y - c0) - yh[d];
+              const float old = lds_f32(ra);
+              sts_f32_if(wa, r, v);
+              const uint32_t wn = wa + C::RSLOT, rn = ra + C::RSLOT;
+              wa = v ? (wn == rend ? rbase : wn) : wa;
+              ra = v ? (rn == rend ? rbase : rn) : ra;
+              W = v ? W + (r - old) : W;
+              const float m = W * inv_scale;
+              msum += v ? m : 0.f;
+              if (v && brk < 0 && fabsf(m) > lam_lo) {
+                const int code = boundary_rare(m, cr + 1, nbar, lam);
+                tie = tie || (code >> 1);
+                brk = (code & 1) ? c * C::DC + 8 * hf + d : brk;
+              }
+              cr += v;
+            }
           }
         }
+        release_yhat();
         warp_arrive(&yempty[ys]);  // every loaded value has been consumed
         yadvance();
       }
