@@ -53,7 +53,7 @@ struct MonitorParams {
 };
 
 // Pivot-ratio thresholds of the fp32 solve.
-constexpr double kRefitRatio = 1e-2;   // worse conditioning -> fp64 refit
+constexpr double kRefitRatio = 3e-2;   // worse conditioning -> fp64 refit
 // |m_j|/B_j within kTieTol of 1 at some j <= j* -> the break decision is
 // re-taken in fp64 by the refit kernel
 constexpr float kTieTol = 1e-4f;
@@ -337,8 +337,14 @@ __global__ void __launch_bounds__(128, 4) monitor_simt_kernel(MonitorParams p) {
       beta[i] += dbf[i];
     }
     sigma = sqrtf(fmaxf(s2 - lin, 0.f) / (float)(nbar - K));
+    // sigma^2 = s2 - lin cancels when the refinement step is large next to
+    // the residual sum: the fp32 sigma-hat is then unreliable -> fp64 refit
+    if (!(lin <= 1e-2f * s2)) refit = true;
   }
   if (!deg && !(sigma > 1e-4f * ymax)) deg = true;
+  // noise within 2e-3 of the signal scale: fp32 fitted values (~1e-7 |y|)
+  // are no longer negligible next to sigma-hat -> fp64 refit (R12)
+  if (!deg && !(sigma > 2e-3f * ymax)) refit = true;
   const float inv_scale = 1.0f / (sigma * sqrtf((float)nbar));
   // MOSUM seed: the last h-1 history residuals (ranks nbar-h+1 .. nbar-1),
   // corrected to the refined fit in the ring, summed into W

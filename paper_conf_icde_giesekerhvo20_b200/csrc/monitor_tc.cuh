@@ -134,6 +134,12 @@ __device__ __forceinline__ uint32_t split2_bf16(float v) {
   const float hi = __uint_as_float(w1 << 16);
   return sm100::pack_bf16x2(v, v - hi);
 }
+// bf16 parts by truncation: hi = top 8 significant bits of v (exactly
+// representable), v - hi exact.  Two words' upper halves -> one packed word.
+__device__ __forceinline__ float bf16_trunc(float v) { return __uint_as_float(__float_as_uint(v) & 0xFFFF0000u); }
+__device__ __forceinline__ uint32_t pack_hi16(float lo_elem, float hi_elem) {
+  return __byte_perm(__float_as_uint(lo_elem), __float_as_uint(hi_elem), 0x7632);
+}
 __device__ __forceinline__ float bf16_round(float v) {
   return __uint_as_float(sm100::pack_bf16x2(v, 0.f) << 16);
 }
@@ -402,6 +408,16 @@ __global__ void __launch_bounds__(224, 2)
       for (int c = 0; c < nch; ++c) {
         sm100::mbar_wait(&yfull[ys], yph);
         const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
+        // offset c = first valid value (warp-uniform pre-scan while a lane lacks it)
+        if (__any_sync(0xffffffffu, !have)) {
+          for (int d = 0; d < C::DC && !have; ++d) {
+            const float y = Ys[d * 128 + tid];
+            if (y == y) {
+              c0 = y;
+              have = true;
+            }
+          }
+        }
         sm100::mbar_wait(&opfree, (opcnt & 1) ^ 1);
 #pragma unroll 1
         for (int hf = 0; hf < 2; ++hf) {  // two halves of 8 dates: half the hot code
@@ -409,18 +425,20 @@ __global__ void __launch_bounds__(224, 2)
 #pragma unroll
           for (int d = 0; d < 8; ++d) yv[d] = Ys[(8 * hf + d) * 128 + tid];  // dates >= n read as NaN (hmap)
           uint32_t mw[4], yw[8];
+          float mf[8];
 #pragma unroll
           for (int d = 0; d < 8; ++d) {
             const float y = yv[d];
             const bool v = (y == y);
-            c0 = have ? c0 : y;
-            have = have || v;
             ymax = fmaxf(ymax, fabsf(y));  // NaN ignored
             nbar += v;
-            yw[d] = split2_bf16(v ? y - c0 : 0.f);
-            const uint32_t mb = v ? 0x3F80u : 0u;
-            mw[d >> 1] = (d & 1) ? (mw[d >> 1] | (mb << 16)) : mb;
+            const float yp = v ? y - c0 : 0.f;
+            const float yh = bf16_trunc(yp);
+            yw[d] = pack_hi16(yh, yp - yh);  // {y' hi, y' lo}
+            mf[d] = v ? 1.0f : 0.0f;
           }
+#pragma unroll
+          for (int q = 0; q < 4; ++q) mw[q] = pack_hi16(mf[2 * q], mf[2 * q + 1]);
           *reinterpret_cast<uint4 *>(opb + sm100::kmajor_off(tid, 8 * hf, 128)) = make_uint4(mw[0], mw[1], mw[2], mw[3]);
 #pragma unroll
           for (int q = 0; q < 2; ++q)
@@ -525,24 +543,22 @@ __global__ void __launch_bounds__(224, 2)
             const bool v = (y == y);
             const float r = v ? (y - c0) - yh[d] : 0.f;
             s2 = fmaf(r, r, s2);
-            const float rh = bf16_round(r), rm = bf16_round(r - rh);
+            // exact 3-way bf16 split by truncation: r = rh + rm + rl
+            const float rh = bf16_trunc(r), t1 = r - rh, rm = bf16_trunc(t1);
             rs3[3 * d] = rh;
             rs3[3 * d + 1] = rm;
-            rs3[3 * d + 2] = (r - rh) - rm;
+            rs3[3 * d + 2] = t1 - rm;
             sts_f32_if(wa, r, v);
             sts_u16_if(wa + dofs, (uint16_t)(c * C::DC + 8 * hf + d), v);
-            const uint32_t wn = wa + C::RSLOT;
-            wa = v ? (wn == rend ? rbase : wn) : wa;
+            wa += v ? C::RSLOT : 0u;
+            wa = (wa == rend) ? rbase : wa;
             cr += v;
           }
 #pragma unroll
-          for (int q = 0; q < 3; ++q) {
-            uint32_t w[4];
-#pragma unroll
-            for (int u = 0; u < 4; ++u) w[u] = sm100::pack_bf16x2(rs3[8 * q + 2 * u], rs3[8 * q + 2 * u + 1]);
+          for (int q = 0; q < 3; ++q)
             *reinterpret_cast<uint4 *>(opb + sm100::kmajor_off(tid, 24 * hf + 8 * q, 128)) =
-                make_uint4(w[0], w[1], w[2], w[3]);
-          }
+                make_uint4(pack_hi16(rs3[8 * q], rs3[8 * q + 1]), pack_hi16(rs3[8 * q + 2], rs3[8 * q + 3]),
+                           pack_hi16(rs3[8 * q + 4], rs3[8 * q + 5]), pack_hi16(rs3[8 * q + 6], rs3[8 * q + 7]));
         }
         release_yhat();
         warp_arrive(&yempty[ys]);  // every loaded value has been consumed
@@ -578,8 +594,14 @@ __global__ void __launch_bounds__(224, 2)
           beta[i] += dbf[i];
         }
         sigma = sqrtf(fmaxf(s2 - lin, 0.f) / (float)(nbar - K));
+        // sigma^2 = s2 - lin cancels when the refinement step is large next to
+        // the residual sum: the fp32 sigma-hat is then unreliable -> fp64 refit
+        if (!(lin <= 1e-2f * s2)) refit = true;
       }
       if (!deg && !(sigma > 1e-4f * ymax)) deg = true;
+      // noise within 2e-3 of the signal scale: fp32 fitted values (~1e-7 |y|)
+      // are no longer negligible next to sigma-hat -> fp64 refit (R12)
+      if (!deg && !(sigma > 2e-3f * ymax)) refit = true;
       const float inv_scale = 1.0f / (sigma * sqrtf((float)nbar));
       sm100::tc_fence_before();
       write_beta_operand(beta);
@@ -615,8 +637,8 @@ __global__ void __launch_bounds__(224, 2)
       }
 
       // ================= pass 2b: monitoring (Alg. 1 l.6-12, Fig. 12 ker 9-10)
-      float msum = 0.f;
-      int brk = -1;
+      float msum = 0.f, mfirst = 0.f;
+      int brk = -1, first = -1;
       bool tie = false;
       const float lam = p.lambda, lam_lo = lam * (1.0f - kTieTol), lam_hi = lam * (1.0f + kTieTol);
       for (int c = 0; c < ncm; ++c) {
@@ -626,6 +648,11 @@ __global__ void __launch_bounds__(224, 2)
         // B_j == lambda for every rank this chunk can reach (rank/nbar <= e):
         // warp-uniform fast path without the out-of-line boundary evaluation
         const bool fast = __all_sync(0xffffffffu, deg || boundary_f32(lam, cr + C::DC, nbar) == lam);
+        if (first >= 0 && brk < 0 && !tie) {  // resolve a fast-path candidate
+          const float am = fabsf(mfirst);
+          if (am > lam_hi) brk = first;
+          else tie = true;
+        }
 #pragma unroll 1
         for (int hf = 0; hf < 2; ++hf) {
           float yh[8], yv[8];
@@ -640,15 +667,19 @@ __global__ void __launch_bounds__(224, 2)
               const float r = (y - c0) - yh[d];
               const float old = lds_f32(ra);  // rank cr - h (zeroed phantom at j = 0)
               sts_f32_if(wa, r, v);
-              const uint32_t wn = wa + C::RSLOT, rn = ra + C::RSLOT;
-              wa = v ? (wn == rend ? rbase : wn) : wa;
-              ra = v ? (rn == rend ? rbase : rn) : ra;
+              const uint32_t inc = v ? C::RSLOT : 0u;
+              wa += inc;
+              ra += inc;
+              wa = (wa == rend) ? rbase : wa;
+              ra = (ra == rend) ? rbase : ra;
               W = v ? W + (r - old) : W;
-              const float m = W * inv_scale, am = fabsf(m);
+              const float m = W * inv_scale;
               msum += v ? m : 0.f;
-              const bool cand = v && brk < 0 && am > lam_lo;
-              tie = tie || (cand && am <= lam_hi);
-              brk = (cand && am > lam) ? c * C::DC + 8 * hf + d : brk;
+              // B_j == lambda here: the first |m| > lambda(1 - tol) decides --
+              // a clear crossing is the break, a near tie goes to the fp64 refit
+              const bool cand = v && first < 0 && fabsf(m) > lam_lo;
+              first = cand ? c * C::DC + 8 * hf + d : first;
+              mfirst = cand ? m : mfirst;
               cr += v;
             }
           } else {
@@ -665,7 +696,7 @@ __global__ void __launch_bounds__(224, 2)
               W = v ? W + (r - old) : W;
               const float m = W * inv_scale;
               msum += v ? m : 0.f;
-              if (v && brk < 0 && fabsf(m) > lam_lo) {
+              if (v && brk < 0 && !tie && first < 0 && fabsf(m) > lam_lo) {
                 const int code = boundary_rare(m, cr + 1, nbar, lam);
                 tie = tie || (code >> 1);
                 brk = (code & 1) ? c * C::DC + 8 * hf + d : brk;
@@ -677,6 +708,10 @@ __global__ void __launch_bounds__(224, 2)
         release_yhat();
         warp_arrive(&yempty[ys]);  // every loaded value has been consumed
         yadvance();
+      }
+      if (first >= 0 && brk < 0 && !tie) {
+        if (fabsf(mfirst) > lam_hi) brk = first;
+        else tie = true;
       }
       const int Nbar = cr;
       if (Nbar - nbar < 1) deg = true;
