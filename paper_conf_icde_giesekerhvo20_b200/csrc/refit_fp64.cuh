@@ -94,6 +94,7 @@ __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
     double s2 = 0.0;
     int cr = 0;
     if (lane == 0) S[0] = 0.0;
+    __syncwarp();  // S[0] is read by every lane below
     for (int t0 = 0; t0 < N; t0 += 32) {
       const int t = t0 + lane;
       const float yf = t < N ? ycol[(int64_t)t * ldY] : __int_as_float(0x7fc00000);

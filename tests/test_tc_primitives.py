@@ -17,3 +17,19 @@ def test_umma_probe(tmp_path):
     r = subprocess.run([exe], capture_output=True, text=True, timeout=120)
     print(r.stdout)
     assert r.returncode == 0 and "ALL OK" in r.stdout, r.stdout + r.stderr
+
+
+def test_compute_sanitizer_clean():
+    """memcheck / racecheck / synccheck on a small invocation of both kernels
+    (and the fp64 refit kernel)."""
+    import shutil
+    import sys
+    exe = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
+    script = os.path.join(os.path.dirname(HERE), "tools", "sanitize_case.py")
+    for tool in ("memcheck", "racecheck", "synccheck"):
+        r = subprocess.run([exe, "--tool", tool, "--error-exitcode", "3", sys.executable, script],
+                           capture_output=True, text=True, timeout=900)
+        out = r.stdout + r.stderr
+        assert r.returncode == 0, out[-3000:]
+        assert "0 errors" in out, out[-3000:]
+        assert "hazard" not in out.lower() or "0 hazards" in out.lower(), out[-3000:]
