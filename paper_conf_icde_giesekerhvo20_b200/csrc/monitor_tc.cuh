@@ -347,6 +347,12 @@ __global__ void __launch_bounds__(224, 2)
     const uint32_t dofs = 512 - 2 * tid;
     int ys = 0;
     uint32_t yph = 0, opcnt = 0, yuse = 0, acnt = 0;
+    // 32-bit shared addresses of the barriers this warp waits on / arrives at
+    const uint32_t a_yfull = sm100::smem_u32(&yfull[0]), a_yempty = sm100::smem_u32(&yempty[0]);
+    const uint32_t a_opfull = sm100::smem_u32(&opfull), a_opfree = sm100::smem_u32(&opfree);
+    const uint32_t a_yhfull = sm100::smem_u32(&yhfull[0]), a_yhfree = sm100::smem_u32(&yhfree[0]);
+    const uint32_t a_accready = sm100::smem_u32(&accready), a_betaready = sm100::smem_u32(&betaready);
+    const uint32_t ybuf0 = sm100::smem_u32(ystages);
 
     auto yadvance = [&]() {
       if (++ys == C::SY) {
@@ -354,9 +360,9 @@ __global__ void __launch_bounds__(224, 2)
         yph ^= 1;
       }
     };
-    auto warp_arrive = [&](uint64_t *bar) {
+    auto warp_arrive = [&](uint32_t bar) {
       __syncwarp();
-      if (lane == 0) sm100::mbar_arrive(bar);
+      if (lane == 0) sm100::mbar_arrive_a(bar);
     };
     auto write_beta_operand = [&](const float (&bt)[K]) {
       // A3 row = [bh | bh | bh | bm | bm | bl | 0...] (6 blocks of K, KY cols)
@@ -383,10 +389,10 @@ __global__ void __launch_bounds__(224, 2)
         *reinterpret_cast<uint4 *>(a3 + sm100::kmajor_off(tid, 8 * q, 128)) =
             make_uint4(w[4 * q], w[4 * q + 1], w[4 * q + 2], w[4 * q + 3]);
       sm100::fence_proxy_async_smem();
-      warp_arrive(&betaready);
+      warp_arrive(a_betaready);
     };
     auto wait_yhat = [&]() {
-      sm100::mbar_wait(&yhfull[yuse & 1], (yuse >> 1) & 1);
+      sm100::mbar_wait_a(a_yhfull + 8 * (yuse & 1), (yuse >> 1) & 1);
       sm100::tc_fence_after();
     };
     auto load_yhat8 = [&](int half, float (&yh)[8]) {
@@ -395,7 +401,7 @@ __global__ void __launch_bounds__(224, 2)
     };
     auto release_yhat = [&]() {
       sm100::tc_fence_before();
-      warp_arrive(&yhfree[yuse & 1]);
+      warp_arrive(a_yhfree + 8 * (yuse & 1));
       ++yuse;
     };
 
@@ -406,7 +412,7 @@ __global__ void __launch_bounds__(224, 2)
       float c0 = qnan, ymax = 0.f;
       bool have = false;
       for (int c = 0; c < nch; ++c) {
-        sm100::mbar_wait(&yfull[ys], yph);
+        sm100::mbar_wait_a(a_yfull + 8 * ys, yph);
         const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
         // offset c = first valid value (warp-uniform pre-scan while a lane lacks it)
         if (__any_sync(0xffffffffu, !have)) {
@@ -418,7 +424,7 @@ __global__ void __launch_bounds__(224, 2)
             }
           }
         }
-        sm100::mbar_wait(&opfree, (opcnt & 1) ^ 1);
+        sm100::mbar_wait_a(a_opfree, (opcnt & 1) ^ 1);
 #pragma unroll 1
         for (int hf = 0; hf < 2; ++hf) {  // two halves of 8 dates: half the hot code
           float yv[8];
@@ -445,13 +451,13 @@ __global__ void __launch_bounds__(224, 2)
             *reinterpret_cast<uint4 *>(opb + C::A1_BYTES + sm100::kmajor_off(tid, 16 * hf + 8 * q, 128)) =
                 make_uint4(yw[4 * q], yw[4 * q + 1], yw[4 * q + 2], yw[4 * q + 3]);
         }
-        warp_arrive(&yempty[ys]);  // every loaded value has been consumed
+        warp_arrive(a_yempty + 8 * ys);  // every loaded value has been consumed
         sm100::fence_proxy_async_smem();
-        warp_arrive(&opfull);
+        warp_arrive(a_opfull);
         ++opcnt;
         yadvance();
       }
-      sm100::mbar_wait(&accready, acnt & 1);
+      sm100::mbar_wait_a(a_accready, acnt & 1);
       ++acnt;
       sm100::tc_fence_after();
 
@@ -526,10 +532,10 @@ __global__ void __launch_bounds__(224, 2)
       int cr = 0;
       uint32_t wa = rbase;  // ring write address (slot of rank cr)
       for (int c = 0; c < nch; ++c) {
-        sm100::mbar_wait(&yfull[ys], yph);
+        sm100::mbar_wait_a(a_yfull + 8 * ys, yph);
         wait_yhat();
         const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
-        sm100::mbar_wait(&opfree, (opcnt & 1) ^ 1);
+        sm100::mbar_wait_a(a_opfree, (opcnt & 1) ^ 1);
 #pragma unroll 1
         for (int hf = 0; hf < 2; ++hf) {
           float yh[8], yv[8];
@@ -561,13 +567,13 @@ __global__ void __launch_bounds__(224, 2)
                            pack_hi16(rs3[8 * q + 4], rs3[8 * q + 5]), pack_hi16(rs3[8 * q + 6], rs3[8 * q + 7]));
         }
         release_yhat();
-        warp_arrive(&yempty[ys]);  // every loaded value has been consumed
+        warp_arrive(a_yempty + 8 * ys);  // every loaded value has been consumed
         sm100::fence_proxy_async_smem();
-        warp_arrive(&opfull);
+        warp_arrive(a_opfull);
         ++opcnt;
         yadvance();
       }
-      sm100::mbar_wait(&accready, acnt & 1);
+      sm100::mbar_wait_a(a_accready, acnt & 1);
       ++acnt;
       sm100::tc_fence_after();
 
@@ -640,14 +646,25 @@ __global__ void __launch_bounds__(224, 2)
       float msum = 0.f, mfirst = 0.f;
       int brk = -1, first = -1;
       bool tie = false;
+      // largest 1-based rank with B == lambda (rank/nbar <= e), evaluated with
+      // the exact boundary formula around floor(e * nbar)
+      int rank_flat;
+      {
+        int r0 = (int)(2.718281828f * (float)nbar) - 2;
+        r0 = r0 < 0 ? 0 : r0;
+        rank_flat = r0;
+#pragma unroll
+        for (int q = 1; q <= 4; ++q)
+          if (nbar > 0 && boundary_f32(p.lambda, r0 + q, nbar) == p.lambda) rank_flat = r0 + q;
+      }
       const float lam = p.lambda, lam_lo = lam * (1.0f - kTieTol), lam_hi = lam * (1.0f + kTieTol);
       for (int c = 0; c < ncm; ++c) {
-        sm100::mbar_wait(&yfull[ys], yph);
+        sm100::mbar_wait_a(a_yfull + 8 * ys, yph);
         wait_yhat();
         const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
         // B_j == lambda for every rank this chunk can reach (rank/nbar <= e):
         // warp-uniform fast path without the out-of-line boundary evaluation
-        const bool fast = __all_sync(0xffffffffu, deg || boundary_f32(lam, cr + C::DC, nbar) == lam);
+        const bool fast = __all_sync(0xffffffffu, deg || cr + C::DC <= rank_flat);
         if (first >= 0 && brk < 0 && !tie) {  // resolve a fast-path candidate
           const float am = fabsf(mfirst);
           if (am > lam_hi) brk = first;
@@ -706,7 +723,7 @@ __global__ void __launch_bounds__(224, 2)
           }
         }
         release_yhat();
-        warp_arrive(&yempty[ys]);  // every loaded value has been consumed
+        warp_arrive(a_yempty + 8 * ys);  // every loaded value has been consumed
         yadvance();
       }
       if (first >= 0 && brk < 0 && !tie) {

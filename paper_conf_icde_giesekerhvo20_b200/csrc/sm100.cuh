@@ -58,6 +58,27 @@ __device__ __forceinline__ bool mbar_try_wait_suspend(uint64_t *bar, uint32_t pa
   return ok != 0;
 }
 
+// Same operations on precomputed 32-bit shared addresses (no per-call
+// address materialisation in hot loops).
+__device__ __forceinline__ void mbar_arrive_a(uint32_t a) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(a) : "memory");
+}
+__device__ __forceinline__ bool mbar_try_wait_a(uint32_t a, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+      "selp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(ok)
+      : "r"(a), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait_a(uint32_t a, uint32_t parity) {
+  while (!mbar_try_wait_a(a, parity)) {
+  }
+}
+
 // Make generic-proxy shared-memory writes visible to the async proxy
 // (tensor-core operand reads, bulk copies).
 __device__ __forceinline__ void fence_proxy_async_smem() {
