@@ -87,22 +87,24 @@ def _grid_shape(P: int):
     return H, W
 
 
-def _cloud_field(H: int, W: int, g: torch.Generator, device) -> torch.Tensor:
-    """Smooth value noise: U[0,1) lattice every 64 px, bilinear in between."""
-    gh, gw = H // 64 + 2, W // 64 + 2
-    lat = torch.rand(1, 1, gh, gw, generator=g, device=device)
-    up = torch.nn.functional.interpolate(lat, size=((gh - 1) * 64 + 1, (gw - 1) * 64 + 1),
-                                         mode="bilinear", align_corners=True)
-    return up[0, 0, :H, :W].reshape(-1)
+BLOCK = 1 << 20  # pixels per independently seeded block
 
 
 def generate(spec: StackSpec, device="cpu", ldY: int | None = None, out: torch.Tensor | None = None,
-             return_truth: bool = False, chunk_elems: int = 1 << 28):
-    """Return (Y [N][ldY] float32 on `device`, dates float64 numpy[, truth])."""
+             return_truth: bool = False, chunk_elems: int = 1 << 28, columns: tuple | None = None):
+    """Return (Y [N][ldY] float32 on `device`, dates float64 numpy[, truth]).
+
+    Block-deterministic: pixel parameters, noise and i.i.d. masks are drawn
+    per block of BLOCK pixels from their own seeds, and the cloud field of a
+    date from a global lattice, so `columns=(b, e)` generates exactly the
+    pixels [b, e) of the full scene (a shard for strong scaling) without
+    generating the rest.  Y then holds e - b columns."""
     P, N = int(spec.P), int(spec.N)
-    ldY = P if ldY is None else int(ldY)
-    if ldY < P:
-        raise ValueError("ldY < P")
+    b0, e0 = (0, P) if columns is None else (int(columns[0]), int(columns[1]))
+    W_ = e0 - b0
+    ldY = W_ if ldY is None else int(ldY)
+    if ldY < W_:
+        raise ValueError("ldY < number of columns")
     dev = torch.device(device)
     if out is None:
         Y = torch.empty((N, ldY), dtype=torch.float32, device=dev)
@@ -110,60 +112,98 @@ def generate(spec: StackSpec, device="cpu", ldY: int | None = None, out: torch.T
         Y = out
         assert Y.shape == (N, ldY) and Y.dtype == torch.float32
     dates = make_dates(N, spec.f, spec.year0)
-
-    g = _gen(dev, spec.seed, 0)
-    u = lambda lo, hi, *shape: torch.rand(*shape, generator=g, device=dev) * (hi - lo) + lo
-    a = u(0.3, 0.8, P)
-    b = u(-0.01, 0.01, P)
-    amp_s = u(-0.1, 0.1, 3, P)
-    amp_c = u(-0.1, 0.1, 3, P)
-    s = u(spec.noise_lo, spec.noise_hi, P)
-    has_break = torch.rand(P, generator=g, device=dev) < spec.break_frac
-    delta = u(0.1, 0.5, P) * has_break
-    t0 = torch.randint(spec.n_hist, N, (P,), generator=g, device=dev)
-    cover = None
-    if spec.mask == "cloud":
-        m = float(spec.miss)
-        lo, hi = max(0.0, 2 * m - 1), min(1.0, 2 * m)
-        cover = (torch.rand(N, generator=g, device=dev) * (hi - lo) + lo).cpu().numpy()
-    H, W = _grid_shape(P)
-
-    Tc = max(1, min(N, chunk_elems // max(P, 1)))
-    dd = torch.tensor(dates - dates[0], dtype=torch.float32, device=dev)
+    H, Wd = _grid_shape(P)
     two_pi = 2.0 * math.pi
+    dd = torch.tensor(dates - dates[0], dtype=torch.float32, device=dev)
     sin_t = torch.tensor(np.stack([np.sin(two_pi * j * dates) for j in (1, 2, 3)]),
                          dtype=torch.float32, device=dev)
     cos_t = torch.tensor(np.stack([np.cos(two_pi * j * dates) for j in (1, 2, 3)]),
                          dtype=torch.float32, device=dev)
+    cover = None
+    if spec.mask == "cloud":
+        gc0 = _gen(dev, spec.seed, 3)
+        m = float(spec.miss)
+        lo, hi = max(0.0, 2 * m - 1), min(1.0, 2 * m)
+        cover = (torch.rand(N, generator=gc0, device=dev) * (hi - lo) + lo).cpu().numpy()
+    truth = {"has_break": [], "delta": [], "t0": [], "noise_sd": []}
     tidx = torch.arange(N, device=dev)
-    for c0 in range(0, N, Tc):
-        c1 = min(N, c0 + Tc)
-        gc = _gen(dev, spec.seed, 1 + c0)
-        blk = a[None, :] + b[None, :] * dd[c0:c1, None]
-        for j in range(3):
-            blk += amp_s[j][None, :] * sin_t[j, c0:c1, None]
-            blk += amp_c[j][None, :] * cos_t[j, c0:c1, None]
-        blk += torch.randn(c1 - c0, P, generator=gc, device=dev) * s[None, :]
-        blk -= delta[None, :] * (tidx[c0:c1, None] >= t0[None, :])
-        if spec.mask == "iid":
-            miss = torch.rand(c1 - c0, P, generator=gc, device=dev) < spec.miss
-            blk.masked_fill_(miss, float("nan"))
-        elif spec.mask == "cloud":
-            for t in range(c0, c1):
-                field = _cloud_field(H, W, gc, dev)[:P]
-                sub = field[:: max(1, P // (1 << 20))]
-                thr = torch.quantile(sub, float(cover[t]))
-                blk[t - c0].masked_fill_(field < thr, float("nan"))
-        elif spec.mask != "none":
-            raise ValueError(spec.mask)
-        Y[c0:c1, :P] = blk
-        del blk
-    if ldY > P:
-        Y[:, P:] = float("nan")
+    Tc = max(1, min(N, chunk_elems // max(min(W_, BLOCK), 1)))
+    first_blk, last_blk = b0 // BLOCK, (e0 - 1) // BLOCK if e0 > b0 else b0 // BLOCK - 1
+    for blk in range(first_blk, last_blk + 1):
+        pb, pe = blk * BLOCK, min(P, (blk + 1) * BLOCK)   # block in scene coordinates
+        sb, se = max(pb, b0), min(pe, e0)                # part of it we want
+        nb = pe - pb
+        g = _gen(dev, spec.seed, 1_000_000 + blk)
+        u = lambda lo_, hi_, *shape: torch.rand(*shape, generator=g, device=dev) * (hi_ - lo_) + lo_
+        a = u(0.3, 0.8, nb)
+        b = u(-0.01, 0.01, nb)
+        amp_s = u(-0.1, 0.1, 3, nb)
+        amp_c = u(-0.1, 0.1, 3, nb)
+        s = u(spec.noise_lo, spec.noise_hi, nb)
+        has_break = torch.rand(nb, generator=g, device=dev) < spec.break_frac
+        delta = u(0.1, 0.5, nb) * has_break
+        t0 = torch.randint(spec.n_hist, N, (nb,), generator=g, device=dev)
+        sl = slice(sb - pb, se - pb)
+        if return_truth:
+            truth["has_break"].append(has_break[sl]); truth["delta"].append(delta[sl])
+            truth["t0"].append(t0[sl]); truth["noise_sd"].append(s[sl])
+        for c0 in range(0, N, Tc):
+            c1 = min(N, c0 + Tc)
+            gcn = _gen(dev, spec.seed, 2_000_000 + blk * 65536 + c0)
+            blkv = a[None, :] + b[None, :] * dd[c0:c1, None]
+            for j in range(3):
+                blkv += amp_s[j][None, :] * sin_t[j, c0:c1, None]
+                blkv += amp_c[j][None, :] * cos_t[j, c0:c1, None]
+            blkv += torch.randn(c1 - c0, nb, generator=gcn, device=dev) * s[None, :]
+            blkv -= delta[None, :] * (tidx[c0:c1, None] >= t0[None, :])
+            if spec.mask == "iid":
+                miss = torch.rand(c1 - c0, nb, generator=gcn, device=dev) < spec.miss
+                blkv.masked_fill_(miss, float("nan"))
+            elif spec.mask == "cloud":
+                for t in range(c0, c1):
+                    field, thr = _cloud_rows(H, Wd, P, spec.seed, t, float(cover[t]), pb, pe, dev)
+                    blkv[t - c0].masked_fill_(field < thr, float("nan"))
+            elif spec.mask != "none":
+                raise ValueError(spec.mask)
+            Y[c0:c1, sb - b0:se - b0] = blkv[:, sl]
+            del blkv
+    if ldY > W_:
+        Y[:, W_:] = float("nan")
     if return_truth:
-        truth = {"has_break": has_break, "delta": delta, "t0": t0, "noise_sd": s}
+        truth = {k: torch.cat(v) for k, v in truth.items()}
         return Y, dates, truth
     return Y, dates
+
+
+_FIELD_CACHE = {}
+
+
+def _cloud_rows(H, W, P, seed, t, cover, pb, pe, dev):
+    """Cloud field values for scene pixels [pb, pe) at date t, and the date's
+    threshold (the cover-quantile of the full field, from a fixed subsample)."""
+    key = (H, W, seed, t, str(dev))
+    if key not in _FIELD_CACHE:
+        if len(_FIELD_CACHE) > 8192:
+            _FIELD_CACHE.clear()
+        g = _gen(dev, seed, 3_000_000 + t)
+        gh, gw = H // 64 + 2, W // 64 + 2
+        lat = torch.rand(1, 1, gh, gw, generator=g, device=dev)
+        # threshold from a coarse full-field sample (every 8th row / column)
+        coarse = torch.nn.functional.interpolate(lat, size=((gh - 1) * 8 + 1, (gw - 1) * 8 + 1),
+                                                 mode="bilinear", align_corners=True)
+        thr = torch.quantile(coarse[0, 0, : (H + 7) // 8, : (W + 7) // 8].reshape(-1)[: 1 << 24], cover)
+        _FIELD_CACHE[key] = (lat, thr)
+    lat, thr = _FIELD_CACHE[key]
+    gh, gw = lat.shape[2], lat.shape[3]
+    r0, r1 = pb // W, (pe - 1) // W + 1
+    # rows r0..r1-1 of the bilinear upsampling (align_corners: row y <-> lattice y/64)
+    lr0, lr1 = r0 // 64, min(gh - 1, (r1 - 1) // 64 + 1)
+    sub = lat[:, :, lr0:lr1 + 1, :]
+    up = torch.nn.functional.interpolate(sub, size=((lr1 - lr0) * 64 + 1, (gw - 1) * 64 + 1),
+                                         mode="bilinear", align_corners=True)[0, 0]
+    rows = up[r0 - lr0 * 64: r1 - lr0 * 64, :W].reshape(-1)
+    off = pb - r0 * W
+    return rows[off: off + (pe - pb)], thr
 
 
 def sample_columns(Y: torch.Tensor, P: int, count: int, seed: int = 0) -> np.ndarray:
