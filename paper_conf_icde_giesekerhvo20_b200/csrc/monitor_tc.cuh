@@ -364,14 +364,17 @@ __global__ void __launch_bounds__(224, 2)
       __syncwarp();
       if (lane == 0) sm100::mbar_arrive_a(bar);
     };
-    auto write_beta_operand = [&](const float (&bt)[K]) {
-      // A3 row = [bh | bh | bh | bm | bm | bl | 0...] (6 blocks of K, KY cols)
+    auto write_beta_operand = [&](const float (&bt)[K], float off) {
+      // A3 row = [bh | bh | bh | bm | bm | bl | 0...] (6 blocks of K, KY cols);
+      // `off` would fold an offset into the intercept (kept at 0: the GEMM's
+      // accumulation error scales with |yhat|, so the offset stays outside)
       float h[K], m[K], l[K];
 #pragma unroll
       for (int i = 0; i < K; ++i) {
-        h[i] = bf16_round(bt[i]);
-        m[i] = bf16_round(bt[i] - h[i]);
-        l[i] = bt[i] - h[i] - m[i];
+        const float bi = i == 0 ? bt[0] + off : bt[i];
+        h[i] = bf16_round(bi);
+        m[i] = bf16_round(bi - h[i]);
+        l[i] = bi - h[i] - m[i];
       }
       uint32_t w[C::KY / 2];
 #pragma unroll
@@ -524,7 +527,7 @@ __global__ void __launch_bounds__(224, 2)
         }
       }
       sm100::tc_fence_before();
-      write_beta_operand(beta);
+      write_beta_operand(beta, 0.f);
 
       // ================= pass 2a: residuals r0, sigma, refinement moment, ring
       const int hh = deg ? 1 : h;
@@ -610,7 +613,7 @@ __global__ void __launch_bounds__(224, 2)
       if (!deg && !(sigma > 2e-3f * ymax)) refit = true;
       const float inv_scale = 1.0f / (sigma * sqrtf((float)nbar));
       sm100::tc_fence_before();
-      write_beta_operand(beta);
+      write_beta_operand(beta, 0.f);
       // MOSUM seed (m^fst, L518): the last h-1 history residuals, corrected
       // to the refined fit.  ra = slot of rank cr - hh (the next to drop).
       float W = 0.f;
@@ -689,9 +692,9 @@ __global__ void __launch_bounds__(224, 2)
               ra += inc;
               wa = (wa == rend) ? rbase : wa;
               ra = (ra == rend) ? rbase : ra;
-              W = v ? W + (r - old) : W;
+              if (v) W += r - old;
               const float m = W * inv_scale;
-              msum += v ? m : 0.f;
+              if (v) msum += m;
               // B_j == lambda here: the first |m| > lambda(1 - tol) decides --
               // a clear crossing is the break, a near tie goes to the fp64 refit
               const bool cand = v && first < 0 && fabsf(m) > lam_lo;
