@@ -24,6 +24,13 @@ def deps():
         os.path.join(ROOT, "include", "bfast.h")]
 
 
+def _nvcc() -> str:
+    nvcc = os.environ.get("NVCC", "nvcc")
+    if not os.path.exists(nvcc) and os.path.exists("/usr/local/cuda/bin/nvcc"):
+        nvcc = "/usr/local/cuda/bin/nvcc"
+    return nvcc
+
+
 def up_to_date() -> bool:
     if not os.path.exists(OUT):
         return False
@@ -31,13 +38,19 @@ def up_to_date() -> bool:
     return all(os.path.getmtime(d) <= t for d in deps())
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
+def build(force: bool = False, verbose: bool = False, out: str | None = None, defines=()) -> str:
+    """Build the package's libbfast.so; `out` + `defines` build a variant
+    elsewhere (kernel A/B experiments, tools/ab_bench.sh), never the default."""
+    if out is not None:
+        cmd = [_nvcc(), *NVCC_FLAGS, *[f"-D{d}" for d in defines], "-I", os.path.join(ROOT, "include"),
+               *sources(), "-o", out]
+        r = subprocess.run(cmd, capture_output=True, text=True)
+        if r.returncode != 0:
+            raise RuntimeError(r.stderr[-4000:])
+        return out
     if not force and up_to_date():
         return OUT
-    nvcc = os.environ.get("NVCC", "nvcc")
-    if not os.path.exists(nvcc) and os.path.exists("/usr/local/cuda/bin/nvcc"):
-        nvcc = "/usr/local/cuda/bin/nvcc"
-    cmd = [nvcc, *NVCC_FLAGS, "-I", os.path.join(ROOT, "include"), *sources(), "-o", OUT + ".tmp"]
+    cmd = [_nvcc(), *NVCC_FLAGS, "-I", os.path.join(ROOT, "include"), *sources(), "-o", OUT + ".tmp"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     log = os.path.join(HERE, "build.log")
     with open(log, "w") as f:

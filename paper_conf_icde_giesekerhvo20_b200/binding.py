@@ -14,7 +14,9 @@ from typing import Optional
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libbfast.so")
+# BFAST_LIB: another in-tree build of the same ABI (A/B timing of kernel
+# variants on one box, tools/ab_bench.sh); the default is the package's own
+LIB_PATH = os.environ.get("BFAST_LIB") or os.path.join(_HERE, "libbfast.so")
 _lib = None
 
 BFAST_OK, BFAST_EINVAL, BFAST_EUNSUPPORTED, BFAST_ECUDA, BFAST_ENOMEM = 0, -1, -2, -3, -4

@@ -339,7 +339,32 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
   // tensor-core path on the full 128-pixel tiles when the stack rows allow
   // 16-byte bulk copies; SIMT kernel on the ragged tail (or everything)
   const int tc_hcap = pl.hcap;
-  const size_t tc_smem = TC::smem_bytes(tc_hcap);
+  // shared-memory layout: two CTAs per SM hide each other's latencies
+  // (measured 1.5x over one), so take the first layout that fits twice.
+  // Two stack stages already cover the HBM latency of this compute-bound
+  // kernel (2 and 4 stages time alike); double operand buffers let the
+  // consumers fill chunk c+1 while the MMA still reads chunk c.
+  auto fits2 = [&](size_t b) { return (b + 1024) * 2 + 2048 <= (size_t)kMaxSmem; };
+  int tc_sy = 2, tc_nop = 2, per_sm = 1;
+  {
+    const int cand[4][2] = {{2, 2}, {2, 1}, {3, 2}, {3, 1}};
+    for (auto &c : cand)
+      if (fits2(TC::smem_bytes(tc_hcap, pl.nch, c[0], c[1]))) {
+        tc_sy = c[0];
+        tc_nop = c[1];
+        per_sm = 2;
+        break;
+      }
+  }
+  if (const char *lay = std::getenv("BFAST_TC_LAYOUT")) {  // experiments: "sy,nop,per_sm"
+    int a = 0, b = 0, c = 0;
+    if (std::sscanf(lay, "%d,%d,%d", &a, &b, &c) == 3 && a >= 2 && a <= 4 && b >= 1 && b <= 2 && c >= 1 && c <= 2) {
+      tc_sy = a;
+      tc_nop = b;
+      per_sm = c;
+    }
+  }
+  const size_t tc_smem = TC::smem_bytes(tc_hcap, pl.nch, tc_sy, tc_nop);
   const bool tc_ok = pl.dtab && pl.mode != 1 && (prm.ldY % 4) == 0 &&
                      ((uintptr_t)(prm.Y + prm.p0) % 16) == 0 && tc_smem + 1024 <= (size_t)kMaxSmem;
   CUtensorMap ymap, hmap;  // full stack; history only (dates >= n out of bounds)
@@ -364,7 +389,8 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
     tb.nch = pl.nch;
     tb.ncm = pl.ncm;
     tb.ntiles = ntiles;
-    const int per_sm = (tc_smem + 1024) * 2 + 2048 <= (size_t)kMaxSmem ? 2 : 1;
+    tb.sy = tc_sy;
+    tb.nop = tc_nop;
     const int64_t grid = std::min<int64_t>(ntiles, (int64_t)sms * per_sm);
     bfast::MonitorParams q = prm;
     q.hcap = tc_hcap;

@@ -69,21 +69,27 @@ struct TcCfg {
   static constexpr int TABMAX = TAB1 > TAB2 ? TAB1 : TAB2;
   static constexpr int YBYTES = DC * 128 * 4;             // one [16 dates x 128 px] box
   static constexpr int TSTAGE = ((TABMAX + 127) / 128) * 128;
-  static constexpr int SY = 4;                             // stack ring stages (released on read)
+  static constexpr int SY_MAX = 4;                         // stack ring stages (released on read; 3 or 4)
   static constexpr int ST = 3;                             // table ring stages (released by MMA commit)
   static constexpr int A1_BYTES = 128 * DC * 2;
   static constexpr int A2_BYTES = 128 * 2 * DC * 2;
   static constexpr int A4_BYTES = 128 * 3 * DC * 2;        // r0 hi|mid|lo per date
   static constexpr int OPBUF = A1_BYTES + A2_BYTES > A4_BYTES ? A1_BYTES + A2_BYTES : A4_BYTES;
   static constexpr int A3_BYTES = 128 * KY * 2;
-  static constexpr int RSLOT = 128 * 4 + 128 * 2;         // ring slot: 128 residuals + 128 dates
-  static constexpr size_t smem_fixed() { return (size_t)SY * YBYTES + (size_t)ST * TSTAGE + OPBUF + A3_BYTES; }
-  static constexpr size_t smem_bytes(int hcap) { return smem_fixed() + (size_t)hcap * RSLOT; }
+  static constexpr int RSLOT = 128 * 4;                   // ring slot: one residual per pixel
+  static constexpr int VSLOT = 128 * 2;                   // validity mask: 16 bits per pixel per chunk
+  // sy stack stages, nop operand buffers (2: the consumers fill one while the
+  // MMA reads the other), the MOSUM ring of hcap slots, nch history masks
+  static constexpr size_t smem_bytes(int hcap, int nch, int sy, int nop) {
+    return (size_t)sy * YBYTES + (size_t)ST * TSTAGE + (size_t)nop * OPBUF + A3_BYTES + (size_t)hcap * RSLOT +
+           (size_t)nch * VSLOT;
+  }
 };
 
 struct TcTables {
   const uint8_t *tab1, *tab2, *tab3;  // per-chunk B operands, canonical K-major layout
   int nch, ncm;                       // history / monitoring chunks of 16 dates
+  int sy, nop;                        // stack stages (3|4), operand buffers (1|2)
   int64_t ntiles;                     // 128-pixel tiles (the last may be ragged)
 };
 
@@ -94,14 +100,12 @@ __device__ __forceinline__ void sts_f32(uint32_t a, float v) {
 __device__ __forceinline__ void sts_u16(uint32_t a, uint16_t v) {
   asm volatile("st.shared.u16 [%0], %1;" ::"r"(a), "h"(v) : "memory");
 }
-__device__ __forceinline__ void sts_f32_if(uint32_t a, float v, bool pred) {
+// store v if `inc` (the ring advance of this date: 0 for a missing one) is
+// non-zero.  The advance is materialised anyway, so the predicate costs one
+// compare instead of a re-evaluated NaN test (only 7 predicate registers).
+__device__ __forceinline__ void sts_f32_inc(uint32_t a, float v, uint32_t inc) {
   asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.shared.f32 [%0], %1;\n\t}" ::"r"(a), "f"(v),
-               "r"((uint32_t)pred)
-               : "memory");
-}
-__device__ __forceinline__ void sts_u16_if(uint32_t a, uint16_t v, bool pred) {
-  asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.shared.u16 [%0], %1;\n\t}" ::"r"(a), "h"(v),
-               "r"((uint32_t)pred)
+               "r"(inc)
                : "memory");
 }
 __device__ __forceinline__ float lds_f32(uint32_t a) {
@@ -116,9 +120,30 @@ __device__ __forceinline__ int lds_u16(uint32_t a) {
 }
 // producer-side wait with back-off so a waiting producer does not steal
 // issue slots from the consumer warps of its SM sub-partition
-__device__ __forceinline__ void mbar_wait_sleep(uint64_t *bar, uint32_t parity) {
-  while (!sm100::mbar_try_wait_suspend(bar, parity, 1000000u)) {
+#ifndef BFAST_AUX_WAIT
+#define BFAST_AUX_WAIT 0
+#endif
+#ifndef BFAST_MMA_WAIT
+#define BFAST_MMA_WAIT 0
+#endif
+template <int MODE>
+__device__ __forceinline__ void mbar_wait_mode(uint64_t *bar, uint32_t parity) {
+  if (MODE == 0) {
+    while (!sm100::mbar_try_wait_suspend(bar, parity, 1000000u)) {
+    }
+  } else if (MODE == 1) {
+    while (!sm100::mbar_try_wait(bar, parity)) {
+    }
+  } else {
+    while (!sm100::mbar_try_wait_suspend(bar, parity, (uint32_t)MODE)) {
+    }
   }
+}
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t *bar, uint32_t parity) {
+  mbar_wait_mode<BFAST_AUX_WAIT>(bar, parity);
+}
+__device__ __forceinline__ void mbar_wait_mma(uint64_t *bar, uint32_t parity) {
+  mbar_wait_mode<BFAST_MMA_WAIT>(bar, parity);
 }
 // the rare branch of the boundary test (Alg. 1 l.10-12), kept out of line
 // returns bit 0: |m| > B (a break), bit 1: |m|/B within kTieTol of 1
@@ -150,20 +175,21 @@ __global__ void __launch_bounds__(224, 2)
                       const __grid_constant__ CUtensorMap hmap) {
   using C = TcCfg<K>;
   extern __shared__ __align__(1024) uint8_t smem[];
-  __shared__ __align__(8) uint64_t yfull[C::SY], yempty[C::SY], tfull[C::ST], tempty[C::ST], opfull, opfree,
-      yhfull[2], yhfree[2], accready, betaready;
+  __shared__ __align__(8) uint64_t yfull[C::SY_MAX], yempty[C::SY_MAX], tfull[C::ST], tempty[C::ST], opfull[2],
+      opfree[2], yhfull[2], yhfree[2], accready, betaready;
   __shared__ uint32_t tmem_base_s;
+  const int hcap = p.hcap, SY = tb.sy, NOP = tb.nop;
   uint8_t *ystages = smem;
-  uint8_t *tstages = ystages + C::SY * C::YBYTES;
+  uint8_t *tstages = ystages + SY * C::YBYTES;
   uint8_t *opb = tstages + C::ST * C::TSTAGE;
-  uint8_t *a3 = opb + C::OPBUF;
+  uint8_t *a3 = opb + NOP * C::OPBUF;
   uint8_t *ring = a3 + C::A3_BYTES;
-  const int hcap = p.hcap;
+  uint8_t *vmask = ring + hcap * C::RSLOT;
   constexpr int NCW = 4;  // consumer warps
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   if (tid == 0) {
-    for (int i = 0; i < C::SY; ++i) {
+    for (int i = 0; i < C::SY_MAX; ++i) {
       sm100::mbar_init(&yfull[i], 1);
       sm100::mbar_init(&yempty[i], NCW);
     }
@@ -171,9 +197,9 @@ __global__ void __launch_bounds__(224, 2)
       sm100::mbar_init(&tfull[i], 1);
       sm100::mbar_init(&tempty[i], 1);
     }
-    sm100::mbar_init(&opfull, NCW);
-    sm100::mbar_init(&opfree, 1);
     for (int i = 0; i < 2; ++i) {
+      sm100::mbar_init(&opfull[i], NCW);
+      sm100::mbar_init(&opfree[i], 1);
       sm100::mbar_init(&yhfull[i], 1);
       sm100::mbar_init(&yhfree[i], NCW);
     }
@@ -213,7 +239,7 @@ __global__ void __launch_bounds__(224, 2)
             else
               sm100::tma_load_2d_hint(yst, phase == 1 ? &hmap : &ymap, x0, tbeg + c * C::DC, &yfull[ys],
                                       pol_first);  // last use
-            if (++ys == C::SY) {
+            if (++ys == SY) {
               ys = 0;
               yph ^= 1;
             }
@@ -269,13 +295,20 @@ __global__ void __launch_bounds__(224, 2)
           tph ^= 1;
         }
       };
+      // operand buffer of the opcnt-th chunk and its phase parity
+      auto opwait = [&]() -> uint32_t {
+        const uint32_t ob = NOP == 2 ? (opcnt & 1) : 0;
+        const uint32_t par = NOP == 2 ? ((opcnt >> 1) & 1) : (opcnt & 1);
+        mbar_wait_mma(&opfull[ob], par);
+        return ob;
+      };
       // yhat of the chunk `ahead` chunks after the current one (table offset)
       auto issue_yhat = [&](int ahead, uint32_t tab_off) {
         uint32_t par;
         const int s = tslot(ahead, par);
         const uint32_t slot = yissue & 1;
-        mbar_wait_sleep(&yhfree[slot], ((yissue >> 1) & 1) ^ 1);  // consumers done with the slot
-        mbar_wait_sleep(&tfull[s], par);
+        mbar_wait_mma(&yhfree[slot], ((yissue >> 1) & 1) ^ 1);  // consumers done with the slot
+        mbar_wait_mma(&tfull[s], par);
         sm100::tc_fence_after();
         const uint32_t b3 = tss + s * C::TSTAGE + tab_off;
 #pragma unroll
@@ -288,10 +321,10 @@ __global__ void __launch_bounds__(224, 2)
       for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
         // pass 1: Gram + moment per chunk
         for (int c = 0; c < nch; ++c) {
-          mbar_wait_sleep(&opfull, opcnt & 1);
-          mbar_wait_sleep(&tfull[ts], tph);
+          const uint32_t ob = opwait();
+          mbar_wait_mma(&tfull[ts], tph);
           sm100::tc_fence_after();
-          const uint32_t a1 = aop, a2 = a1 + C::A1_BYTES;
+          const uint32_t a1 = aop + ob * C::OPBUF, a2 = a1 + C::A1_BYTES;
           const uint32_t b1 = tss + ts * C::TSTAGE, b2 = b1 + C::B1_BYTES;
           sm100::umma_bf16(tbase + C::COL_G, sm100::smem_desc(a1, 2048, 128),
                            sm100::smem_desc(b1, C::NGp * 16, 128), idG, c > 0);
@@ -299,26 +332,26 @@ __global__ void __launch_bounds__(224, 2)
           for (int q = 0; q < 2; ++q)
             sm100::umma_bf16(tbase + C::COL_B, sm100::smem_desc(a2 + q * 2 * 2048, 2048, 128),
                              sm100::smem_desc(b2 + q * 2 * C::KB * 16, C::KB * 16, 128), idB, (c > 0 || q > 0));
-          sm100::umma_commit(&opfree);
+          sm100::umma_commit(&opfree[ob]);
           sm100::umma_commit(&tempty[ts]);
           if (c == nch - 1) sm100::umma_commit(&accready);
           ++opcnt;
           tadvance();
         }
         // pass 2a: yhat0 two chunks ahead, refinement moment per chunk
-        mbar_wait_sleep(&betaready, bcnt & 1);
+        mbar_wait_mma(&betaready, bcnt & 1);
         ++bcnt;
         for (int a = 0; a < 2 && a < nch; ++a) issue_yhat(a, C::BR_BYTES);
         for (int c = 0; c < nch; ++c) {
-          mbar_wait_sleep(&opfull, opcnt & 1);
-          mbar_wait_sleep(&tfull[ts], tph);
+          const uint32_t ob = opwait();
+          mbar_wait_mma(&tfull[ts], tph);
           sm100::tc_fence_after();
           const uint32_t br = tss + ts * C::TSTAGE;
 #pragma unroll
           for (int q = 0; q < 3; ++q)
-            sm100::umma_bf16(tbase + C::COL_DB, sm100::smem_desc(aop + q * 2 * 2048, 2048, 128),
+            sm100::umma_bf16(tbase + C::COL_DB, sm100::smem_desc(aop + ob * C::OPBUF + q * 2 * 2048, 2048, 128),
                              sm100::smem_desc(br + q * 2 * C::KB3 * 16, C::KB3 * 16, 128), idR, (c > 0 || q > 0));
-          sm100::umma_commit(&opfree);
+          sm100::umma_commit(&opfree[ob]);
           if (c + 2 < nch) issue_yhat(2, C::BR_BYTES);
           sm100::umma_commit(&tempty[ts]);
           if (c == nch - 1) sm100::umma_commit(&accready);
@@ -326,7 +359,7 @@ __global__ void __launch_bounds__(224, 2)
           tadvance();
         }
         // pass 2b: yhat with the refined beta, two chunks ahead
-        mbar_wait_sleep(&betaready, bcnt & 1);
+        mbar_wait_mma(&betaready, bcnt & 1);
         ++bcnt;
         for (int a = 0; a < 2 && a < ncm; ++a) issue_yhat(a, 0);
         for (int c = 0; c < ncm; ++c) {
@@ -340,22 +373,22 @@ __global__ void __launch_bounds__(224, 2)
     // ------------------------------------------------------------ consumers
     const uint32_t lanebase = tbase + ((uint32_t)(32 * warp) << 16);
     const float qnan = __int_as_float(0x7fc00000);
-    // ring: slot s = [128 residuals f32][128 date indices u16]; this thread's
-    // residual of slot s at rbase + s*RSLOT, its date at +dofs
+    // ring: slot s = 128 residuals f32, this thread's at rbase + s*RSLOT;
+    // history validity: 16 bits per chunk, this thread's at vbase + c*VSLOT
     const uint32_t rbase = sm100::smem_u32(ring) + 4 * tid;
     const uint32_t rend = rbase + hcap * C::RSLOT;
-    const uint32_t dofs = 512 - 2 * tid;
+    const uint32_t vbase = sm100::smem_u32(vmask) + 2 * tid;
     int ys = 0;
     uint32_t yph = 0, opcnt = 0, yuse = 0, acnt = 0;
     // 32-bit shared addresses of the barriers this warp waits on / arrives at
     const uint32_t a_yfull = sm100::smem_u32(&yfull[0]), a_yempty = sm100::smem_u32(&yempty[0]);
-    const uint32_t a_opfull = sm100::smem_u32(&opfull), a_opfree = sm100::smem_u32(&opfree);
+    const uint32_t a_opfull = sm100::smem_u32(&opfull[0]), a_opfree = sm100::smem_u32(&opfree[0]);
     const uint32_t a_yhfull = sm100::smem_u32(&yhfull[0]), a_yhfree = sm100::smem_u32(&yhfree[0]);
     const uint32_t a_accready = sm100::smem_u32(&accready), a_betaready = sm100::smem_u32(&betaready);
     const uint32_t ybuf0 = sm100::smem_u32(ystages);
 
     auto yadvance = [&]() {
-      if (++ys == C::SY) {
+      if (++ys == SY) {
         ys = 0;
         yph ^= 1;
       }
@@ -363,6 +396,19 @@ __global__ void __launch_bounds__(224, 2)
     auto warp_arrive = [&](uint32_t bar) {
       __syncwarp();
       if (lane == 0) sm100::mbar_arrive_a(bar);
+    };
+    // wait until the MMA has released the operand buffer of chunk opcnt
+    auto opbuf_acquire = [&]() -> uint8_t * {
+      const uint32_t ob = NOP == 2 ? (opcnt & 1) : 0;
+      const uint32_t par = NOP == 2 ? ((opcnt >> 1) & 1) : (opcnt & 1);
+      sm100::mbar_wait_a(a_opfree + 8 * ob, par ^ 1);
+      return opb + ob * C::OPBUF;
+    };
+    auto opbuf_publish = [&]() {
+      const uint32_t ob = NOP == 2 ? (opcnt & 1) : 0;
+      sm100::fence_proxy_async_smem();
+      warp_arrive(a_opfull + 8 * ob);
+      ++opcnt;
     };
     auto write_beta_operand = [&](const float (&bt)[K], float off) {
       // A3 row = [bh | bh | bh | bm | bm | bl | 0...] (6 blocks of K, KY cols);
@@ -427,7 +473,7 @@ __global__ void __launch_bounds__(224, 2)
             }
           }
         }
-        sm100::mbar_wait_a(a_opfree, (opcnt & 1) ^ 1);
+        uint8_t *const ob = opbuf_acquire();
 #pragma unroll 1
         for (int hf = 0; hf < 2; ++hf) {  // two halves of 8 dates: half the hot code
           float yv[8];
@@ -448,16 +494,14 @@ __global__ void __launch_bounds__(224, 2)
           }
 #pragma unroll
           for (int q = 0; q < 4; ++q) mw[q] = pack_hi16(mf[2 * q], mf[2 * q + 1]);
-          *reinterpret_cast<uint4 *>(opb + sm100::kmajor_off(tid, 8 * hf, 128)) = make_uint4(mw[0], mw[1], mw[2], mw[3]);
+          *reinterpret_cast<uint4 *>(ob + sm100::kmajor_off(tid, 8 * hf, 128)) = make_uint4(mw[0], mw[1], mw[2], mw[3]);
 #pragma unroll
           for (int q = 0; q < 2; ++q)
-            *reinterpret_cast<uint4 *>(opb + C::A1_BYTES + sm100::kmajor_off(tid, 16 * hf + 8 * q, 128)) =
+            *reinterpret_cast<uint4 *>(ob + C::A1_BYTES + sm100::kmajor_off(tid, 16 * hf + 8 * q, 128)) =
                 make_uint4(yw[4 * q], yw[4 * q + 1], yw[4 * q + 2], yw[4 * q + 3]);
         }
         warp_arrive(a_yempty + 8 * ys);  // every loaded value has been consumed
-        sm100::fence_proxy_async_smem();
-        warp_arrive(a_opfull);
-        ++opcnt;
+        opbuf_publish();
         yadvance();
       }
       sm100::mbar_wait_a(a_accready, acnt & 1);
@@ -538,10 +582,12 @@ __global__ void __launch_bounds__(224, 2)
         sm100::mbar_wait_a(a_yfull + 8 * ys, yph);
         wait_yhat();
         const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
-        sm100::mbar_wait_a(a_opfree, (opcnt & 1) ^ 1);
+        uint8_t *const ob = opbuf_acquire();
+        uint32_t vm = 0;  // validity of the chunk's 16 dates
 #pragma unroll 1
         for (int hf = 0; hf < 2; ++hf) {
           float yh[8], yv[8];
+          uint32_t m8 = 0;  // bit 9+d: date d valid (ring advances accumulated)
           load_yhat8(hf, yh);
 #pragma unroll
           for (int d = 0; d < 8; ++d) yv[d] = Ys[(8 * hf + d) * 128 + tid];  // dates >= n read as NaN (hmap)
@@ -557,23 +603,25 @@ __global__ void __launch_bounds__(224, 2)
             rs3[3 * d] = rh;
             rs3[3 * d + 1] = rm;
             rs3[3 * d + 2] = t1 - rm;
-            sts_f32_if(wa, r, v);
-            sts_u16_if(wa + dofs, (uint16_t)(c * C::DC + 8 * hf + d), v);
-            wa += v ? C::RSLOT : 0u;
+            const uint32_t inc = v ? C::RSLOT : 0u;
+            sts_f32_inc(wa, r, inc);
+            m8 += inc << d;
+            wa += inc;
             wa = (wa == rend) ? rbase : wa;
-            cr += v;
           }
+          static_assert(C::RSLOT == 512, "m8 packs the advances as bit 9 + d");
+          cr += __popc(m8);
+          vm |= (m8 >> 9) << (8 * hf);
 #pragma unroll
           for (int q = 0; q < 3; ++q)
-            *reinterpret_cast<uint4 *>(opb + sm100::kmajor_off(tid, 24 * hf + 8 * q, 128)) =
+            *reinterpret_cast<uint4 *>(ob + sm100::kmajor_off(tid, 24 * hf + 8 * q, 128)) =
                 make_uint4(pack_hi16(rs3[8 * q], rs3[8 * q + 1]), pack_hi16(rs3[8 * q + 2], rs3[8 * q + 3]),
                            pack_hi16(rs3[8 * q + 4], rs3[8 * q + 5]), pack_hi16(rs3[8 * q + 6], rs3[8 * q + 7]));
         }
+        sts_u16(vbase + c * C::VSLOT, (uint16_t)vm);
         release_yhat();
         warp_arrive(a_yempty + 8 * ys);  // every loaded value has been consumed
-        sm100::fence_proxy_async_smem();
-        warp_arrive(a_opfull);
-        ++opcnt;
+        opbuf_publish();
         yadvance();
       }
       sm100::mbar_wait_a(a_accready, acnt & 1);
@@ -619,12 +667,18 @@ __global__ void __launch_bounds__(224, 2)
       float W = 0.f;
       uint32_t ra;
       {
+        // walk back from the newest history residual; its date is the
+        // highest set bit of the chunk masks (scanned from the last chunk)
         const int nseed = deg ? 0 : hh - 1;
         uint32_t a = wa;
-        for (int q = 0; q < nseed; ++q) a = (a == rbase ? rend : a) - C::RSLOT;  // back nseed slots
-        ra = (a == rbase ? rend : a) - C::RSLOT;                                 // rank cr - hh
+        int cm = nch;
+        uint32_t bits = 0;
         for (int q = 0; q < nseed; ++q) {
-          const int t = lds_u16(a + dofs);
+          a = (a == rbase ? rend : a) - C::RSLOT;
+          while (bits == 0 && cm > 0) bits = (uint32_t)lds_u16(vbase + (--cm) * C::VSLOT);
+          const int d = 31 - __clz(bits);
+          bits ^= 1u << d;
+          const int t = cm * C::DC + d;
           const float *xr = p.X + (size_t)t * p.KP;
           float corr = 0.f;
 #pragma unroll
@@ -636,9 +690,8 @@ __global__ void __launch_bounds__(224, 2)
           const float r = lds_f32(a) - corr;
           sts_f32(a, r);
           W += r;
-          a += C::RSLOT;
-          a = (a == rend) ? rbase : a;
         }
+        ra = (a == rbase ? rend : a) - C::RSLOT;  // rank cr - hh
         if (deg) ra = wa;
         // the window of j = 0 drops nothing: the slot of rank nbar - h (or
         // the write slot for invalid pixels) reads as 0 at the first step
@@ -680,16 +733,18 @@ __global__ void __launch_bounds__(224, 2)
 #pragma unroll
           for (int d = 0; d < 8; ++d) yv[d] = Ys[(8 * hf + d) * 128 + tid];  // dates >= N read as NaN (TMA OOB)
           if (fast) {
+            uint32_t adv = 0;  // ring bytes advanced = valid dates * RSLOT
 #pragma unroll
             for (int d = 0; d < 8; ++d) {
               const float y = yv[d];
               const bool v = (y == y);
               const float r = (y - c0) - yh[d];
               const float old = lds_f32(ra);  // rank cr - h (zeroed phantom at j = 0)
-              sts_f32_if(wa, r, v);
               const uint32_t inc = v ? C::RSLOT : 0u;
+              sts_f32_inc(wa, r, inc);
               wa += inc;
               ra += inc;
+              adv += inc;
               wa = (wa == rend) ? rbase : wa;
               ra = (ra == rend) ? rbase : ra;
               if (v) W += r - old;
@@ -700,8 +755,8 @@ __global__ void __launch_bounds__(224, 2)
               const bool cand = v && first < 0 && fabsf(m) > lam_lo;
               first = cand ? c * C::DC + 8 * hf + d : first;
               mfirst = cand ? m : mfirst;
-              cr += v;
             }
+            cr += adv >> 9;
           } else {
 #pragma unroll
             for (int d = 0; d < 8; ++d) {
@@ -709,7 +764,7 @@ __global__ void __launch_bounds__(224, 2)
               const bool v = (y == y);
               const float r = (y - c0) - yh[d];
               const float old = lds_f32(ra);
-              sts_f32_if(wa, r, v);
+              sts_f32_inc(wa, r, v ? C::RSLOT : 0u);
               const uint32_t wn = wa + C::RSLOT, rn = ra + C::RSLOT;
               wa = v ? (wn == rend ? rbase : wn) : wa;
               ra = v ? (rn == rend ? rbase : rn) : ra;
