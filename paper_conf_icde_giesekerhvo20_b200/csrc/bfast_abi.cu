@@ -47,7 +47,8 @@ int fail(int status, const char *fmt, ...) {
                   "%s: %s (%s:%d)", #expr, cudaGetErrorString(e_), __FILE__, __LINE__); \
   } while (0)
 
-constexpr int kMaxSmem = 227 * 1024;
+constexpr int kMaxSmem = 227 * 1024;    // per CTA
+constexpr size_t kSmemPerSM = 228 * 1024;  // per SM (B200)
 
 int validate_scalar(int64_t N, const double *dates, int32_t n_hist, int32_t k, float h,
                     float lambda) {
@@ -331,6 +332,10 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
       CUDA_TRY(cudaFuncGetAttributes(&fa, bfast::monitor_tc_kernel<K>));
       CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_tc_kernel<K>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                     kMaxSmem - (int)fa.sharedSizeBytes));
+      // all of the unified L1/shared array as shared memory: the stack is
+      // streamed by TMA, nothing is reused through L1
+      CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_tc_kernel<K>, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                    (int)cudaSharedmemCarveoutMaxShared));
     }
     configured_dev = pl.device;
   }
@@ -339,33 +344,47 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
   // tensor-core path on the full 128-pixel tiles when the stack rows allow
   // 16-byte bulk copies; SIMT kernel on the ragged tail (or everything)
   const int tc_hcap = pl.hcap;
-  // shared-memory layout: two CTAs per SM hide each other's latencies
-  // (measured 1.5x over one), so take the first layout that fits twice.
-  // Two stack stages already cover the HBM latency of this compute-bound
-  // kernel (2 and 4 stages time alike); double operand buffers let the
-  // consumers fill chunk c+1 while the MMA still reads chunk c.
-  auto fits2 = [&](size_t b) { return (b + 1024) * 2 + 2048 <= (size_t)kMaxSmem; };
-  int tc_sy = 2, tc_nop = 2, per_sm = 1;
+  // shared-memory layout and CTAs per SM.  Co-resident CTAs hide each
+  // other's latencies (1 -> 2 -> 3 CTAs/SM measured 1.5x, then 1.08x), so
+  // take the layout that admits the most CTAs, preferring among equals the
+  // earlier entry: two stack stages already cover the HBM latency of this
+  // compute-bound kernel (2 and 4 stages time alike), double operand buffers
+  // let the consumers fill chunk c+1 while the MMA still reads chunk c.
+  // Limits: registers (80 x 256 threads at launch -> 3 CTAs), shared memory
+  // (228 KB per SM, 1 KB reserved + 1 KB static per CTA), TMEM (512 columns).
+  // (The occupancy API is not used: it does not model setmaxnreg kernels.)
+  int tc_sy = 2, tc_nop = 1, per_sm = 0;
   {
     const int cand[4][2] = {{2, 2}, {2, 1}, {3, 2}, {3, 1}};
-    for (auto &c : cand)
-      if (fits2(TC::smem_bytes(tc_hcap, pl.nch, c[0], c[1]))) {
+    const int reg_cap = 65536 / (bfast::kTcThreads * bfast::kTcLaunchRegs);
+    const int tmem_cap = 512 / TC::TMEM_COLS;
+    for (auto &c : cand) {
+      const size_t b = TC::smem_bytes(tc_hcap, pl.nch, c[0], c[1]);
+      if (b + 1024 > (size_t)kMaxSmem) continue;
+      int nb = (int)(kSmemPerSM / (b + 2048));
+      nb = std::min(nb, std::min(reg_cap, tmem_cap));
+      if (std::getenv("BFAST_VERBOSE"))
+        std::fprintf(stderr, "bfast: candidate sy=%d nop=%d smem=%zu ctas/sm=%d\n", c[0], c[1], b, nb);
+      if (nb > per_sm) {
+        per_sm = nb;
         tc_sy = c[0];
         tc_nop = c[1];
-        per_sm = 2;
-        break;
       }
+    }
   }
   if (const char *lay = std::getenv("BFAST_TC_LAYOUT")) {  // experiments: "sy,nop,per_sm"
     int a = 0, b = 0, c = 0;
-    if (std::sscanf(lay, "%d,%d,%d", &a, &b, &c) == 3 && a >= 2 && a <= 4 && b >= 1 && b <= 2 && c >= 1 && c <= 2) {
+    if (std::sscanf(lay, "%d,%d,%d", &a, &b, &c) == 3 && a >= 2 && a <= 4 && b >= 1 && b <= 2 && c >= 1 && c <= 3) {
       tc_sy = a;
       tc_nop = b;
       per_sm = c;
     }
   }
   const size_t tc_smem = TC::smem_bytes(tc_hcap, pl.nch, tc_sy, tc_nop);
-  const bool tc_ok = pl.dtab && pl.mode != 1 && (prm.ldY % 4) == 0 &&
+  if (std::getenv("BFAST_VERBOSE"))
+    std::fprintf(stderr, "bfast: tc layout k=%d hcap=%d nch=%d sy=%d nop=%d smem=%zu per_sm=%d tmem_cols=%d\n", pl.k,
+                 tc_hcap, pl.nch, tc_sy, tc_nop, tc_smem, per_sm, TC::TMEM_COLS);
+  const bool tc_ok = per_sm > 0 && pl.dtab && pl.mode != 1 && (prm.ldY % 4) == 0 &&
                      ((uintptr_t)(prm.Y + prm.p0) % 16) == 0 && tc_smem + 1024 <= (size_t)kMaxSmem;
   CUtensorMap ymap, hmap;  // full stack; history only (dates >= n out of bounds)
   const bool tma_ok = tc_ok && make_stack_map(&ymap, prm.Y + prm.p0, prm.ldY, prm.P, pl.N) &&
@@ -394,7 +413,7 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
     const int64_t grid = std::min<int64_t>(ntiles, (int64_t)sms * per_sm);
     bfast::MonitorParams q = prm;
     q.hcap = tc_hcap;
-    bfast::monitor_tc_kernel<K><<<(unsigned)grid, 224, tc_smem, st>>>(q, tb, ymap, hmap);
+    bfast::monitor_tc_kernel<K><<<(unsigned)grid, bfast::kTcThreads, tc_smem, st>>>(q, tb, ymap, hmap);
     CUDA_TRY(cudaGetLastError());
     ++launches;
   }

@@ -46,6 +46,16 @@
 
 namespace bfast {
 
+// CTA = consumer warpgroup (warps 0-3, one pixel per thread) + producer
+// warpgroup (warp 4 stack TMA, 5 table copies, 6 MMA issue, 7 idle).  At
+// launch every thread holds 80 registers (3 CTAs x 256 threads); the
+// producers drop to kTcAuxRegs, the consumers rise to kTcConsumerRegs
+// (80*256 = 128*kTcAuxRegs + 128*kTcConsumerRegs).
+constexpr int kTcThreads = 256;
+constexpr int kTcLaunchRegs = 80;
+constexpr int kTcAuxRegs = 32;
+constexpr int kTcConsumerRegs = 2 * kTcLaunchRegs - kTcAuxRegs;
+
 template <int K>
 struct TcCfg {
   static constexpr int k = (K - 2) / 2;
@@ -55,8 +65,14 @@ struct TcCfg {
   static constexpr int KY = ((6 * K + 15) / 16) * 16;      // yhat GEMM K
   static constexpr int KB3 = ((3 * K + 15) / 16) * 16;     // refinement GEMM N (x hi|mid|lo)
   static constexpr int DC = 16;                            // dates per chunk
-  static constexpr int COL_G = 0, COL_B = NGp, COL_DB = NGp + KB, COL_Y = NGp + KB + KB3;
-  static constexpr int COLS_USED = COL_Y + 2 * DC;
+  // TMEM columns.  Pass 1 accumulates the Gram moments and the moment b;
+  // pass 2 the refinement moment, two yhat slots and the beta operand (the
+  // A operand of the yhat GEMM, bf16 pairs).  The consumers read G and b in
+  // the solve before any pass-2 MMA is issued, so pass 2 reuses their columns.
+  static constexpr int COL_G = 0, COL_B = NGp;
+  static constexpr int COL_DB = 0, COL_Y = KB3, COL_A3 = KB3 + 2 * DC;
+  static constexpr int COLS_P1 = NGp + KB, COLS_P2 = COL_A3 + KY / 2;
+  static constexpr int COLS_USED = COLS_P1 > COLS_P2 ? COLS_P1 : COLS_P2;
   static constexpr int TMEM_COLS = COLS_USED <= 32 ? 32 : COLS_USED <= 64 ? 64 : COLS_USED <= 128 ? 128
                                    : COLS_USED <= 256 ? 256 : 512;
   static constexpr int B1_BYTES = NGp * DC * 2;            // [NGp x 16] bf16
@@ -75,13 +91,12 @@ struct TcCfg {
   static constexpr int A2_BYTES = 128 * 2 * DC * 2;
   static constexpr int A4_BYTES = 128 * 3 * DC * 2;        // r0 hi|mid|lo per date
   static constexpr int OPBUF = A1_BYTES + A2_BYTES > A4_BYTES ? A1_BYTES + A2_BYTES : A4_BYTES;
-  static constexpr int A3_BYTES = 128 * KY * 2;
   static constexpr int RSLOT = 128 * 4;                   // ring slot: one residual per pixel
   static constexpr int VSLOT = 128 * 2;                   // validity mask: 16 bits per pixel per chunk
   // sy stack stages, nop operand buffers (2: the consumers fill one while the
   // MMA reads the other), the MOSUM ring of hcap slots, nch history masks
   static constexpr size_t smem_bytes(int hcap, int nch, int sy, int nop) {
-    return (size_t)sy * YBYTES + (size_t)ST * TSTAGE + (size_t)nop * OPBUF + A3_BYTES + (size_t)hcap * RSLOT +
+    return (size_t)sy * YBYTES + (size_t)ST * TSTAGE + (size_t)nop * OPBUF + (size_t)hcap * RSLOT +
            (size_t)nch * VSLOT;
   }
 };
@@ -170,7 +185,7 @@ __device__ __forceinline__ float bf16_round(float v) {
 }
 
 template <int K>
-__global__ void __launch_bounds__(224, 2)
+__global__ void __launch_bounds__(kTcThreads, 3)
     monitor_tc_kernel(MonitorParams p, TcTables tb, const __grid_constant__ CUtensorMap ymap,
                       const __grid_constant__ CUtensorMap hmap) {
   using C = TcCfg<K>;
@@ -182,8 +197,7 @@ __global__ void __launch_bounds__(224, 2)
   uint8_t *ystages = smem;
   uint8_t *tstages = ystages + SY * C::YBYTES;
   uint8_t *opb = tstages + C::ST * C::TSTAGE;
-  uint8_t *a3 = opb + NOP * C::OPBUF;
-  uint8_t *ring = a3 + C::A3_BYTES;
+  uint8_t *ring = opb + NOP * C::OPBUF;
   uint8_t *vmask = ring + hcap * C::RSLOT;
   constexpr int NCW = 4;  // consumer warps
 
@@ -214,6 +228,10 @@ __global__ void __launch_bounds__(224, 2)
   const uint32_t tbase = tmem_base_s;
   const int n = p.n, N = p.N, nch = tb.nch, ncm = tb.ncm;
 
+  if (warp >= NCW) {
+    // producer warpgroup: three single-thread roles need few registers; hand
+    // them to the consumer warpgroup (3 CTAs per SM fit the register file)
+    sm100::setmaxnreg_dec<kTcAuxRegs>();
   if (warp == 4) {
     // ------------------------------------------------------------ stack producer
     if (lane == 0) {
@@ -277,7 +295,7 @@ __global__ void __launch_bounds__(224, 2)
       const uint32_t idB = sm100::idesc_bf16_f32(128, C::KB);
       const uint32_t idY = sm100::idesc_bf16_f32(128, C::DC);
       const uint32_t idR = sm100::idesc_bf16_f32(128, C::KB3);
-      const uint32_t aop = sm100::smem_u32(opb), a3s = sm100::smem_u32(a3), tss = sm100::smem_u32(tstages);
+      const uint32_t aop = sm100::smem_u32(opb), tss = sm100::smem_u32(tstages);
       int ts = 0;
       uint32_t tph = 0, opcnt = 0, yissue = 0, bcnt = 0;
       auto tslot = [&](int ahead, uint32_t &par) {
@@ -313,8 +331,8 @@ __global__ void __launch_bounds__(224, 2)
         const uint32_t b3 = tss + s * C::TSTAGE + tab_off;
 #pragma unroll
         for (int q = 0; q < C::KY / 16; ++q)
-          sm100::umma_bf16(tbase + C::COL_Y + slot * C::DC, sm100::smem_desc(a3s + q * 2 * 2048, 2048, 128),
-                           sm100::smem_desc(b3 + q * 2 * 256, 256, 128), idY, q > 0);
+          sm100::umma_bf16_ts(tbase + C::COL_Y + slot * C::DC, tbase + C::COL_A3 + 8 * q,
+                              sm100::smem_desc(b3 + q * 2 * 256, 256, 128), idY, q > 0);
         sm100::umma_commit(&yhfull[slot]);
         ++yissue;
       };
@@ -369,8 +387,10 @@ __global__ void __launch_bounds__(224, 2)
         }
       }
     }
+  }  // warp 7 idles: it completes the producer warpgroup
   } else {
     // ------------------------------------------------------------ consumers
+    sm100::setmaxnreg_inc<kTcConsumerRegs>();
     const uint32_t lanebase = tbase + ((uint32_t)(32 * warp) << 16);
     const float qnan = __int_as_float(0x7fc00000);
     // ring: slot s = 128 residuals f32, this thread's at rbase + s*RSLOT;
@@ -411,7 +431,7 @@ __global__ void __launch_bounds__(224, 2)
       ++opcnt;
     };
     auto write_beta_operand = [&](const float (&bt)[K], float off) {
-      // A3 row = [bh | bh | bh | bm | bm | bl | 0...] (6 blocks of K, KY cols);
+      // A3 row (TMEM) = [bh | bh | bh | bm | bm | bl | 0...] (6 blocks of K, KY bf16);
       // `off` would fold an offset into the intercept (kept at 0: the GEMM's
       // accumulation error scales with |yhat|, so the offset stays outside)
       float h[K], m[K], l[K];
@@ -434,10 +454,14 @@ __global__ void __launch_bounds__(224, 2)
         w[j] = sm100::pack_bf16x2(e[0], e[1]);
       }
 #pragma unroll
-      for (int q = 0; q < C::KY / 8; ++q)
-        *reinterpret_cast<uint4 *>(a3 + sm100::kmajor_off(tid, 8 * q, 128)) =
-            make_uint4(w[4 * q], w[4 * q + 1], w[4 * q + 2], w[4 * q + 3]);
-      sm100::fence_proxy_async_smem();
+      for (int q = 0; q < C::KY / 16; ++q) {
+        uint32_t w8[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) w8[i] = w[8 * q + i];
+        sm100::tmem_st8(lanebase + C::COL_A3 + 8 * q, w8);  // this pixel's row of the A operand
+      }
+      sm100::tmem_st_wait();
+      sm100::tc_fence_before();
       warp_arrive(a_betaready);
     };
     auto wait_yhat = [&]() {
