@@ -434,9 +434,9 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
   }
   // fp64 refit of flagged pixels; exits at once when the list is empty
   const int rwarps = 4;
-  const size_t rsmem = (size_t)rwarps * (pl.N + 1) * sizeof(double);
+  const size_t rsmem = (size_t)rwarps * bfast::refit_warp_doubles((int)pl.N) * sizeof(double);
   if (rsmem > (size_t)kMaxSmem) return fail(BFAST_EUNSUPPORTED, "refit smem too large");
-  bfast::refit_fp64_kernel<K><<<sms * 4, rwarps * 32, rsmem, st>>>(prm);
+  bfast::refit_fp64_kernel<K><<<sms * 8, rwarps * 32, rsmem, st>>>(prm);
   CUDA_TRY(cudaGetLastError());
   CUDA_TRY(cudaEventRecord(pl.scratch_free, st));
   g_launches = launches + 1;

@@ -53,7 +53,10 @@ namespace bfast {
 // (80*256 = 128*kTcAuxRegs + 128*kTcConsumerRegs).
 constexpr int kTcThreads = 256;
 constexpr int kTcLaunchRegs = 80;
-constexpr int kTcAuxRegs = 32;
+#ifndef BFAST_TC_AUX_REGS
+#define BFAST_TC_AUX_REGS 32
+#endif
+constexpr int kTcAuxRegs = BFAST_TC_AUX_REGS;
 constexpr int kTcConsumerRegs = 2 * kTcLaunchRegs - kTcAuxRegs;
 
 template <int K>
@@ -585,10 +588,19 @@ __global__ void __launch_bounds__(kTcThreads, 3)
       bool deg = (nbar < K + 1) || (h < 1);
       float beta[K];
       bool refit = false;
+#ifdef BFAST_REFIT_WHY
+      uint32_t why = 0;  // diagnostics build: which trigger sent the pixel to the refit
+#define BFAST_WHY(b) why |= (b)
+#else
+#define BFAST_WHY(b)
+#endif
       {
         const float minratio = chol_factor<K, float>(A);
         chol_solve<K, float>(A, b, beta);
-        if (!deg && !(minratio >= (float)kRefitRatio)) refit = true;
+        if (!deg && !(minratio >= (float)kRefitRatio)) {
+          refit = true;
+          BFAST_WHY(0x10);
+        }
         if (deg) {
 #pragma unroll
           for (int i = 0; i < K; ++i) beta[i] = 0.f;
@@ -677,12 +689,18 @@ __global__ void __launch_bounds__(kTcThreads, 3)
         sigma = sqrtf(fmaxf(s2 - lin, 0.f) / (float)(nbar - K));
         // sigma^2 = s2 - lin cancels when the refinement step is large next to
         // the residual sum: the fp32 sigma-hat is then unreliable -> fp64 refit
-        if (!(lin <= 1e-2f * s2)) refit = true;
+        if (!(lin <= 1e-2f * s2)) {
+          refit = true;
+          BFAST_WHY(0x20);
+        }
       }
       if (!deg && !(sigma > 1e-4f * ymax)) deg = true;
       // noise within 2e-3 of the signal scale: fp32 fitted values (~1e-7 |y|)
       // are no longer negligible next to sigma-hat -> fp64 refit (R12)
-      if (!deg && !(sigma > 2e-3f * ymax)) refit = true;
+      if (!deg && !(sigma > 2e-3f * ymax)) {
+        refit = true;
+        BFAST_WHY(0x40);
+      }
       const float inv_scale = 1.0f / (sigma * sqrtf((float)nbar));
       sm100::tc_fence_before();
       write_beta_operand(beta, 0.f);
@@ -823,7 +841,11 @@ __global__ void __launch_bounds__(kTcThreads, 3)
         p.out_mag[pix] = deg ? qnan : msum / (float)(Nbar - nbar);
         if (p.out_sigma) p.out_sigma[pix] = fit_ok ? sigma : qnan;
         if (p.out_nbar) p.out_nbar[pix] = nbar;
+#ifdef BFAST_REFIT_WHY
+        if (p.out_flags) p.out_flags[pix] = (deg ? 1u : 0u) | why | (tie ? 0x80u : 0u);
+#else
         if (p.out_flags) p.out_flags[pix] = deg ? 1u : 0u;
+#endif
         store_beta<K, float>(p, pix, beta, c0, fit_ok);
       }
       const bool want = (refit || tie) && fit_ok && inside;

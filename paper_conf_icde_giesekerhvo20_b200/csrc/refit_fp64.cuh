@@ -26,13 +26,19 @@ __device__ __forceinline__ double warp_sum(double v) {
   return v;
 }
 
+// shared memory per warp, in doubles: prefix sums [N + 1] + column [N] f32
+__host__ __device__ constexpr size_t refit_warp_doubles(int N) { return (size_t)(N + 1) + ((size_t)N + 1) / 2; }
+
 template <int K>
 __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
-  extern __shared__ double rbuf_all[];  // [warps][N + 1] compacted residual prefix sums
+  // per warp: [N + 1] compacted residual prefix sums (fp64), then the
+  // pixel's column [N] (fp32), staged once so every pass reads shared memory
+  extern __shared__ double rbuf_all[];
   const int lane = threadIdx.x & 31;
   const int wib = threadIdx.x >> 5;
   const int wpb = blockDim.x >> 5;
-  double *S = rbuf_all + (size_t)wib * (p.N + 1);
+  double *S = rbuf_all + (size_t)wib * refit_warp_doubles(p.N);
+  float *Yc = reinterpret_cast<float *>(S + p.N + 1);
   const int count = *p.refit_count;
   const int n = p.n, N = p.N;
   const int64_t ldY = p.ldY;
@@ -40,7 +46,25 @@ __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
 
   for (int item = blockIdx.x * wpb + wib; item < count; item += gridDim.x * wpb) {
     const int64_t pix = p.refit_list[item];  // absolute pixel index
-    const float *ycol = p.Y + pix;
+    {
+      // the column is N strided loads (one sector each): issue them all
+      // before any is used, so the pixel pays one memory latency, not N/32
+      const float *ycol = p.Y + pix;
+      float v4[4];
+      for (int t0 = 0; t0 < N; t0 += 128) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int t = t0 + 32 * u + lane;
+          v4[u] = t < N ? __ldcs(ycol + (int64_t)t * ldY) : 0.f;
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int t = t0 + 32 * u + lane;
+          if (t < N) Yc[t] = v4[u];
+        }
+      }
+      __syncwarp();
+    }
     // ---- history: offset, Gram, moment (fp64)
     double A[Tri<K>::kN], b[K];
 #pragma unroll
@@ -53,7 +77,7 @@ __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
     double ymax = 0.0;
     for (int t0 = 0; t0 < n; t0 += 32) {
       const int t = t0 + lane;
-      const float yf = t < n ? ycol[(int64_t)t * ldY] : __int_as_float(0x7fc00000);
+      const float yf = t < n ? Yc[t] : __int_as_float(0x7fc00000);
       const bool v = (yf == yf);
       const unsigned bal = __ballot_sync(0xffffffffu, v);
       if (!bal) continue;
@@ -97,7 +121,7 @@ __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
     __syncwarp();  // S[0] is read by every lane below
     for (int t0 = 0; t0 < N; t0 += 32) {
       const int t = t0 + lane;
-      const float yf = t < N ? ycol[(int64_t)t * ldY] : __int_as_float(0x7fc00000);
+      const float yf = t < N ? Yc[t] : __int_as_float(0x7fc00000);
       const bool v = (yf == yf);
       const unsigned bal = __ballot_sync(0xffffffffu, v);
       double r = 0.0;
@@ -152,7 +176,7 @@ __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
       int target = nbar + jstar, seen = 0;
       for (int t0 = 0; t0 < N; t0 += 32) {
         const int t = t0 + lane;
-        const float yf = t < N ? ycol[(int64_t)t * ldY] : __int_as_float(0x7fc00000);
+        const float yf = t < N ? Yc[t] : __int_as_float(0x7fc00000);
         const unsigned bal = __ballot_sync(0xffffffffu, yf == yf);
         const int c = __popc(bal);
         if (seen + c > target) {
@@ -168,7 +192,11 @@ __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
       p.out_break[pix] = deg ? -2 : brk;
       p.out_mag[pix] = deg ? (float)qnan : (float)(msum / (double)J);
       if (p.out_sigma) p.out_sigma[pix] = (float)sigma;
+#ifdef BFAST_REFIT_WHY
+      if (p.out_flags) p.out_flags[pix] = (uint8_t)((p.out_flags[pix] & 0xF0u) | (deg ? 1u : 0u) | 2u);
+#else
       if (p.out_flags) p.out_flags[pix] = (uint8_t)((deg ? 1u : 0u) | 2u);
+#endif
       if (p.out_beta) {
         float *o = p.out_beta + pix * K;
         const bool rank_def = !(minratio > 1e-9);
