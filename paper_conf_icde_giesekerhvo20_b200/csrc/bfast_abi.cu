@@ -94,7 +94,7 @@ struct bfast_plan {
   cudaEvent_t scratch_free = nullptr;  // orders executions sharing the refit scratch
   // tensor-core path: per-chunk B-operand tables (monitor_tc.cuh)
   uint8_t *dtab = nullptr;
-  size_t tab2_off = 0, tab3_off = 0;
+  size_t tab2_off = 0, taby_off = 0;
   int nch = 0, ncm = 0;
   int mode = 0;  // 0 auto, 1 force SIMT, 2 force tensor cores (BFAST_KERNEL env at plan creation)
   std::mutex mu;
@@ -183,10 +183,6 @@ double bf16_val(uint16_t h) {
   std::memcpy(&f, &u, 4);
   return (double)f;
 }
-void split2(double v, uint16_t &h, uint16_t &l) {
-  h = bf16_rne(v);
-  l = bf16_rne(v - bf16_val(h));
-}
 void split3(double v, uint16_t &h, uint16_t &m, uint16_t &l) {
   h = bf16_rne(v);
   m = bf16_rne(v - bf16_val(h));
@@ -196,8 +192,17 @@ inline size_t kmaj(int row, int k, int rows) { return sm100::kmajor_off(row, k, 
 
 // Chunk tables of the tensor-core kernel (monitor_tc.cuh): B operands in the
 // canonical K-major layout, fp64 values split into bf16 parts.
+//   tab1[c] (history chunk c, pass 1): F_hi | F_mid | F_lo ([NGn x 16] each,
+//           row q = moment function f_q (the last one the constant 1),
+//           column d = date 16c + d), then x_hi | x_mid | x_lo ([KBn x 16]
+//           each, row i = basis column i);
+//   tab2[c] (history chunk c, pass 2): the yhat table [16 x KY] of its dates
+//           (row d = date, K index = 6 blocks of K: x_hi | x_mid | x_lo |
+//           x_hi | x_mid | x_hi, paired in the GEMM with beta hi | hi | hi |
+//           mid | mid | lo), then x_hi | x_mid | x_lo as in tab1;
+//   taby[c] (monitoring chunk c): the yhat table of dates n + 16c + d.
 template <int K>
-void build_tc_tables(const bfast_plan &pl, std::vector<uint16_t> &tab, size_t &off2, size_t &off3) {
+void build_tc_tables(const bfast_plan &pl, std::vector<uint16_t> &tab, size_t &off2, size_t &offy) {
   using C = bfast::TcCfg<K>;
   const int k = pl.k, n = pl.n, N = (int)pl.N, DC = C::DC;
   const int nch = (n + DC - 1) / DC, ncm = (N - n + DC - 1) / DC;
@@ -211,7 +216,7 @@ void build_tc_tables(const bfast_plan &pl, std::vector<uint16_t> &tab, size_t &o
       x[2 * j + 1] = std::cos(j * th);
     }
   };
-  auto frow = [&](int t, double *f) {  // tau, tau^2, tau sin_j, tau cos_j, sin_m, cos_m
+  auto frow = [&](int t, double *f) {  // tau, tau^2, tau sin_j, tau cos_j, sin_m, cos_m, 1
     const double tau = ((double)(t + 1) - pl.tc) / pl.ts, th = two_pi * pl.dates[t];
     f[0] = tau;
     f[1] = tau * tau;
@@ -223,30 +228,13 @@ void build_tc_tables(const bfast_plan &pl, std::vector<uint16_t> &tab, size_t &o
       f[2 + 2 * k + 2 * (m - 1)] = std::sin(m * th);
       f[3 + 2 * k + 2 * (m - 1)] = std::cos(m * th);
     }
+    f[C::NF] = 1.0;  // the constant function: its masked moment is nbar
   };
-  const size_t T1 = C::TAB1 / 2, T2 = C::TAB2 / 2, T3 = C::TAB3 / 2;
-  tab.assign((size_t)nch * T1 + (size_t)nch * T2 + (size_t)ncm * T3, 0);
+  const size_t T1 = C::TAB1 / 2, T2 = C::TAB2 / 2, TY = C::TABY / 2;
+  tab.assign((size_t)nch * (T1 + T2) + (size_t)ncm * TY, 0);
   off2 = (size_t)nch * T1;
-  off3 = off2 + (size_t)nch * T2;
-  double x[2 + 2 * BFAST_K_MAX_HARMONICS], f[2 + 6 * BFAST_K_MAX_HARMONICS];
-  auto put_b2 = [&](uint16_t *b2, int d, const double *xv) {  // [KB x 32], k = 2d + {yhi, ylo}
-    for (int i = 0; i < K; ++i) {
-      uint16_t h, l;
-      split2(xv[i], h, l);
-      b2[kmaj(i, 2 * d, C::KB)] = h;
-      b2[kmaj(i, 2 * d + 1, C::KB)] = h;
-      b2[kmaj(K + i, 2 * d, C::KB)] = l;
-    }
-  };
-  auto put_br = [&](uint16_t *br, int d, const double *xv) {  // [KB3 x 48], k = 3d + e
-    for (int i = 0; i < K; ++i) {
-      uint16_t h, m, l;
-      split3(xv[i], h, m, l);
-      const uint16_t blk[3] = {h, m, l};
-      for (int b = 0; b < 3; ++b)
-        for (int e = 0; e < 3; ++e) br[kmaj(b * K + i, 3 * d + e, C::KB3)] = blk[b];
-    }
-  };
+  offy = off2 + (size_t)nch * T2;
+  double x[2 + 2 * BFAST_K_MAX_HARMONICS], f[3 + 6 * BFAST_K_MAX_HARMONICS];
   auto put_b3 = [&](uint16_t *b3, int d, const double *xv) {  // [16 x KY]: xh|xm|xl|xh|xm|xh
     for (int i = 0; i < K; ++i) {
       uint16_t h, m, l;
@@ -255,30 +243,35 @@ void build_tc_tables(const bfast_plan &pl, std::vector<uint16_t> &tab, size_t &o
       for (int b = 0; b < 6; ++b) b3[kmaj(d, b * K + i, C::DC)] = blk[b];
     }
   };
+  auto put_bx = [&](uint16_t *bx, int d, const double *xv) {  // 3 x [KBn x 16]
+    for (int i = 0; i < K; ++i) {
+      uint16_t h, m, l;
+      split3(xv[i], h, m, l);
+      const uint16_t prt[3] = {h, m, l};
+      for (int e = 0; e < 3; ++e) bx[e * C::BX_BYTES / 2 + kmaj(i, d, C::KBn)] = prt[e];
+    }
+  };
   for (int c = 0; c < nch; ++c) {
-    uint16_t *b1 = tab.data() + (size_t)c * T1;
-    uint16_t *b2 = b1 + C::B1_BYTES / 2;
-    uint16_t *c2 = tab.data() + off2 + (size_t)c * T2;
-    uint16_t *c3 = c2 + C::BR_BYTES / 2;
+    uint16_t *bf = tab.data() + (size_t)c * T1;
+    uint16_t *t2 = tab.data() + off2 + (size_t)c * T2;
     for (int d = 0; d < DC; ++d) {
       const int t = c * DC + d;
       if (t >= n) continue;
       xrow(t, x);
       frow(t, f);
-      for (int q = 0; q < C::NF; ++q) {
+      for (int q = 0; q <= C::NF; ++q) {
         uint16_t h, m, l;
         split3(f[q], h, m, l);
-        b1[kmaj(q, d, C::NGp)] = h;
-        b1[kmaj(C::NF + q, d, C::NGp)] = m;
-        b1[kmaj(2 * C::NF + q, d, C::NGp)] = l;
+        const uint16_t prt[3] = {h, m, l};
+        for (int e = 0; e < 3; ++e) bf[e * C::BF_BYTES / 2 + kmaj(q, d, C::NGn)] = prt[e];
       }
-      put_b2(b2, d, x);
-      put_br(c2, d, x);
-      put_b3(c3, d, x);
+      put_bx(bf + 3 * C::BF_BYTES / 2, d, x);
+      put_b3(t2, d, x);
+      put_bx(t2 + C::B3_BYTES / 2, d, x);
     }
   }
   for (int c = 0; c < ncm; ++c) {
-    uint16_t *b3 = tab.data() + off3 + (size_t)c * T3;
+    uint16_t *b3 = tab.data() + offy + (size_t)c * TY;
     for (int d = 0; d < DC; ++d) {
       const int t = n + c * DC + d;
       if (t >= N) continue;
@@ -290,21 +283,21 @@ void build_tc_tables(const bfast_plan &pl, std::vector<uint16_t> &tab, size_t &o
 
 int build_tc(bfast_plan &pl) {
   std::vector<uint16_t> tab;
-  size_t o2 = 0, o3 = 0;
+  size_t o2 = 0, oy = 0;
   switch (pl.k) {
-    case 0: build_tc_tables<2>(pl, tab, o2, o3); break;
-    case 1: build_tc_tables<4>(pl, tab, o2, o3); break;
-    case 2: build_tc_tables<6>(pl, tab, o2, o3); break;
-    case 3: build_tc_tables<8>(pl, tab, o2, o3); break;
-    case 4: build_tc_tables<10>(pl, tab, o2, o3); break;
-    case 5: build_tc_tables<12>(pl, tab, o2, o3); break;
-    case 6: build_tc_tables<14>(pl, tab, o2, o3); break;
+    case 0: build_tc_tables<2>(pl, tab, o2, oy); break;
+    case 1: build_tc_tables<4>(pl, tab, o2, oy); break;
+    case 2: build_tc_tables<6>(pl, tab, o2, oy); break;
+    case 3: build_tc_tables<8>(pl, tab, o2, oy); break;
+    case 4: build_tc_tables<10>(pl, tab, o2, oy); break;
+    case 5: build_tc_tables<12>(pl, tab, o2, oy); break;
+    case 6: build_tc_tables<14>(pl, tab, o2, oy); break;
     default: return BFAST_EUNSUPPORTED;
   }
   pl.nch = (pl.n + 15) / 16;
   pl.ncm = ((int)pl.N - pl.n + 15) / 16;
   pl.tab2_off = o2 * 2;
-  pl.tab3_off = o3 * 2;
+  pl.taby_off = oy * 2;
   CUDA_TRY(cudaMalloc(&pl.dtab, tab.size() * 2));
   CUDA_TRY(cudaMemcpy(pl.dtab, tab.data(), tab.size() * 2, cudaMemcpyHostToDevice));
   return BFAST_OK;
@@ -404,7 +397,7 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
     bfast::TcTables tb;
     tb.tab1 = pl.dtab;
     tb.tab2 = pl.dtab + pl.tab2_off;
-    tb.tab3 = pl.dtab + pl.tab3_off;
+    tb.taby = pl.dtab + pl.taby_off;
     tb.nch = pl.nch;
     tb.ncm = pl.ncm;
     tb.ntiles = ntiles;

@@ -4,41 +4,48 @@
 // PAPER.md L134; Fig. 12), re-mapped so that every contraction
 // shared by a 128-pixel tile runs as a tcgen05.mma with fp32 accumulators
 // in Tensor Memory, and the CUDA cores only do per-(pixel, date) scalar
-// work:
+// work, as little of it as the method allows:
 //
 //   masked Gram  A = sum_t v_t x_t x_t^T  (Alg. 1 l.2, Fig. 4)
 //       The K(K+1)/2 entries are linear in NF = 2+6k masked moments
 //       sum_t v_t f_q(t) of the functions f = {tau, tau^2, tau sin_j,
 //       tau cos_j, sin_m, cos_m (m <= 2k)} (product-to-sum identities), so
-//       the tile's Gram is ONE bf16 GEMM: D_G[128 x 3NF] += V[128 x 16] *
-//       F[16 x 3NF] per 16 dates, with V the exact 0/1 mask and F split in
-//       hi+mid+lo bf16 (24-bit mantissa: the products are exact, so the
-//       Gram carries fp32 accumulation error only).
-//   moment b = sum_t v_t y'_t x_t  (Alg. 1 l.4): D_b += [y'hi y'lo] * [xhi xlo]
-//   yhat = X beta (Fig. 12 ker 6): D_y[128 x 16 dates] = [beta hi/mid/lo] *
-//       [x hi/mid/lo] with the 6 cross terms of a 3-way bf16 split
-//       (~24-bit accuracy, fp32 accumulate).
-//   refinement db = sum_t v_t r0_t x_t, r0 = y' - x beta0: a sum with heavy
-//       cancellation (db -> 0 as beta0 -> beta), so both r0 and x are split
-//       3-way (24-bit): D_db[128 x 3K] += [r0 hi,mid,lo per date] * [x hi|mid|lo].
-//   Because the refinement step re-solves with the residual moment, the
-//   16-bit moment only sets beta0; the final beta carries fp32-level error
-//   (DESIGN.md "Numerics").
+//       the tile's Gram is D_G[128 x NF] += V[128 x 16] * F_e[16 x NF],
+//       e = hi, mid, lo (three MMAs on the same exact 0/1 mask operand V;
+//       F split in three bf16 parts: the products are exact, the Gram
+//       carries fp32 accumulation error only).
+//   moment b = sum_t v_t y'_t x_t  (Alg. 1 l.4): y' = y - c (c = the pixel's
+//       first valid value) is split exactly in three bf16 parts by
+//       truncation and x in three rounded parts; the six cross terms above
+//       2^-24 are six MMAs into D_b[128 x K].
+//   Gram and moment alternate between two TMEM accumulator sets (even / odd
+//       chunks), which halves the fp32 accumulation error (DESIGN.md
+//       "Numerics"); the solve adds the two sets.
+//   yhat' = X beta (Fig. 12 ker 6) of the offset data y - c: D_y[128 x 16
+//       dates] = [beta hi/mid/lo] * [x hi/mid/lo] with the 6 cross terms of a
+//       3-way bf16 split (~24-bit accuracy, fp32 accumulate).
 //
-// Roles (160 threads): warps 0-3 own one pixel per thread (TMEM lane =
+// Roles (256 threads): warps 0-3 own one pixel per thread (TMEM lane =
 // pixel row); warp 4 streams 16-date x 128-pixel boxes of the time-major
-// stack (one 2-D TMA copy each) into a 4-stage ring that the consumer warps
-// release as soon as they have read a box; warp 5 streams the chunk's
-// B-operand tables (one 1-D bulk copy each, L2-resident) into a 3-stage ring
-// released by tcgen05.commit of the MMAs that read them; warp 6 issues every
-// tcgen05.mma.  All hand-offs are mbarriers (per-warp arrivals), so no warp
-// ever waits at a CTA-wide barrier inside the date loops.  Thread 0 issues the MMAs after a
-// named barrier and signals completion with tcgen05.commit on mbarriers.
-// Per tile the chunk sequence is: history (Gram+moment), history again
-// (residuals, sigma, refinement moment, MOSUM ring), monitoring (MOSUM,
-// boundary, first break, mean).  The stack is read through a 2-D TMA tensor
-// map whose out-of-bounds fill is NaN, so a ragged last tile needs no
-// special case (its missing pixels are "all missing").
+// stack (one 2-D TMA copy each) into a ring the consumer warps release as
+// soon as they have read a box; warp 5 streams the chunk's B-operand tables
+// (one 1-D bulk copy each, L2-resident) into a ring released by
+// tcgen05.commit of the MMAs that read them; warp 6 issues every
+// tcgen05.mma; warp 7 idles.  All hand-offs are mbarriers (per-warp
+// arrivals), so no warp waits at a CTA-wide barrier inside the date loops.
+//
+// Per tile the chunk sequence is two sweeps:
+//   pass 1, history chunks:  mask + y' operands -> Gram and moment (MMA)
+//   solve:                   fp32 register Cholesky (Alg. 1 l.3-4)
+//   pass 2, history chunks:  r = y - yhat, sigma-hat (L513-L515); the last h
+//                            valid residuals land in a per-pixel ring of h
+//                            slots (the MOSUM seed m^fst, L518)
+//   pass 2, monitoring:      r, MOSUM recurrence over the ring (the slot
+//                            about to be overwritten holds rank c-h),
+//                            boundary, first break, mean (L520-L537)
+// The stack is read through a 2-D TMA tensor map whose out-of-bounds fill is
+// NaN, so a ragged last tile needs no special case (its missing pixels are
+// "all missing").
 #pragma once
 #include "monitor_simt.cuh"
 #include "sm100.cuh"
@@ -63,68 +70,54 @@ template <int K>
 struct TcCfg {
   static constexpr int k = (K - 2) / 2;
   static constexpr int NF = 2 + 6 * k;                     // masked moment functions
-  static constexpr int NGp = ((3 * NF + 15) / 16) * 16;    // Gram GEMM N (hi, mid, lo)
-  static constexpr int KB = ((2 * K + 15) / 16) * 16;      // moment GEMM N
+  static constexpr int NGn = ((NF + 1 + 15) / 16) * 16;    // Gram GEMM N (+ the constant 1: nbar)
+  static constexpr int KBn = ((K + 15) / 16) * 16;         // moment GEMM N
   static constexpr int KY = ((6 * K + 15) / 16) * 16;      // yhat GEMM K
-  static constexpr int KB3 = ((3 * K + 15) / 16) * 16;     // refinement GEMM N (x hi|mid|lo)
   static constexpr int DC = 16;                            // dates per chunk
-  // TMEM columns.  Pass 1 accumulates the Gram moments and the moment b;
-  // pass 2 the refinement moment, two yhat slots and the beta operand (the
-  // A operand of the yhat GEMM, bf16 pairs).  The consumers read G and b in
-  // the solve before any pass-2 MMA is issued, so pass 2 reuses their columns.
-  static constexpr int COL_G = 0, COL_B = NGp;
-  static constexpr int COL_DB = 0, COL_Y = KB3, COL_A3 = KB3 + 2 * DC;
-  static constexpr int COLS_P1 = NGp + KB, COLS_P2 = COL_A3 + KY / 2;
+  // TMEM columns.  Pass 1: two accumulator sets [Gram | moment]; pass 2
+  // (after the solve has read them): two yhat slots, the beta operand (the A
+  // operand of the yhat GEMM, bf16 pairs) and the refinement moment.
+  static constexpr int SET = NGn + KBn;
+  static constexpr int COL_Y = 0, COL_A3 = 2 * DC, COL_DB = ((COL_A3 + KY / 2 + 15) / 16) * 16;
+  static constexpr int COLS_P1 = 2 * SET, COLS_P2 = COL_DB + KBn;
   static constexpr int COLS_USED = COLS_P1 > COLS_P2 ? COLS_P1 : COLS_P2;
   static constexpr int TMEM_COLS = COLS_USED <= 32 ? 32 : COLS_USED <= 64 ? 64 : COLS_USED <= 128 ? 128
                                    : COLS_USED <= 256 ? 256 : 512;
-  static constexpr int B1_BYTES = NGp * DC * 2;            // [NGp x 16] bf16
-  static constexpr int B2_BYTES = KB * 2 * DC * 2;         // [KB x 32] bf16
-  static constexpr int B3_BYTES = DC * KY * 2;             // [16 x KY] bf16
-  static constexpr int BR_BYTES = KB3 * 3 * DC * 2;        // [KB3 x 48] bf16 (refinement)
-  static constexpr int TAB1 = B1_BYTES + B2_BYTES;         // pass 1 chunk tables
-  static constexpr int TAB2 = BR_BYTES + B3_BYTES;         // pass 2a
-  static constexpr int TAB3 = B3_BYTES;                    // pass 2b
+  static constexpr int BF_BYTES = NGn * DC * 2;            // one part of the Gram table [NGn x 16]
+  static constexpr int BX_BYTES = KBn * DC * 2;            // one part of x [KBn x 16]
+  static constexpr int B3_BYTES = DC * KY * 2;             // yhat table [16 x KY]
+  static constexpr int TAB1 = 3 * BF_BYTES + 3 * BX_BYTES; // pass 1 (history): F parts, x parts
+  static constexpr int TAB2 = B3_BYTES + 3 * BX_BYTES;     // pass 2 history: yhat table, x parts
+  static constexpr int TABY = B3_BYTES;                    // pass 2 monitoring: yhat table
   static constexpr int TABMAX = TAB1 > TAB2 ? TAB1 : TAB2;
   static constexpr int YBYTES = DC * 128 * 4;             // one [16 dates x 128 px] box
   static constexpr int TSTAGE = ((TABMAX + 127) / 128) * 128;
-  static constexpr int SY_MAX = 4;                         // stack ring stages (released on read; 3 or 4)
+  static constexpr int SY_MAX = 4;                         // stack ring stages (released on read)
   static constexpr int ST = 3;                             // table ring stages (released by MMA commit)
-  static constexpr int A1_BYTES = 128 * DC * 2;
-  static constexpr int A2_BYTES = 128 * 2 * DC * 2;
-  static constexpr int A4_BYTES = 128 * 3 * DC * 2;        // r0 hi|mid|lo per date
-  static constexpr int OPBUF = A1_BYTES + A2_BYTES > A4_BYTES ? A1_BYTES + A2_BYTES : A4_BYTES;
-  static constexpr int RSLOT = 128 * 4;                   // ring slot: one residual per pixel
-  static constexpr int VSLOT = 128 * 2;                   // validity mask: 16 bits per pixel per chunk
+  static constexpr int ATILE = 128 * DC * 2;               // one [128 x 16] bf16 A tile
+  static constexpr int OPBUF = 3 * ATILE;                  // pass 1: mask, y'hi, y'lo; pass 2: r0hi, r0lo
+  static constexpr int RSLOT = 128 * 4;                    // ring slot: one residual per pixel
+  static constexpr int VSLOT = 128 * 2;                    // history validity: 16 bits per pixel per chunk
   // sy stack stages, nop operand buffers (2: the consumers fill one while the
-  // MMA reads the other), the MOSUM ring of hcap slots, nch history masks
+  // MMA reads the other), the MOSUM ring of hcap slots, nch validity masks
   static constexpr size_t smem_bytes(int hcap, int nch, int sy, int nop) {
     return (size_t)sy * YBYTES + (size_t)ST * TSTAGE + (size_t)nop * OPBUF + (size_t)hcap * RSLOT +
-           (size_t)nch * VSLOT;
+           (size_t)((nch * VSLOT + 15) / 16) * 16;
   }
 };
 
 struct TcTables {
-  const uint8_t *tab1, *tab2, *tab3;  // per-chunk B operands, canonical K-major layout
+  const uint8_t *tab1, *tab2, *taby;  // per-chunk B operands, canonical K-major layout
   int nch, ncm;                       // history / monitoring chunks of 16 dates
-  int sy, nop;                        // stack stages (3|4), operand buffers (1|2)
+  int sy, nop;                        // stack stages (2..4), operand buffers (1|2)
   int64_t ntiles;                     // 128-pixel tiles (the last may be ragged)
 };
 
-__device__ __forceinline__ void named_bar_sync_128() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
 __device__ __forceinline__ void sts_f32(uint32_t a, float v) {
   asm volatile("st.shared.f32 [%0], %1;" ::"r"(a), "f"(v) : "memory");
 }
 __device__ __forceinline__ void sts_u16(uint32_t a, uint16_t v) {
   asm volatile("st.shared.u16 [%0], %1;" ::"r"(a), "h"(v) : "memory");
-}
-// store v if `inc` (the ring advance of this date: 0 for a missing one) is
-// non-zero.  The advance is materialised anyway, so the predicate costs one
-// compare instead of a re-evaluated NaN test (only 7 predicate registers).
-__device__ __forceinline__ void sts_f32_inc(uint32_t a, float v, uint32_t inc) {
-  asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.u32 p, %2, 0;\n\t@p st.shared.f32 [%0], %1;\n\t}" ::"r"(a), "f"(v),
-               "r"(inc)
-               : "memory");
 }
 __device__ __forceinline__ float lds_f32(uint32_t a) {
   float v;
@@ -136,13 +129,96 @@ __device__ __forceinline__ int lds_u16(uint32_t a) {
   asm volatile("ld.shared.u16 %0, [%1];" : "=h"(v) : "r"(a) : "memory");
   return v;
 }
-// producer-side wait with back-off so a waiting producer does not steal
-// issue slots from the consumer warps of its SM sub-partition
+// ---- per-date steps (inline PTX: the validity predicate never leaves the asm)
+// Pass 1: vm = all-ones if y is a value (set.num), y' = (y - c) & vm (NaN -> 0),
+// 2-way bf16 split of y' by truncation: y' = h + l (l exact in fp32; its bf16
+// packing keeps 16 significant bits in all, enough for the first fit).
+__device__ __forceinline__ void p1_date(float y, float c0, uint32_t &vm, float &h, float &l) {
+  asm("{\n\t.reg .f32 yp;\n\t"
+      "set.num.u32.f32 %0, %3, %3;\n\t"
+      "sub.f32 yp, %3, %4;\n\t"
+      "and.b32 yp, yp, %0;\n\t"
+      "and.b32 %1, yp, 0xFFFF0000;\n\t"
+      "sub.f32 %2, yp, %1;\n\t}"
+      : "=r"(vm), "=f"(h), "=f"(l)
+      : "f"(y), "f"(c0));
+}
+// Pass 2, history date: r0 = (y - c) - yhat0 (NaN if missing); if r0 is a
+// value: s2 += r0^2 and bit BIT of vb is set; (h, l) = 2-way split of r0
+// (0 when missing) for the refinement moment.
+template <int BIT>
+__device__ __forceinline__ void p2h_date(float y, float c0, float yh, float &s2, uint32_t &vb, float &h, float &l) {
+  asm("{\n\t.reg .pred p;\n\t.reg .f32 r;\n\t"
+      "sub.f32 r, %4, %5;\n\t"
+      "sub.f32 r, r, %6;\n\t"
+      "setp.num.f32 p, r, r;\n\t"
+      "@p fma.rn.f32 %0, r, r, %0;\n\t"
+      "@p or.b32 %1, %1, %7;\n\t"
+      "selp.f32 r, r, 0f00000000, p;\n\t"
+      "and.b32 %2, r, 0xFFFF0000;\n\t"
+      "sub.f32 %3, r, %2;\n\t}"
+      : "+f"(s2), "+r"(vb), "=f"(h), "=f"(l)
+      : "f"(y), "f"(c0), "f"(yh), "n"(1u << BIT));
+}
+// ... and the residual also enters the per-pixel ring of h slots at wa
+// (wrap at rend back by hbytes).
+template <int BIT>
+__device__ __forceinline__ void p2h_date_ring(float y, float c0, float yh, float &s2, uint32_t &vb, float &h,
+                                              float &l, uint32_t &wa, uint32_t rend, uint32_t hbytes) {
+  asm volatile(
+      "{\n\t.reg .pred p, q;\n\t.reg .f32 r;\n\t"
+      "sub.f32 r, %5, %6;\n\t"
+      "sub.f32 r, r, %7;\n\t"
+      "setp.num.f32 p, r, r;\n\t"
+      "@p fma.rn.f32 %0, r, r, %0;\n\t"
+      "@p or.b32 %1, %1, %8;\n\t"
+      "@p st.shared.f32 [%4], r;\n\t"
+      "@p add.u32 %4, %4, 512;\n\t"
+      "setp.ge.u32 q, %4, %9;\n\t"
+      "@q sub.u32 %4, %4, %10;\n\t"
+      "selp.f32 r, r, 0f00000000, p;\n\t"
+      "and.b32 %2, r, 0xFFFF0000;\n\t"
+      "sub.f32 %3, r, %2;\n\t}"
+      : "+f"(s2), "+r"(vb), "=f"(h), "=f"(l), "+r"(wa)
+      : "f"(y), "f"(c0), "f"(yh), "n"(1u << BIT), "r"(rend), "r"(hbytes)
+      : "memory");
+}
+// Monitoring date (Eq. (4) recurrence, L520-L525): r = y - yhat; the ring
+// slot at wa holds rank cr - h (`old`); if r is a value it replaces it,
+// W += r - old, msum += W, cr += 1 and mx = max(mx, |W|).  r and old are
+// returned for the exact replay of a half-chunk in which mx crossed.
+__device__ __forceinline__ void mon_date(float y, float c0, float yh, float &W, float &msum, float &mx, int &cr,
+                                         uint32_t &wa, uint32_t rend, uint32_t hbytes, float &r, float &old) {
+  asm volatile(
+      "{\n\t.reg .pred p, q;\n\t.reg .f32 t;\n\t"
+      "sub.f32 %5, %7, %8;\n\t"
+      "sub.f32 %5, %5, %9;\n\t"
+      "setp.num.f32 p, %5, %5;\n\t"
+      "ld.shared.f32 %6, [%4];\n\t"
+      "@p st.shared.f32 [%4], %5;\n\t"
+      "@p add.u32 %4, %4, 512;\n\t"
+      "setp.ge.u32 q, %4, %10;\n\t"
+      "@q sub.u32 %4, %4, %11;\n\t"
+      "@p add.s32 %3, %3, 1;\n\t"
+      "sub.f32 t, %5, %6;\n\t"
+      "@p add.f32 %0, %0, t;\n\t"
+      "@p add.f32 %1, %1, %0;\n\t"
+      "abs.f32 t, %0;\n\t"
+      "@p max.f32 %2, %2, t;\n\t}"
+      : "+f"(W), "+f"(msum), "+f"(mx), "+r"(cr), "+r"(wa), "=f"(r), "=f"(old)
+      : "f"(y), "f"(c0), "f"(yh), "r"(rend), "r"(hbytes)
+      : "memory");
+}
+// producer-side waits with back-off so a waiting producer does not steal
+// issue slots from the consumer warps of its SM sub-partition: MODE 0 =
+// try_wait with a suspend hint, 1 = poll, N > 1 = poll with an N-ns sleep.
+// Measured on the Landsat config (tools/ab_bench.sh): stack/table producers
+// 256 ns and the MMA issuer 32 ns are 8% faster than polling.
 #ifndef BFAST_AUX_WAIT
-#define BFAST_AUX_WAIT 0
+#define BFAST_AUX_WAIT 256
 #endif
 #ifndef BFAST_MMA_WAIT
-#define BFAST_MMA_WAIT 0
+#define BFAST_MMA_WAIT 32
 #endif
 template <int MODE>
 __device__ __forceinline__ void mbar_wait_mode(uint64_t *bar, uint32_t parity) {
@@ -153,8 +229,7 @@ __device__ __forceinline__ void mbar_wait_mode(uint64_t *bar, uint32_t parity) {
     while (!sm100::mbar_try_wait(bar, parity)) {
     }
   } else {
-    while (!sm100::mbar_try_wait_suspend(bar, parity, (uint32_t)MODE)) {
-    }
+    while (!sm100::mbar_try_wait(bar, parity)) __nanosleep(MODE);
   }
 }
 __device__ __forceinline__ void mbar_wait_sleep(uint64_t *bar, uint32_t parity) {
@@ -171,12 +246,6 @@ __device__ __noinline__ int boundary_rare(float m, int rank1, int nbar, float la
   return (am > B ? 1 : 0) | (fabsf(am - B) <= kTieTol * B ? 2 : 0);
 }
 
-// y split into hi and lo bf16 halves packed {lo16: hi part, hi16: lo part}
-__device__ __forceinline__ uint32_t split2_bf16(float v) {
-  const uint32_t w1 = sm100::pack_bf16x2(v, 0.f);
-  const float hi = __uint_as_float(w1 << 16);
-  return sm100::pack_bf16x2(v, v - hi);
-}
 // bf16 parts by truncation: hi = top 8 significant bits of v (exactly
 // representable), v - hi exact.  Two words' upper halves -> one packed word.
 __device__ __forceinline__ float bf16_trunc(float v) { return __uint_as_float(__float_as_uint(v) & 0xFFFF0000u); }
@@ -229,168 +298,181 @@ __global__ void __launch_bounds__(kTcThreads, 3)
   __syncthreads();
   sm100::tc_fence_after();
   const uint32_t tbase = tmem_base_s;
-  const int n = p.n, N = p.N, nch = tb.nch, ncm = tb.ncm;
+  const int n = p.n, nch = tb.nch, ncm = tb.ncm;
 
   if (warp >= NCW) {
     // producer warpgroup: three single-thread roles need few registers; hand
     // them to the consumer warpgroup (3 CTAs per SM fit the register file)
     sm100::setmaxnreg_dec<kTcAuxRegs>();
-  if (warp == 4) {
-    // ------------------------------------------------------------ stack producer
-    if (lane == 0) {
-      // one 2-D TMA box [16 dates x 128 px] per chunk.  History chunks read
-      // through `hmap` (dates >= n are out of bounds), monitoring chunks
-      // through `ymap`; out-of-bounds elements arrive as NaN = missing.
-      sm100::prefetch_tmap(&ymap);
-      sm100::prefetch_tmap(&hmap);
-      const uint64_t pol_first = sm100::policy_evict_first();
-      int ys = 0;
-      uint32_t yph = 0;
-      for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
-        const int x0 = (int)(tile * 128);
-        for (int phase = 0; phase < 3; ++phase) {
-          const int nc = phase < 2 ? nch : ncm;
-          const int tbeg = phase < 2 ? 0 : n;
-          for (int c = 0; c < nc; ++c) {
-            mbar_wait_sleep(&yempty[ys], yph ^ 1);
-            uint8_t *yst = ystages + ys * C::YBYTES;
-            sm100::mbar_arrive_expect_tx(&yfull[ys], C::YBYTES);
-            if (phase == 0)
-              sm100::tma_load_2d(yst, &hmap, x0, c * C::DC, &yfull[ys]);  // re-read in pass 2a (L2)
-            else
-              sm100::tma_load_2d_hint(yst, phase == 1 ? &hmap : &ymap, x0, tbeg + c * C::DC, &yfull[ys],
-                                      pol_first);  // last use
-            if (++ys == SY) {
-              ys = 0;
-              yph ^= 1;
+    if (warp == 4) {
+      // ------------------------------------------------------------ stack producer
+      if (lane == 0) {
+        // one 2-D TMA box [16 dates x 128 px] per chunk.  History chunks read
+        // through `hmap` (dates >= n are out of bounds), monitoring chunks
+        // through `ymap`; out-of-bounds elements arrive as NaN = missing.
+        sm100::prefetch_tmap(&ymap);
+        sm100::prefetch_tmap(&hmap);
+        const uint64_t pol_first = sm100::policy_evict_first();
+        int ys = 0;
+        uint32_t yph = 0;
+        for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
+          const int x0 = (int)(tile * 128);
+          for (int phase = 0; phase < 3; ++phase) {
+            const int nc = phase < 2 ? nch : ncm;
+            const int tbeg = phase < 2 ? 0 : n;
+            for (int c = 0; c < nc; ++c) {
+              mbar_wait_sleep(&yempty[ys], yph ^ 1);
+              uint8_t *yst = ystages + ys * C::YBYTES;
+              sm100::mbar_arrive_expect_tx(&yfull[ys], C::YBYTES);
+              if (phase == 0)
+                sm100::tma_load_2d(yst, &hmap, x0, c * C::DC, &yfull[ys]);  // re-read in pass 2 (L2)
+              else
+                sm100::tma_load_2d_hint(yst, phase == 1 ? &hmap : &ymap, x0, tbeg + c * C::DC, &yfull[ys],
+                                        pol_first);  // last use
+              if (++ys == SY) {
+                ys = 0;
+                yph ^= 1;
+              }
             }
           }
         }
       }
-    }
-  } else if (warp == 5) {
-    // ------------------------------------------------------------ table producer
-    if (lane == 0) {
-      int ts = 0;
-      uint32_t tph = 0;
-      for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
-        for (int phase = 0; phase < 3; ++phase) {
-          const int nc = phase < 2 ? nch : ncm;
-          const uint32_t tabbytes = phase == 0 ? C::TAB1 : phase == 1 ? C::TAB2 : C::TAB3;
-          const uint8_t *tabsrc = phase == 0 ? tb.tab1 : phase == 1 ? tb.tab2 : tb.tab3;
-          for (int c = 0; c < nc; ++c) {
-            mbar_wait_sleep(&tempty[ts], tph ^ 1);
-            uint8_t *tst = tstages + ts * C::TSTAGE;
-            sm100::mbar_arrive_expect_tx(&tfull[ts], tabbytes);
-            sm100::bulk_g2s(tst, tabsrc + (size_t)c * tabbytes, tabbytes, &tfull[ts]);
-            if (++ts == C::ST) {
-              ts = 0;
-              tph ^= 1;
+    } else if (warp == 5) {
+      // ------------------------------------------------------------ table producer
+      if (lane == 0) {
+        int ts = 0;
+        uint32_t tph = 0;
+        for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
+          for (int phase = 0; phase < 3; ++phase) {
+            const int nc = phase < 2 ? nch : ncm;
+            const uint32_t tabbytes = phase == 0 ? C::TAB1 : phase == 1 ? C::TAB2 : C::TABY;
+            const uint8_t *tabsrc = phase == 0 ? tb.tab1 : phase == 1 ? tb.tab2 : tb.taby;
+            for (int c = 0; c < nc; ++c) {
+              mbar_wait_sleep(&tempty[ts], tph ^ 1);
+              uint8_t *tst = tstages + ts * C::TSTAGE;
+              sm100::mbar_arrive_expect_tx(&tfull[ts], tabbytes);
+              sm100::bulk_g2s(tst, tabsrc + (size_t)c * tabbytes, tabbytes, &tfull[ts]);
+              if (++ts == C::ST) {
+                ts = 0;
+                tph ^= 1;
+              }
             }
           }
         }
       }
-    }
-  } else if (warp == 6) {
-    // ------------------------------------------------------------ MMA issuer
-    if (lane == 0) {
-      const uint32_t idG = sm100::idesc_bf16_f32(128, C::NGp);
-      const uint32_t idB = sm100::idesc_bf16_f32(128, C::KB);
-      const uint32_t idY = sm100::idesc_bf16_f32(128, C::DC);
-      const uint32_t idR = sm100::idesc_bf16_f32(128, C::KB3);
-      const uint32_t aop = sm100::smem_u32(opb), tss = sm100::smem_u32(tstages);
-      int ts = 0;
-      uint32_t tph = 0, opcnt = 0, yissue = 0, bcnt = 0;
-      auto tslot = [&](int ahead, uint32_t &par) {
-        int s = ts + ahead;
-        par = tph;
-        while (s >= C::ST) {
-          s -= C::ST;
-          par ^= 1;
-        }
-        return s;
-      };
-      auto tadvance = [&]() {
-        if (++ts == C::ST) {
-          ts = 0;
-          tph ^= 1;
-        }
-      };
-      // operand buffer of the opcnt-th chunk and its phase parity
-      auto opwait = [&]() -> uint32_t {
-        const uint32_t ob = NOP == 2 ? (opcnt & 1) : 0;
-        const uint32_t par = NOP == 2 ? ((opcnt >> 1) & 1) : (opcnt & 1);
-        mbar_wait_mma(&opfull[ob], par);
-        return ob;
-      };
-      // yhat of the chunk `ahead` chunks after the current one (table offset)
-      auto issue_yhat = [&](int ahead, uint32_t tab_off) {
-        uint32_t par;
-        const int s = tslot(ahead, par);
-        const uint32_t slot = yissue & 1;
-        mbar_wait_mma(&yhfree[slot], ((yissue >> 1) & 1) ^ 1);  // consumers done with the slot
-        mbar_wait_mma(&tfull[s], par);
-        sm100::tc_fence_after();
-        const uint32_t b3 = tss + s * C::TSTAGE + tab_off;
-#pragma unroll
-        for (int q = 0; q < C::KY / 16; ++q)
-          sm100::umma_bf16_ts(tbase + C::COL_Y + slot * C::DC, tbase + C::COL_A3 + 8 * q,
-                              sm100::smem_desc(b3 + q * 2 * 256, 256, 128), idY, q > 0);
-        sm100::umma_commit(&yhfull[slot]);
-        ++yissue;
-      };
-      for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
-        // pass 1: Gram + moment per chunk
-        for (int c = 0; c < nch; ++c) {
-          const uint32_t ob = opwait();
-          mbar_wait_mma(&tfull[ts], tph);
+    } else if (warp == 6) {
+      // ------------------------------------------------------------ MMA issuer
+      if (lane == 0) {
+        const uint32_t idG = sm100::idesc_bf16_f32(128, C::NGn);
+        const uint32_t idB = sm100::idesc_bf16_f32(128, C::KBn);
+        const uint32_t idY = sm100::idesc_bf16_f32(128, C::DC);
+        const uint32_t aop = sm100::smem_u32(opb), tss = sm100::smem_u32(tstages);
+        int ts = 0;
+        uint32_t tph = 0, opcnt = 0, yissue = 0, bcnt = 0;
+        auto tslot = [&](int ahead, uint32_t &par) {
+          int s = ts + ahead;
+          par = tph;
+          while (s >= C::ST) {
+            s -= C::ST;
+            par ^= 1;
+          }
+          return s;
+        };
+        auto tadvance = [&]() {
+          if (++ts == C::ST) {
+            ts = 0;
+            tph ^= 1;
+          }
+        };
+        // operand buffer of the opcnt-th chunk and its phase parity
+        auto opwait = [&]() -> uint32_t {
+          const uint32_t ob = NOP == 2 ? (opcnt & 1) : 0;
+          const uint32_t par = NOP == 2 ? ((opcnt >> 1) & 1) : (opcnt & 1);
+          mbar_wait_mma(&opfull[ob], par);
+          return ob;
+        };
+        // yhat of the chunk `ahead` chunks after the current one (its table
+        // stage starts with the [16 x KY] yhat table)
+        auto issue_yhat = [&](int ahead) {
+          uint32_t par;
+          const int s = tslot(ahead, par);
+          const uint32_t slot = yissue & 1;
+          mbar_wait_mma(&yhfree[slot], ((yissue >> 1) & 1) ^ 1);  // consumers done with the slot
+          mbar_wait_mma(&tfull[s], par);
           sm100::tc_fence_after();
-          const uint32_t a1 = aop + ob * C::OPBUF, a2 = a1 + C::A1_BYTES;
-          const uint32_t b1 = tss + ts * C::TSTAGE, b2 = b1 + C::B1_BYTES;
-          sm100::umma_bf16(tbase + C::COL_G, sm100::smem_desc(a1, 2048, 128),
-                           sm100::smem_desc(b1, C::NGp * 16, 128), idG, c > 0);
+          const uint32_t b3 = tss + s * C::TSTAGE;
 #pragma unroll
-          for (int q = 0; q < 2; ++q)
-            sm100::umma_bf16(tbase + C::COL_B, sm100::smem_desc(a2 + q * 2 * 2048, 2048, 128),
-                             sm100::smem_desc(b2 + q * 2 * C::KB * 16, C::KB * 16, 128), idB, (c > 0 || q > 0));
-          sm100::umma_commit(&opfree[ob]);
-          sm100::umma_commit(&tempty[ts]);
-          if (c == nch - 1) sm100::umma_commit(&accready);
-          ++opcnt;
-          tadvance();
-        }
-        // pass 2a: yhat0 two chunks ahead, refinement moment per chunk
-        mbar_wait_mma(&betaready, bcnt & 1);
-        ++bcnt;
-        for (int a = 0; a < 2 && a < nch; ++a) issue_yhat(a, C::BR_BYTES);
-        for (int c = 0; c < nch; ++c) {
-          const uint32_t ob = opwait();
-          mbar_wait_mma(&tfull[ts], tph);
-          sm100::tc_fence_after();
-          const uint32_t br = tss + ts * C::TSTAGE;
+          for (int q = 0; q < C::KY / 16; ++q)
+            sm100::umma_bf16_ts(tbase + C::COL_Y + slot * C::DC, tbase + C::COL_A3 + 8 * q,
+                                sm100::smem_desc(b3 + q * 2 * 256, 256, 128), idY, q > 0);
+          sm100::umma_commit(&yhfull[slot]);
+          ++yissue;
+        };
+        for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
+          // pass 1: Gram + moment per chunk, accumulator set c & 1
+          for (int c = 0; c < nch; ++c) {
+            const uint32_t ob = opwait();
+            mbar_wait_mma(&tfull[ts], tph);
+            sm100::tc_fence_after();
+            const uint32_t am = aop + ob * C::OPBUF;  // mask, y' hi, y' lo tiles
+            const uint32_t bf = tss + ts * C::TSTAGE, bx = bf + 3 * C::BF_BYTES;
+            const uint32_t dG = tbase + (c & 1) * C::SET, dB = dG + C::NGn;
+            const uint32_t first = c >= 2 ? 1u : 0u;
 #pragma unroll
-          for (int q = 0; q < 3; ++q)
-            sm100::umma_bf16(tbase + C::COL_DB, sm100::smem_desc(aop + ob * C::OPBUF + q * 2 * 2048, 2048, 128),
-                             sm100::smem_desc(br + q * 2 * C::KB3 * 16, C::KB3 * 16, 128), idR, (c > 0 || q > 0));
-          sm100::umma_commit(&opfree[ob]);
-          if (c + 2 < nch) issue_yhat(2, C::BR_BYTES);
-          sm100::umma_commit(&tempty[ts]);
-          if (c == nch - 1) sm100::umma_commit(&accready);
-          ++opcnt;
-          tadvance();
-        }
-        // pass 2b: yhat with the refined beta, two chunks ahead
-        mbar_wait_mma(&betaready, bcnt & 1);
-        ++bcnt;
-        for (int a = 0; a < 2 && a < ncm; ++a) issue_yhat(a, 0);
-        for (int c = 0; c < ncm; ++c) {
-          if (c + 2 < ncm) issue_yhat(2, 0);
-          sm100::umma_commit(&tempty[ts]);  // chunk c's table was read by its yhat MMA
-          tadvance();
+            for (int e = 0; e < 3; ++e)
+              sm100::umma_bf16(dG, sm100::smem_desc(am, 2048, 128),
+                               sm100::smem_desc(bf + e * C::BF_BYTES, C::NGn * 16, 128), idG, first | (e > 0));
+            // y'hi x_hi, y'hi x_mid, y'lo x_hi
+            sm100::umma_bf16(dB, sm100::smem_desc(am + C::ATILE, 2048, 128), sm100::smem_desc(bx, C::KBn * 16, 128),
+                             idB, first);
+            sm100::umma_bf16(dB, sm100::smem_desc(am + C::ATILE, 2048, 128),
+                             sm100::smem_desc(bx + C::BX_BYTES, C::KBn * 16, 128), idB, 1);
+            sm100::umma_bf16(dB, sm100::smem_desc(am + 2 * C::ATILE, 2048, 128),
+                             sm100::smem_desc(bx, C::KBn * 16, 128), idB, 1);
+            sm100::umma_commit(&opfree[ob]);
+            sm100::umma_commit(&tempty[ts]);
+            if (c == nch - 1) sm100::umma_commit(&accready);
+            ++opcnt;
+            tadvance();
+          }
+          // pass 2, history: yhat0 two chunks ahead, refinement moment per chunk
+          mbar_wait_mma(&betaready, bcnt & 1);
+          ++bcnt;
+          for (int a = 0; a < 2 && a < nch; ++a) issue_yhat(a);
+          for (int c = 0; c < nch; ++c) {
+            const uint32_t ob = opwait();
+            mbar_wait_mma(&tfull[ts], tph);
+            sm100::tc_fence_after();
+            const uint32_t am = aop + ob * C::OPBUF;  // r0 hi, r0 lo tiles
+            const uint32_t bx = tss + ts * C::TSTAGE + C::B3_BYTES;
+            const uint32_t dD = tbase + C::COL_DB;
+            // r0hi (x_hi + x_mid + x_lo) + r0lo (x_hi + x_mid)
+#pragma unroll
+            for (int e = 0; e < 2; ++e)
+#pragma unroll
+              for (int q = 0; q < 3 - e; ++q)
+                sm100::umma_bf16(dD, sm100::smem_desc(am + e * C::ATILE, 2048, 128),
+                                 sm100::smem_desc(bx + q * C::BX_BYTES, C::KBn * 16, 128), idB,
+                                 (c > 0 || e > 0 || q > 0) ? 1u : 0u);
+            sm100::umma_commit(&opfree[ob]);
+            if (c + 2 < nch) issue_yhat(2);
+            sm100::umma_commit(&tempty[ts]);
+            if (c == nch - 1) sm100::umma_commit(&accready);
+            ++opcnt;
+            tadvance();
+          }
+          // pass 2, monitoring: yhat with the refined beta, two chunks ahead
+          mbar_wait_mma(&betaready, bcnt & 1);
+          ++bcnt;
+          for (int a = 0; a < 2 && a < ncm; ++a) issue_yhat(a);
+          for (int c = 0; c < ncm; ++c) {
+            if (c + 2 < ncm) issue_yhat(2);
+            sm100::umma_commit(&tempty[ts]);  // chunk c's table was read by its yhat MMA
+            tadvance();
+          }
         }
       }
-    }
-  }  // warp 7 idles: it completes the producer warpgroup
+    }  // warp 7 idles: it completes the producer warpgroup
   } else {
     // ------------------------------------------------------------ consumers
     sm100::setmaxnreg_inc<kTcConsumerRegs>();
@@ -399,7 +481,6 @@ __global__ void __launch_bounds__(kTcThreads, 3)
     // ring: slot s = 128 residuals f32, this thread's at rbase + s*RSLOT;
     // history validity: 16 bits per chunk, this thread's at vbase + c*VSLOT
     const uint32_t rbase = sm100::smem_u32(ring) + 4 * tid;
-    const uint32_t rend = rbase + hcap * C::RSLOT;
     const uint32_t vbase = sm100::smem_u32(vmask) + 2 * tid;
     int ys = 0;
     uint32_t yph = 0, opcnt = 0, yuse = 0, acnt = 0;
@@ -408,7 +489,6 @@ __global__ void __launch_bounds__(kTcThreads, 3)
     const uint32_t a_opfull = sm100::smem_u32(&opfull[0]), a_opfree = sm100::smem_u32(&opfree[0]);
     const uint32_t a_yhfull = sm100::smem_u32(&yhfull[0]), a_yhfree = sm100::smem_u32(&yhfree[0]);
     const uint32_t a_accready = sm100::smem_u32(&accready), a_betaready = sm100::smem_u32(&betaready);
-    const uint32_t ybuf0 = sm100::smem_u32(ystages);
 
     auto yadvance = [&]() {
       if (++ys == SY) {
@@ -433,17 +513,14 @@ __global__ void __launch_bounds__(kTcThreads, 3)
       warp_arrive(a_opfull + 8 * ob);
       ++opcnt;
     };
-    auto write_beta_operand = [&](const float (&bt)[K], float off) {
-      // A3 row (TMEM) = [bh | bh | bh | bm | bm | bl | 0...] (6 blocks of K, KY bf16);
-      // `off` would fold an offset into the intercept (kept at 0: the GEMM's
-      // accumulation error scales with |yhat|, so the offset stays outside)
+    auto write_beta_operand = [&](const float (&bt)[K]) {
+      // A3 row (TMEM) = [bh | bh | bh | bm | bm | bl | 0...] (6 blocks of K, KY bf16)
       float h[K], m[K], l[K];
 #pragma unroll
       for (int i = 0; i < K; ++i) {
-        const float bi = i == 0 ? bt[0] + off : bt[i];
-        h[i] = bf16_round(bi);
-        m[i] = bf16_round(bi - h[i]);
-        l[i] = bi - h[i] - m[i];
+        h[i] = bf16_round(bt[i]);
+        m[i] = bf16_round(bt[i] - h[i]);
+        l[i] = bt[i] - h[i] - m[i];
       }
       uint32_t w[C::KY / 2];
 #pragma unroll
@@ -484,7 +561,6 @@ __global__ void __launch_bounds__(kTcThreads, 3)
     for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
       const int64_t pix = p.p0 + tile * 128 + tid;
       // ================= pass 1: masked Gram + moment on the tensor cores
-      int nbar = 0;
       float c0 = qnan, ymax = 0.f;
       bool have = false;
       for (int c = 0; c < nch; ++c) {
@@ -500,32 +576,31 @@ __global__ void __launch_bounds__(kTcThreads, 3)
             }
           }
         }
-        uint8_t *const ob = opbuf_acquire();
+        uint8_t *ob = nullptr;
 #pragma unroll 1
         for (int hf = 0; hf < 2; ++hf) {  // two halves of 8 dates: half the hot code
           float yv[8];
 #pragma unroll
           for (int d = 0; d < 8; ++d) yv[d] = Ys[(8 * hf + d) * 128 + tid];  // dates >= n read as NaN (hmap)
-          uint32_t mw[4], yw[8];
-          float mf[8];
+          uint32_t vm[8];
+          float ph[8], pl[8];
 #pragma unroll
           for (int d = 0; d < 8; ++d) {
-            const float y = yv[d];
-            const bool v = (y == y);
-            ymax = fmaxf(ymax, fabsf(y));  // NaN ignored
-            nbar += v;
-            const float yp = v ? y - c0 : 0.f;
-            const float yh = bf16_trunc(yp);
-            yw[d] = pack_hi16(yh, yp - yh);  // {y' hi, y' lo}
-            mf[d] = v ? 1.0f : 0.0f;
+            ymax = fmaxf(ymax, fabsf(yv[d]));  // NaN ignored
+            p1_date(yv[d], c0, vm[d], ph[d], pl[d]);
           }
-#pragma unroll
-          for (int q = 0; q < 4; ++q) mw[q] = pack_hi16(mf[2 * q], mf[2 * q + 1]);
-          *reinterpret_cast<uint4 *>(ob + sm100::kmajor_off(tid, 8 * hf, 128)) = make_uint4(mw[0], mw[1], mw[2], mw[3]);
-#pragma unroll
-          for (int q = 0; q < 2; ++q)
-            *reinterpret_cast<uint4 *>(ob + C::A1_BYTES + sm100::kmajor_off(tid, 16 * hf + 8 * q, 128)) =
-                make_uint4(yw[4 * q], yw[4 * q + 1], yw[4 * q + 2], yw[4 * q + 3]);
+          // the MMA of the previous chunk frees the operand buffer while the
+          // first half is computed
+          if (hf == 0) ob = opbuf_acquire();
+          const uint32_t off = sm100::kmajor_off(tid, 8 * hf, 128);
+          // mask pair words: bf16 1.0 (0x3F80) in each half whose date is valid
+          *reinterpret_cast<uint4 *>(ob + off) =
+              make_uint4((vm[0] & 0x3F80u) | (vm[1] & 0x3F800000u), (vm[2] & 0x3F80u) | (vm[3] & 0x3F800000u),
+                         (vm[4] & 0x3F80u) | (vm[5] & 0x3F800000u), (vm[6] & 0x3F80u) | (vm[7] & 0x3F800000u));
+          *reinterpret_cast<uint4 *>(ob + C::ATILE + off) = make_uint4(
+              pack_hi16(ph[0], ph[1]), pack_hi16(ph[2], ph[3]), pack_hi16(ph[4], ph[5]), pack_hi16(ph[6], ph[7]));
+          *reinterpret_cast<uint4 *>(ob + 2 * C::ATILE + off) = make_uint4(
+              pack_hi16(pl[0], pl[1]), pack_hi16(pl[2], pl[3]), pack_hi16(pl[4], pl[5]), pack_hi16(pl[6], pl[7]));
         }
         warp_arrive(a_yempty + 8 * ys);  // every loaded value has been consumed
         opbuf_publish();
@@ -537,30 +612,34 @@ __global__ void __launch_bounds__(kTcThreads, 3)
 
       // ================= solve (Alg. 1 l.3-4): Gram from the masked moments
       float A[Tri<K>::kN], b[K];
+      int nbar;
       {
-        float F[C::NGp];
+        float G[C::NF + 1];  // moments, then the count of valid history dates
 #pragma unroll
-        for (int q = 0; q < C::NGp / 16; ++q) {
-          float v16[16];
-          sm100::tmem_ld16(lanebase + C::COL_G + 16 * q, v16);
-          sm100::tmem_ld_wait();
+        for (int i = 0; i <= C::NF; ++i) G[i] = 0.f;
 #pragma unroll
-          for (int i = 0; i < 16; ++i) F[16 * q + i] = v16[i];
+        for (int i = 0; i < K; ++i) b[i] = 0.f;
+#pragma unroll
+        for (int s = 0; s < 2; ++s) {
+          if (s == 1 && nch < 2) break;
+#pragma unroll
+          for (int q = 0; q < C::NGn / 16; ++q) {
+            float v16[16];
+            sm100::tmem_ld16(lanebase + s * C::SET + 16 * q, v16);
+            sm100::tmem_ld_wait();
+#pragma unroll
+            for (int i = 0; i < 16; ++i)
+              if (16 * q + i <= C::NF) G[16 * q + i] += v16[i];
+          }
+          {
+            float v16[16];
+            sm100::tmem_ld16(lanebase + s * C::SET + C::NGn, v16);
+            sm100::tmem_ld_wait();
+#pragma unroll
+            for (int i = 0; i < K; ++i) b[i] += v16[i];
+          }
         }
-        float Bm[C::KB];
-#pragma unroll
-        for (int q = 0; q < C::KB / 16; ++q) {
-          float v16[16];
-          sm100::tmem_ld16(lanebase + C::COL_B + 16 * q, v16);
-          sm100::tmem_ld_wait();
-#pragma unroll
-          for (int i = 0; i < 16; ++i) Bm[16 * q + i] = v16[i];
-        }
-        float G[C::NF];
-#pragma unroll
-        for (int q = 0; q < C::NF; ++q) G[q] = F[q] + F[C::NF + q] + F[2 * C::NF + q];
-#pragma unroll
-        for (int i = 0; i < K; ++i) b[i] = Bm[i] + Bm[K + i];
+        nbar = (int)G[C::NF];  // exact: a sum of 0/1 products in fp32
         const float nb = (float)nbar;
         auto Cf = [&](int m) -> float { return m == 0 ? nb : G[2 + 2 * C::k + 2 * ((m < 0 ? -m : m) - 1) + 1]; };
         auto Sf = [&](int m) -> float {
@@ -607,54 +686,60 @@ __global__ void __launch_bounds__(kTcThreads, 3)
         }
       }
       sm100::tc_fence_before();
-      write_beta_operand(beta, 0.f);
+      write_beta_operand(beta);
 
-      // ================= pass 2a: residuals r0, sigma, refinement moment, ring
+      // ================= pass 2, history: residuals r0 of the first fit,
+      // sigma-hat sums, the refinement moment operand, the seed ring.
+      // The ring holds h slots (hh for invalid pixels); the slot about to be
+      // written always holds rank cr - h.  Only chunks that can contain one
+      // of the last h valid history dates of some lane of the warp write it;
+      // starting earlier only writes ranks that are overwritten later.
       const int hh = deg ? 1 : h;
+      const uint32_t hbytes = (uint32_t)hh * C::RSLOT, rend = rbase + hbytes;
+      const int ring_from = nbar - hh;  // rank of the oldest residual the ring must keep
       float s2 = 0.f;
-      int cr = 0;
-      uint32_t wa = rbase;  // ring write address (slot of rank cr)
+      uint32_t wa = rbase;
+      int cr = 0;  // valid history dates before the current chunk
+      bool ring_on = false;
       for (int c = 0; c < nch; ++c) {
         sm100::mbar_wait_a(a_yfull + 8 * ys, yph);
+        // this chunk can hold rank nbar - hh or later for some lane of the warp
+        ring_on = ring_on || __any_sync(0xffffffffu, cr + C::DC > ring_from);
         wait_yhat();
         const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
-        uint8_t *const ob = opbuf_acquire();
-        uint32_t vm = 0;  // validity of the chunk's 16 dates
+        uint8_t *ob = nullptr;
+        uint32_t vb = 0;  // validity of the chunk's 16 dates
 #pragma unroll 1
         for (int hf = 0; hf < 2; ++hf) {
           float yh[8], yv[8];
-          uint32_t m8 = 0;  // bit 9+d: date d valid (ring advances accumulated)
           load_yhat8(hf, yh);
 #pragma unroll
           for (int d = 0; d < 8; ++d) yv[d] = Ys[(8 * hf + d) * 128 + tid];  // dates >= n read as NaN (hmap)
-          float rs3[24];
-#pragma unroll
-          for (int d = 0; d < 8; ++d) {
-            const float y = yv[d];
-            const bool v = (y == y);
-            const float r = v ? (y - c0) - yh[d] : 0.f;
-            s2 = fmaf(r, r, s2);
-            // exact 3-way bf16 split by truncation: r = rh + rm + rl
-            const float rh = bf16_trunc(r), t1 = r - rh, rm = bf16_trunc(t1);
-            rs3[3 * d] = rh;
-            rs3[3 * d + 1] = rm;
-            rs3[3 * d + 2] = t1 - rm;
-            const uint32_t inc = v ? C::RSLOT : 0u;
-            sts_f32_inc(wa, r, inc);
-            m8 += inc << d;
-            wa += inc;
-            wa = (wa == rend) ? rbase : wa;
+          float rh[8], rl[8];
+          uint32_t v8 = 0;
+          if (ring_on) {
+            SFor<0, 8>::run([&](auto dc) {
+              constexpr int d = decltype(dc)::value;
+              p2h_date_ring<d>(yv[d], c0, yh[d], s2, v8, rh[d], rl[d], wa, rend, hbytes);
+            });
+          } else {
+            SFor<0, 8>::run([&](auto dc) {
+              constexpr int d = decltype(dc)::value;
+              p2h_date<d>(yv[d], c0, yh[d], s2, v8, rh[d], rl[d]);
+            });
           }
-          static_assert(C::RSLOT == 512, "m8 packs the advances as bit 9 + d");
-          cr += __popc(m8);
-          vm |= (m8 >> 9) << (8 * hf);
-#pragma unroll
-          for (int q = 0; q < 3; ++q)
-            *reinterpret_cast<uint4 *>(ob + sm100::kmajor_off(tid, 24 * hf + 8 * q, 128)) =
-                make_uint4(pack_hi16(rs3[8 * q], rs3[8 * q + 1]), pack_hi16(rs3[8 * q + 2], rs3[8 * q + 3]),
-                           pack_hi16(rs3[8 * q + 4], rs3[8 * q + 5]), pack_hi16(rs3[8 * q + 6], rs3[8 * q + 7]));
+          vb |= v8 << (8 * hf);
+          if (hf == 0) ob = opbuf_acquire();
+          const uint32_t off = sm100::kmajor_off(tid, 8 * hf, 128);
+          // r0 = hi (truncated, exact) + lo (rounded to nearest: unbiased)
+          *reinterpret_cast<uint4 *>(ob + off) = make_uint4(
+              pack_hi16(rh[0], rh[1]), pack_hi16(rh[2], rh[3]), pack_hi16(rh[4], rh[5]), pack_hi16(rh[6], rh[7]));
+          *reinterpret_cast<uint4 *>(ob + C::ATILE + off) =
+              make_uint4(sm100::pack_bf16x2(rl[0], rl[1]), sm100::pack_bf16x2(rl[2], rl[3]),
+                         sm100::pack_bf16x2(rl[4], rl[5]), sm100::pack_bf16x2(rl[6], rl[7]));
         }
-        sts_u16(vbase + c * C::VSLOT, (uint16_t)vm);
+        sts_u16(vbase + c * C::VSLOT, (uint16_t)vb);
+        cr += __popc(vb);
         release_yhat();
         warp_arrive(a_yempty + 8 * ys);  // every loaded value has been consumed
         opbuf_publish();
@@ -667,17 +752,14 @@ __global__ void __launch_bounds__(kTcThreads, 3)
       // ================= refinement: beta = beta0 + A^-1 db; sigma-hat
       float sigma, dbf[K];
       {
-        float db[K], Dd[C::KB3];
-#pragma unroll
-        for (int q = 0; q < C::KB3 / 16; ++q) {
+        float db[K];
+        {
           float v16[16];
-          sm100::tmem_ld16(lanebase + C::COL_DB + 16 * q, v16);
+          sm100::tmem_ld16(lanebase + C::COL_DB, v16);
           sm100::tmem_ld_wait();
 #pragma unroll
-          for (int i = 0; i < 16; ++i) Dd[16 * q + i] = v16[i];
+          for (int i = 0; i < K; ++i) db[i] = v16[i];
         }
-#pragma unroll
-        for (int i = 0; i < K; ++i) db[i] = Dd[i] + Dd[K + i] + Dd[2 * K + i];
         chol_solve<K, float>(A, db, dbf);
         float lin = 0.f;
 #pragma unroll
@@ -686,9 +768,10 @@ __global__ void __launch_bounds__(kTcThreads, 3)
           lin = fmaf(dbf[i], db[i], lin);
           beta[i] += dbf[i];
         }
+        // sigma^2 (nbar - K) = sum (r0 - x dbeta)^2 = s2 - dbeta . db (A dbeta = db)
         sigma = sqrtf(fmaxf(s2 - lin, 0.f) / (float)(nbar - K));
-        // sigma^2 = s2 - lin cancels when the refinement step is large next to
-        // the residual sum: the fp32 sigma-hat is then unreliable -> fp64 refit
+        // sigma^2 cancels when the refinement step is large next to the
+        // residual sum: the fp32 sigma-hat is then unreliable -> fp64 refit
         if (!(lin <= 1e-2f * s2)) {
           refit = true;
           BFAST_WHY(0x20);
@@ -701,27 +784,27 @@ __global__ void __launch_bounds__(kTcThreads, 3)
         refit = true;
         BFAST_WHY(0x40);
       }
-      const float inv_scale = 1.0f / (sigma * sqrtf((float)nbar));
+      const float scale = sigma * sqrtf((float)nbar);  // MOSUM = W / scale (L524)
+      const float inv_scale = 1.0f / scale;
       sm100::tc_fence_before();
-      write_beta_operand(beta, 0.f);
-      // MOSUM seed (m^fst, L518): the last h-1 history residuals, corrected
-      // to the refined fit.  ra = slot of rank cr - hh (the next to drop).
+      write_beta_operand(beta);
+      // The ring holds ranks nbar-h .. nbar-1 as residuals of the first fit;
+      // correct each to the refined one, r = r0 - x_t dbeta, walking back
+      // from the newest (its date = the highest set bit of the chunk masks,
+      // scanned from the last history chunk).  W = their sum is the window of
+      // rank nbar - 1; the first monitoring step drops rank nbar - h, so
+      // W_0 = m^fst + r_nbar (L518).
       float W = 0.f;
-      uint32_t ra;
-      {
-        // walk back from the newest history residual; its date is the
-        // highest set bit of the chunk masks (scanned from the last chunk)
-        const int nseed = deg ? 0 : hh - 1;
+      if (!deg) {
         uint32_t a = wa;
         int cm = nch;
         uint32_t bits = 0;
-        for (int q = 0; q < nseed; ++q) {
+        for (int q = 0; q < hh; ++q) {
           a = (a == rbase ? rend : a) - C::RSLOT;
           while (bits == 0 && cm > 0) bits = (uint32_t)lds_u16(vbase + (--cm) * C::VSLOT);
           const int d = 31 - __clz(bits);
           bits ^= 1u << d;
-          const int t = cm * C::DC + d;
-          const float *xr = p.X + (size_t)t * p.KP;
+          const float *xr = p.X + (size_t)(cm * C::DC + d) * p.KP;
           float corr = 0.f;
 #pragma unroll
           for (int i = 0; i < K; i += 2) {
@@ -733,16 +816,13 @@ __global__ void __launch_bounds__(kTcThreads, 3)
           sts_f32(a, r);
           W += r;
         }
-        ra = (a == rbase ? rend : a) - C::RSLOT;  // rank cr - hh
-        if (deg) ra = wa;
-        // the window of j = 0 drops nothing: the slot of rank nbar - h (or
-        // the write slot for invalid pixels) reads as 0 at the first step
-        sts_f32(ra, 0.f);
       }
 
-      // ================= pass 2b: monitoring (Alg. 1 l.6-12, Fig. 12 ker 9-10)
+      // ================= pass 2, monitoring (Alg. 1 l.6-12, Fig. 12 ker 9-10)
       float msum = 0.f, mfirst = 0.f;
       int brk = -1, first = -1;
+      float mx = 0.f;  // max |W| over the valid monitoring dates so far
+      cr = nbar;
       bool tie = false;
       // largest 1-based rank with B == lambda (rank/nbar <= e), evaluated with
       // the exact boundary formula around floor(e * nbar)
@@ -755,7 +835,9 @@ __global__ void __launch_bounds__(kTcThreads, 3)
         for (int q = 1; q <= 4; ++q)
           if (nbar > 0 && boundary_f32(p.lambda, r0 + q, nbar) == p.lambda) rank_flat = r0 + q;
       }
-      const float lam = p.lambda, lam_lo = lam * (1.0f - kTieTol), lam_hi = lam * (1.0f + kTieTol);
+      const float lam = p.lambda;
+      // thresholds on W: |m| > lambda (1 - tol)  <=>  |W| > lambda (1 - tol) scale
+      float thr_lo = deg ? __int_as_float(0x7f800000) : lam * (1.0f - kTieTol) * scale;
       for (int c = 0; c < ncm; ++c) {
         sm100::mbar_wait_a(a_yfull + 8 * ys, yph);
         wait_yhat();
@@ -763,11 +845,6 @@ __global__ void __launch_bounds__(kTcThreads, 3)
         // B_j == lambda for every rank this chunk can reach (rank/nbar <= e):
         // warp-uniform fast path without the out-of-line boundary evaluation
         const bool fast = __all_sync(0xffffffffu, deg || cr + C::DC <= rank_flat);
-        if (first >= 0 && brk < 0 && !tie) {  // resolve a fast-path candidate
-          const float am = fabsf(mfirst);
-          if (am > lam_hi) brk = first;
-          else tie = true;
-        }
 #pragma unroll 1
         for (int hf = 0; hf < 2; ++hf) {
           float yh[8], yv[8];
@@ -775,60 +852,50 @@ __global__ void __launch_bounds__(kTcThreads, 3)
 #pragma unroll
           for (int d = 0; d < 8; ++d) yv[d] = Ys[(8 * hf + d) * 128 + tid];  // dates >= N read as NaN (TMA OOB)
           if (fast) {
-            uint32_t adv = 0;  // ring bytes advanced = valid dates * RSLOT
+            // B_j == lambda here: the first |m| > lambda(1 - tol) decides (a
+            // clear crossing is the break, a near tie goes to the fp64 refit).
+            // The dates only track max |W|; a half in which it crossed
+            // replays its 8 steps from the saved state (same arithmetic).
+            const float W0 = W;
+            float rr[8], oo[8];
 #pragma unroll
-            for (int d = 0; d < 8; ++d) {
-              const float y = yv[d];
-              const bool v = (y == y);
-              const float r = (y - c0) - yh[d];
-              const float old = lds_f32(ra);  // rank cr - h (zeroed phantom at j = 0)
-              const uint32_t inc = v ? C::RSLOT : 0u;
-              sts_f32_inc(wa, r, inc);
-              wa += inc;
-              ra += inc;
-              adv += inc;
-              wa = (wa == rend) ? rbase : wa;
-              ra = (ra == rend) ? rbase : ra;
-              if (v) W += r - old;
-              const float m = W * inv_scale;
-              if (v) msum += m;
-              // B_j == lambda here: the first |m| > lambda(1 - tol) decides --
-              // a clear crossing is the break, a near tie goes to the fp64 refit
-              const bool cand = v && first < 0 && fabsf(m) > lam_lo;
-              first = cand ? c * C::DC + 8 * hf + d : first;
-              mfirst = cand ? m : mfirst;
+            for (int d = 0; d < 8; ++d)
+              mon_date(yv[d], c0, yh[d], W, msum, mx, cr, wa, rend, hbytes, rr[d], oo[d]);
+            if (mx > thr_lo) {
+              float Wr = W0;
+#pragma unroll
+              for (int d = 0; d < 8; ++d) {
+                if (rr[d] == rr[d]) {
+                  Wr += rr[d] - oo[d];
+                  if (first < 0 && fabsf(Wr) > thr_lo) {
+                    first = c * C::DC + 8 * hf + d;
+                    mfirst = Wr;
+                  }
+                }
+              }
+              thr_lo = __int_as_float(0x7f800000);
             }
-            cr += adv >> 9;
           } else {
 #pragma unroll
             for (int d = 0; d < 8; ++d) {
-              const float y = yv[d];
-              const bool v = (y == y);
-              const float r = (y - c0) - yh[d];
-              const float old = lds_f32(ra);
-              sts_f32_inc(wa, r, v ? C::RSLOT : 0u);
-              const uint32_t wn = wa + C::RSLOT, rn = ra + C::RSLOT;
-              wa = v ? (wn == rend ? rbase : wn) : wa;
-              ra = v ? (rn == rend ? rbase : rn) : ra;
-              W = v ? W + (r - old) : W;
-              const float m = W * inv_scale;
-              msum += v ? m : 0.f;
-              if (v && brk < 0 && !tie && first < 0 && fabsf(m) > lam_lo) {
-                const int code = boundary_rare(m, cr + 1, nbar, lam);
+              float r, old;
+              mon_date(yv[d], c0, yh[d], W, msum, mx, cr, wa, rend, hbytes, r, old);
+              if (r == r && brk < 0 && !tie && first < 0 && fabsf(W) > thr_lo) {
+                const int code = boundary_rare(W * inv_scale, cr, nbar, lam);
                 tie = tie || (code >> 1);
                 brk = (code & 1) ? c * C::DC + 8 * hf + d : brk;
               }
-              cr += v;
             }
           }
         }
         release_yhat();
         warp_arrive(a_yempty + 8 * ys);  // every loaded value has been consumed
         yadvance();
-      }
-      if (first >= 0 && brk < 0 && !tie) {
-        if (fabsf(mfirst) > lam_hi) brk = first;
-        else tie = true;
+        if (first >= 0 && brk < 0 && !tie) {  // resolve a fast-path candidate
+          if (fabsf(mfirst * inv_scale) > lam * (1.0f + kTieTol)) brk = first;
+          else tie = true;
+          thr_lo = __int_as_float(0x7f800000);
+        }
       }
       const int Nbar = cr;
       if (Nbar - nbar < 1) deg = true;
@@ -838,7 +905,7 @@ __global__ void __launch_bounds__(kTcThreads, 3)
       const bool inside = pix < p.p0 + p.P;  // the last tile may be ragged
       if (inside) {
         p.out_break[pix] = deg ? -2 : brk;
-        p.out_mag[pix] = deg ? qnan : msum / (float)(Nbar - nbar);
+        p.out_mag[pix] = deg ? qnan : msum * inv_scale / (float)(Nbar - nbar);
         if (p.out_sigma) p.out_sigma[pix] = fit_ok ? sigma : qnan;
         if (p.out_nbar) p.out_nbar[pix] = nbar;
 #ifdef BFAST_REFIT_WHY

@@ -74,8 +74,31 @@ __device__ __forceinline__ bool mbar_try_wait_a(uint32_t a, uint32_t parity) {
       : "memory");
   return ok != 0;
 }
+// consumer-side wait: BFAST_CONS_WAIT 0 = poll try_wait, 1 = try_wait with a
+// suspend-time hint, N > 1 = poll with an N-ns sleep between probes
+#ifndef BFAST_CONS_WAIT
+#define BFAST_CONS_WAIT 0
+#endif
+__device__ __forceinline__ bool mbar_try_wait_a_hint(uint32_t a, uint32_t parity, uint32_t hint_ns) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
+      "selp.u32 %0, 1, 0, p;\n\t}"
+      : "=r"(ok)
+      : "r"(a), "r"(parity), "r"(hint_ns)
+      : "memory");
+  return ok != 0;
+}
 __device__ __forceinline__ void mbar_wait_a(uint32_t a, uint32_t parity) {
-  while (!mbar_try_wait_a(a, parity)) {
+  if (BFAST_CONS_WAIT == 0) {
+    while (!mbar_try_wait_a(a, parity)) {
+    }
+  } else if (BFAST_CONS_WAIT == 1) {
+    while (!mbar_try_wait_a_hint(a, parity, 0x100000u)) {
+    }
+  } else {
+    while (!mbar_try_wait_a(a, parity)) __nanosleep(BFAST_CONS_WAIT);
   }
 }
 
