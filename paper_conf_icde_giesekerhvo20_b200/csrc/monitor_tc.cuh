@@ -66,6 +66,14 @@ constexpr int kTcLaunchRegs = 80;
 constexpr int kTcAuxRegs = BFAST_TC_AUX_REGS;
 constexpr int kTcConsumerRegs = 2 * kTcLaunchRegs - kTcAuxRegs;
 
+// parts of the bf16 split of the first-fit residual r0 in the refinement
+// moment (2: hi truncated + lo rounded, ~17 bits; 3: three truncated parts,
+// exact -- measured magnitude error 2-5x lower for 2.7% more time)
+#ifndef BFAST_R0_PARTS
+#define BFAST_R0_PARTS 3
+#endif
+constexpr int kR0Parts = BFAST_R0_PARTS;
+
 template <int K>
 struct TcCfg {
   static constexpr int k = (K - 2) / 2;
@@ -97,12 +105,13 @@ struct TcCfg {
   static constexpr int ATILE = 128 * DC * 2;               // one [128 x 16] bf16 A tile
   static constexpr int OPBUF = 3 * ATILE;                  // pass 1: mask, y'hi, y'lo; pass 2: r0hi, r0lo
   static constexpr int RSLOT = 128 * 4;                    // ring slot: one residual per pixel
-  static constexpr int VSLOT = 128 * 2;                    // history validity: 16 bits per pixel per chunk
   // sy stack stages, nop operand buffers (2: the consumers fill one while the
-  // MMA reads the other), the MOSUM ring of hcap slots, nch validity masks
+  // MMA reads the other) and, in the same bytes, the MOSUM ring of hcap slots
+  // (the operands are dead once the refinement moment is accumulated, the
+  // ring is dead once the tile's monitoring is done)
   static constexpr size_t smem_bytes(int hcap, int nch, int sy, int nop) {
-    return (size_t)sy * YBYTES + (size_t)ST * TSTAGE + (size_t)nop * OPBUF + (size_t)hcap * RSLOT +
-           (size_t)((nch * VSLOT + 15) / 16) * 16;
+    const size_t ob = (size_t)nop * OPBUF, rg = (size_t)hcap * RSLOT;
+    return (size_t)sy * YBYTES + (size_t)ST * TSTAGE + ((ob > rg ? ob : rg) + 127) / 128 * 128 + 0 * nch;
   }
 };
 
@@ -160,28 +169,94 @@ __device__ __forceinline__ void p2h_date(float y, float c0, float yh, float &s2,
       : "+f"(s2), "+r"(vb), "=f"(h), "=f"(l)
       : "f"(y), "f"(c0), "f"(yh), "n"(1u << BIT));
 }
-// ... and the residual also enters the per-pixel ring of h slots at wa
-// (wrap at rend back by hbytes).
+// ... with a 3-way split of r0 by truncation (h + m + l exact)
 template <int BIT>
-__device__ __forceinline__ void p2h_date_ring(float y, float c0, float yh, float &s2, uint32_t &vb, float &h,
-                                              float &l, uint32_t &wa, uint32_t rend, uint32_t hbytes) {
-  asm volatile(
-      "{\n\t.reg .pred p, q;\n\t.reg .f32 r;\n\t"
+__device__ __forceinline__ void p2h_date3(float y, float c0, float yh, float &s2, uint32_t &vb, float &h, float &m,
+                                          float &l) {
+  asm("{\n\t.reg .pred p;\n\t.reg .f32 r, t;\n\t"
       "sub.f32 r, %5, %6;\n\t"
       "sub.f32 r, r, %7;\n\t"
       "setp.num.f32 p, r, r;\n\t"
       "@p fma.rn.f32 %0, r, r, %0;\n\t"
       "@p or.b32 %1, %1, %8;\n\t"
-      "@p st.shared.f32 [%4], r;\n\t"
-      "@p add.u32 %4, %4, 512;\n\t"
-      "setp.ge.u32 q, %4, %9;\n\t"
-      "@q sub.u32 %4, %4, %10;\n\t"
       "selp.f32 r, r, 0f00000000, p;\n\t"
       "and.b32 %2, r, 0xFFFF0000;\n\t"
-      "sub.f32 %3, r, %2;\n\t}"
-      : "+f"(s2), "+r"(vb), "=f"(h), "=f"(l), "+r"(wa)
-      : "f"(y), "f"(c0), "f"(yh), "n"(1u << BIT), "r"(rend), "r"(hbytes)
+      "sub.f32 t, r, %2;\n\t"
+      "and.b32 %3, t, 0xFFFF0000;\n\t"
+      "sub.f32 %4, t, %3;\n\t}"
+      : "+f"(s2), "+r"(vb), "=f"(h), "=f"(m), "=f"(l)
+      : "f"(y), "f"(c0), "f"(yh), "n"(1u << BIT));
+}
+// Seed date (history chunks re-read after the refinement): r = (y - c) -
+// yhat with the final beta; if r is a value it enters the per-pixel ring of
+// h slots at wa (wrap at rend back by hbytes).
+__device__ __forceinline__ void seed_date(float y, float c0, float yh, uint32_t &wa, uint32_t rend, uint32_t hbytes) {
+  asm volatile(
+      "{\n\t.reg .pred p, q;\n\t.reg .f32 r;\n\t"
+      "sub.f32 r, %1, %2;\n\t"
+      "sub.f32 r, r, %3;\n\t"
+      "setp.num.f32 p, r, r;\n\t"
+      "@p st.shared.f32 [%0], r;\n\t"
+      "@p add.u32 %0, %0, 512;\n\t"
+      "setp.ge.u32 q, %0, %4;\n\t"
+      "@q sub.u32 %0, %0, %5;\n\t}"
+      : "+r"(wa)
+      : "f"(y), "f"(c0), "f"(yh), "r"(rend), "r"(hbytes)
       : "memory");
+}
+// Cholesky factorisation (Alg. 1 l.3, an SPD Gram) in fp32 with hardware
+// reciprocal square roots: on return A holds L^T off the diagonal and dinv
+// the reciprocal pivots 1/l_jj.  Returns the smallest pivot ratio d_j / A_jj
+// (1 - R^2 of column j on the previous ones), the conditioning proxy of the
+// refit trigger.  The iterative refinement absorbs the ~1 ulp of rsqrt.
+template <int K>
+__device__ __forceinline__ float chol_factor_rsq(float (&A)[Tri<K>::kN], float (&dinv)[K]) {
+  float minratio = 1.f;
+  SFor<0, K>::run([&](auto jc) {
+    constexpr int j = decltype(jc)::value;
+    float d = A[Tri<K>::idx(j, j)];
+    SFor<0, j>::run([&](auto qc) {
+      constexpr int q = decltype(qc)::value;
+      d = fmaf(-A[Tri<K>::idx(q, j)], A[Tri<K>::idx(q, j)], d);
+    });
+    minratio = fminf(minratio, __fdividef(d, A[Tri<K>::idx(j, j)]));
+    const float inv = rsqrtf(fmaxf(d, 1e-30f));
+    dinv[j] = inv;
+    SFor<j + 1, K>::run([&](auto ic) {
+      constexpr int i = decltype(ic)::value;
+      float t = A[Tri<K>::idx(j, i)];
+      SFor<0, j>::run([&](auto qc) {
+        constexpr int q = decltype(qc)::value;
+        t = fmaf(-A[Tri<K>::idx(q, i)], A[Tri<K>::idx(q, j)], t);
+      });
+      A[Tri<K>::idx(j, i)] = t * inv;
+    });
+  });
+  return minratio;
+}
+// Solve L L^T x = b with the factor of chol_factor_rsq.
+template <int K>
+__device__ __forceinline__ void chol_solve_rsq(const float (&L)[Tri<K>::kN], const float (&dinv)[K], const float (&b)[K],
+                                               float (&x)[K]) {
+  float z[K];
+  SFor<0, K>::run([&](auto ic) {
+    constexpr int i = decltype(ic)::value;
+    float t = b[i];
+    SFor<0, i>::run([&](auto qc) {
+      constexpr int q = decltype(qc)::value;
+      t = fmaf(-L[Tri<K>::idx(q, i)], z[q], t);
+    });
+    z[i] = t * dinv[i];
+  });
+  SForDown<0, K>::run([&](auto ic) {
+    constexpr int i = decltype(ic)::value;
+    float t = z[i];
+    SFor<i + 1, K>::run([&](auto qc) {
+      constexpr int q = decltype(qc)::value;
+      t = fmaf(-L[Tri<K>::idx(i, q)], x[q], t);
+    });
+    x[i] = t * dinv[i];
+  });
 }
 // Monitoring date (Eq. (4) recurrence, L520-L525): r = y - yhat; the ring
 // slot at wa holds rank cr - h (`old`); if r is a value it replaces it,
@@ -263,14 +338,14 @@ __global__ void __launch_bounds__(kTcThreads, 3)
   using C = TcCfg<K>;
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ __align__(8) uint64_t yfull[C::SY_MAX], yempty[C::SY_MAX], tfull[C::ST], tempty[C::ST], opfull[2],
-      opfree[2], yhfull[2], yhfree[2], accready, betaready;
+      opfree[2], yhfull[2], yhfree[2], accready, betaready, seedready;
   __shared__ uint32_t tmem_base_s;
-  const int hcap = p.hcap, SY = tb.sy, NOP = tb.nop;
+  __shared__ int seed_slot[4];  // per consumer warp: first history chunk its MOSUM seed needs
+  const int SY = tb.sy, NOP = tb.nop;
   uint8_t *ystages = smem;
   uint8_t *tstages = ystages + SY * C::YBYTES;
   uint8_t *opb = tstages + C::ST * C::TSTAGE;
-  uint8_t *ring = opb + NOP * C::OPBUF;
-  uint8_t *vmask = ring + hcap * C::RSLOT;
+  uint8_t *ring = opb;  // aliases the operand buffers (TcCfg::smem_bytes)
   constexpr int NCW = 4;  // consumer warps
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -291,6 +366,7 @@ __global__ void __launch_bounds__(kTcThreads, 3)
     }
     sm100::mbar_init(&accready, 1);
     sm100::mbar_init(&betaready, NCW);
+    sm100::mbar_init(&seedready, NCW);
     sm100::fence_mbar_init();
   }
   if (warp == 0) sm100::tmem_alloc(&tmem_base_s, C::TMEM_COLS);
@@ -314,21 +390,28 @@ __global__ void __launch_bounds__(kTcThreads, 3)
         sm100::prefetch_tmap(&hmap);
         const uint64_t pol_first = sm100::policy_evict_first();
         int ys = 0;
-        uint32_t yph = 0;
+        uint32_t yph = 0, sph = 0;
         for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
           const int x0 = (int)(tile * 128);
-          for (int phase = 0; phase < 3; ++phase) {
-            const int nc = phase < 2 ? nch : ncm;
-            const int tbeg = phase < 2 ? 0 : n;
-            for (int c = 0; c < nc; ++c) {
+          // history twice (pass 1, pass 2: re-read from L2), then the seed
+          // chunks [s0, nch) once the consumers have found s0, then monitoring
+          int s0 = nch;
+          for (int phase = 0; phase < 4; ++phase) {
+            if (phase == 2) {
+              mbar_wait_sleep(&seedready, sph);
+              sph ^= 1;
+              s0 = min(min(seed_slot[0], seed_slot[1]), min(seed_slot[2], seed_slot[3]));
+            }
+            const int cb = phase == 2 ? s0 : 0, ce = phase < 3 ? nch : ncm;
+            for (int c = cb; c < ce; ++c) {
               mbar_wait_sleep(&yempty[ys], yph ^ 1);
               uint8_t *yst = ystages + ys * C::YBYTES;
               sm100::mbar_arrive_expect_tx(&yfull[ys], C::YBYTES);
-              if (phase == 0)
-                sm100::tma_load_2d(yst, &hmap, x0, c * C::DC, &yfull[ys]);  // re-read in pass 2 (L2)
+              if (phase < 2)
+                sm100::tma_load_2d(yst, &hmap, x0, c * C::DC, &yfull[ys]);  // read again later (L2)
               else
-                sm100::tma_load_2d_hint(yst, phase == 1 ? &hmap : &ymap, x0, tbeg + c * C::DC, &yfull[ys],
-                                        pol_first);  // last use
+                sm100::tma_load_2d_hint(yst, phase == 2 ? &hmap : &ymap, x0, (phase == 2 ? 0 : n) + c * C::DC,
+                                        &yfull[ys], pol_first);  // last use
               if (++ys == SY) {
                 ys = 0;
                 yph ^= 1;
@@ -341,17 +424,25 @@ __global__ void __launch_bounds__(kTcThreads, 3)
       // ------------------------------------------------------------ table producer
       if (lane == 0) {
         int ts = 0;
-        uint32_t tph = 0;
+        uint32_t tph = 0, sph = 0;
         for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
-          for (int phase = 0; phase < 3; ++phase) {
-            const int nc = phase < 2 ? nch : ncm;
+          int s0 = nch;
+          for (int phase = 0; phase < 4; ++phase) {
+            if (phase == 2) {
+              mbar_wait_sleep(&seedready, sph);
+              sph ^= 1;
+              s0 = min(min(seed_slot[0], seed_slot[1]), min(seed_slot[2], seed_slot[3]));
+            }
+            const int cb = phase == 2 ? s0 : 0, ce = phase < 3 ? nch : ncm;
+            // seed chunks only need the yhat part (the head) of their tab2 entry
             const uint32_t tabbytes = phase == 0 ? C::TAB1 : phase == 1 ? C::TAB2 : C::TABY;
-            const uint8_t *tabsrc = phase == 0 ? tb.tab1 : phase == 1 ? tb.tab2 : tb.taby;
-            for (int c = 0; c < nc; ++c) {
+            const uint32_t stride = phase == 0 ? C::TAB1 : phase < 3 ? C::TAB2 : C::TABY;
+            const uint8_t *tabsrc = phase == 0 ? tb.tab1 : phase < 3 ? tb.tab2 : tb.taby;
+            for (int c = cb; c < ce; ++c) {
               mbar_wait_sleep(&tempty[ts], tph ^ 1);
               uint8_t *tst = tstages + ts * C::TSTAGE;
               sm100::mbar_arrive_expect_tx(&tfull[ts], tabbytes);
-              sm100::bulk_g2s(tst, tabsrc + (size_t)c * tabbytes, tabbytes, &tfull[ts]);
+              sm100::bulk_g2s(tst, tabsrc + (size_t)c * stride, tabbytes, &tfull[ts]);
               if (++ts == C::ST) {
                 ts = 0;
                 tph ^= 1;
@@ -446,9 +537,9 @@ __global__ void __launch_bounds__(kTcThreads, 3)
             const uint32_t am = aop + ob * C::OPBUF;  // r0 hi, r0 lo tiles
             const uint32_t bx = tss + ts * C::TSTAGE + C::B3_BYTES;
             const uint32_t dD = tbase + C::COL_DB;
-            // r0hi (x_hi + x_mid + x_lo) + r0lo (x_hi + x_mid)
+            // r0hi (x_hi + x_mid + x_lo) + r0lo (x_hi + x_mid) [+ r0lo2 x_hi]
 #pragma unroll
-            for (int e = 0; e < 2; ++e)
+            for (int e = 0; e < kR0Parts; ++e)
 #pragma unroll
               for (int q = 0; q < 3 - e; ++q)
                 sm100::umma_bf16(dD, sm100::smem_desc(am + e * C::ATILE, 2048, 128),
@@ -461,12 +552,15 @@ __global__ void __launch_bounds__(kTcThreads, 3)
             ++opcnt;
             tadvance();
           }
-          // pass 2, monitoring: yhat with the refined beta, two chunks ahead
+          // pass 3, seed chunks + monitoring: yhat with the refined beta, two
+          // chunks ahead (the consumers published s0 before betaready)
           mbar_wait_mma(&betaready, bcnt & 1);
           ++bcnt;
-          for (int a = 0; a < 2 && a < ncm; ++a) issue_yhat(a);
-          for (int c = 0; c < ncm; ++c) {
-            if (c + 2 < ncm) issue_yhat(2);
+          const int s0 = min(min(seed_slot[0], seed_slot[1]), min(seed_slot[2], seed_slot[3]));
+          const int n3 = nch - s0 + ncm;
+          for (int a = 0; a < 2 && a < n3; ++a) issue_yhat(a);
+          for (int c = 0; c < n3; ++c) {
+            if (c + 2 < n3) issue_yhat(2);
             sm100::umma_commit(&tempty[ts]);  // chunk c's table was read by its yhat MMA
             tadvance();
           }
@@ -478,10 +572,8 @@ __global__ void __launch_bounds__(kTcThreads, 3)
     sm100::setmaxnreg_inc<kTcConsumerRegs>();
     const uint32_t lanebase = tbase + ((uint32_t)(32 * warp) << 16);
     const float qnan = __int_as_float(0x7fc00000);
-    // ring: slot s = 128 residuals f32, this thread's at rbase + s*RSLOT;
-    // history validity: 16 bits per chunk, this thread's at vbase + c*VSLOT
+    // ring: slot s = 128 residuals f32, this thread's at rbase + s*RSLOT
     const uint32_t rbase = sm100::smem_u32(ring) + 4 * tid;
-    const uint32_t vbase = sm100::smem_u32(vmask) + 2 * tid;
     int ys = 0;
     uint32_t yph = 0, opcnt = 0, yuse = 0, acnt = 0;
     // 32-bit shared addresses of the barriers this warp waits on / arrives at
@@ -560,6 +652,9 @@ __global__ void __launch_bounds__(kTcThreads, 3)
 
     for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
       const int64_t pix = p.p0 + tile * 128 + tid;
+      // the operand buffers reuse the ring's bytes: every consumer warp must
+      // be done with the previous tile's monitoring before any writes them
+      asm volatile("bar.sync 1, 128;" ::: "memory");
       // ================= pass 1: masked Gram + moment on the tensor cores
       float c0 = qnan, ymax = 0.f;
       bool have = false;
@@ -673,9 +768,10 @@ __global__ void __launch_bounds__(kTcThreads, 3)
 #else
 #define BFAST_WHY(b)
 #endif
+      float dinv[K];
       {
-        const float minratio = chol_factor<K, float>(A);
-        chol_solve<K, float>(A, b, beta);
+        const float minratio = chol_factor_rsq<K>(A, dinv);
+        chol_solve_rsq<K>(A, dinv, b, beta);
         if (!deg && !(minratio >= (float)kRefitRatio)) {
           refit = true;
           BFAST_WHY(0x10);
@@ -689,22 +785,16 @@ __global__ void __launch_bounds__(kTcThreads, 3)
       write_beta_operand(beta);
 
       // ================= pass 2, history: residuals r0 of the first fit,
-      // sigma-hat sums, the refinement moment operand, the seed ring.
-      // The ring holds h slots (hh for invalid pixels); the slot about to be
-      // written always holds rank cr - h.  Only chunks that can contain one
-      // of the last h valid history dates of some lane of the warp write it;
-      // starting earlier only writes ranks that are overwritten later.
+      // sigma-hat sums, the refinement moment operand; and which chunk holds
+      // the oldest residual of the MOSUM seed (rank nbar - h: the window of
+      // the first monitoring date reaches back to rank nbar - h + 1)
       const int hh = deg ? 1 : h;
-      const uint32_t hbytes = (uint32_t)hh * C::RSLOT, rend = rbase + hbytes;
-      const int ring_from = nbar - hh;  // rank of the oldest residual the ring must keep
+      const int ring_from = nbar - hh;
       float s2 = 0.f;
-      uint32_t wa = rbase;
-      int cr = 0;  // valid history dates before the current chunk
-      bool ring_on = false;
+      int cr = 0;       // valid history dates before the current chunk
+      int sc = nch;     // first chunk holding a rank >= ring_from (nch: no seed needed)
       for (int c = 0; c < nch; ++c) {
         sm100::mbar_wait_a(a_yfull + 8 * ys, yph);
-        // this chunk can hold rank nbar - hh or later for some lane of the warp
-        ring_on = ring_on || __any_sync(0xffffffffu, cr + C::DC > ring_from);
         wait_yhat();
         const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
         uint8_t *ob = nullptr;
@@ -715,44 +805,53 @@ __global__ void __launch_bounds__(kTcThreads, 3)
           load_yhat8(hf, yh);
 #pragma unroll
           for (int d = 0; d < 8; ++d) yv[d] = Ys[(8 * hf + d) * 128 + tid];  // dates >= n read as NaN (hmap)
-          float rh[8], rl[8];
+          float rh[8], rm[8], rl[8];
           uint32_t v8 = 0;
-          if (ring_on) {
-            SFor<0, 8>::run([&](auto dc) {
-              constexpr int d = decltype(dc)::value;
-              p2h_date_ring<d>(yv[d], c0, yh[d], s2, v8, rh[d], rl[d], wa, rend, hbytes);
-            });
-          } else {
-            SFor<0, 8>::run([&](auto dc) {
-              constexpr int d = decltype(dc)::value;
+          SFor<0, 8>::run([&](auto dc) {
+            constexpr int d = decltype(dc)::value;
+            if (kR0Parts == 3)
+              p2h_date3<d>(yv[d], c0, yh[d], s2, v8, rh[d], rm[d], rl[d]);
+            else
               p2h_date<d>(yv[d], c0, yh[d], s2, v8, rh[d], rl[d]);
-            });
-          }
+          });
           vb |= v8 << (8 * hf);
           if (hf == 0) ob = opbuf_acquire();
           const uint32_t off = sm100::kmajor_off(tid, 8 * hf, 128);
-          // r0 = hi (truncated, exact) + lo (rounded to nearest: unbiased)
           *reinterpret_cast<uint4 *>(ob + off) = make_uint4(
               pack_hi16(rh[0], rh[1]), pack_hi16(rh[2], rh[3]), pack_hi16(rh[4], rh[5]), pack_hi16(rh[6], rh[7]));
-          *reinterpret_cast<uint4 *>(ob + C::ATILE + off) =
-              make_uint4(sm100::pack_bf16x2(rl[0], rl[1]), sm100::pack_bf16x2(rl[2], rl[3]),
-                         sm100::pack_bf16x2(rl[4], rl[5]), sm100::pack_bf16x2(rl[6], rl[7]));
+          if (kR0Parts == 3) {
+            *reinterpret_cast<uint4 *>(ob + C::ATILE + off) = make_uint4(
+                pack_hi16(rm[0], rm[1]), pack_hi16(rm[2], rm[3]), pack_hi16(rm[4], rm[5]), pack_hi16(rm[6], rm[7]));
+            *reinterpret_cast<uint4 *>(ob + 2 * C::ATILE + off) = make_uint4(
+                pack_hi16(rl[0], rl[1]), pack_hi16(rl[2], rl[3]), pack_hi16(rl[4], rl[5]), pack_hi16(rl[6], rl[7]));
+          } else {
+            // r0 = hi (truncated, exact) + lo (rounded to nearest: unbiased)
+            *reinterpret_cast<uint4 *>(ob + C::ATILE + off) =
+                make_uint4(sm100::pack_bf16x2(rl[0], rl[1]), sm100::pack_bf16x2(rl[2], rl[3]),
+                           sm100::pack_bf16x2(rl[4], rl[5]), sm100::pack_bf16x2(rl[6], rl[7]));
+          }
         }
-        sts_u16(vbase + c * C::VSLOT, (uint16_t)vb);
         cr += __popc(vb);
+        if (sc == nch && !deg && cr > ring_from) sc = c;
         release_yhat();
         warp_arrive(a_yempty + 8 * ys);  // every loaded value has been consumed
         opbuf_publish();
         yadvance();
+      }
+      // the tile's seed chunks start at the smallest sc: publish this warp's
+      const int sw = __reduce_min_sync(0xffffffffu, sc);
+      if (lane == 0) {
+        seed_slot[warp] = sw;
+        sm100::mbar_arrive_a(sm100::smem_u32(&seedready));
       }
       sm100::mbar_wait_a(a_accready, acnt & 1);
       ++acnt;
       sm100::tc_fence_after();
 
       // ================= refinement: beta = beta0 + A^-1 db; sigma-hat
-      float sigma, dbf[K];
+      float sigma;
       {
-        float db[K];
+        float db[K], dbf[K];
         {
           float v16[16];
           sm100::tmem_ld16(lanebase + C::COL_DB, v16);
@@ -760,7 +859,7 @@ __global__ void __launch_bounds__(kTcThreads, 3)
 #pragma unroll
           for (int i = 0; i < K; ++i) db[i] = v16[i];
         }
-        chol_solve<K, float>(A, db, dbf);
+        chol_solve_rsq<K>(A, dinv, db, dbf);
         float lin = 0.f;
 #pragma unroll
         for (int i = 0; i < K; ++i) {
@@ -788,53 +887,52 @@ __global__ void __launch_bounds__(kTcThreads, 3)
       const float inv_scale = 1.0f / scale;
       sm100::tc_fence_before();
       write_beta_operand(beta);
-      // The ring holds ranks nbar-h .. nbar-1 as residuals of the first fit;
-      // correct each to the refined one, r = r0 - x_t dbeta, walking back
-      // from the newest (its date = the highest set bit of the chunk masks,
-      // scanned from the last history chunk).  W = their sum is the window of
-      // rank nbar - 1; the first monitoring step drops rank nbar - h, so
-      // W_0 = m^fst + r_nbar (L518).
-      float W = 0.f;
-      if (!deg) {
-        uint32_t a = wa;
-        int cm = nch;
-        uint32_t bits = 0;
-        for (int q = 0; q < hh; ++q) {
-          a = (a == rbase ? rend : a) - C::RSLOT;
-          while (bits == 0 && cm > 0) bits = (uint32_t)lds_u16(vbase + (--cm) * C::VSLOT);
-          const int d = 31 - __clz(bits);
-          bits ^= 1u << d;
-          const float *xr = p.X + (size_t)(cm * C::DC + d) * p.KP;
-          float corr = 0.f;
-#pragma unroll
-          for (int i = 0; i < K; i += 2) {
-            const float2 xx = __ldg(reinterpret_cast<const float2 *>(xr + i));
-            corr = fmaf(dbf[i], xx.x, corr);
-            corr = fmaf(dbf[i + 1], xx.y, corr);
-          }
-          const float r = lds_f32(a) - corr;
-          sts_f32(a, r);
-          W += r;
-        }
-      }
 
-      // ================= pass 2, monitoring (Alg. 1 l.6-12, Fig. 12 ker 9-10)
+      // ================= pass 3, seed: the history chunks [s0, nch) again,
+      // residuals of the refined fit into the per-pixel ring of h slots.  The
+      // slot about to be written always holds rank cr - h; writing from any
+      // rank <= nbar - h on leaves ranks nbar-h .. nbar-1 in the ring with the
+      // write slot on rank nbar - h.  A warp starts at its own first chunk sw.
+      const uint32_t hbytes = (uint32_t)hh * C::RSLOT, rend = rbase + hbytes;
+      uint32_t wa = rbase;
+      // every consumer warp has published sw and written its last operands
+      // (the ring overwrites them); the producers wait on seedready instead
+      asm volatile("bar.sync 1, 128;" ::: "memory");
+      const int s0 = min(min(seed_slot[0], seed_slot[1]), min(seed_slot[2], seed_slot[3]));
+      for (int c = s0; c < nch; ++c) {
+        sm100::mbar_wait_a(a_yfull + 8 * ys, yph);
+        wait_yhat();
+        if (c >= sw) {
+          const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
+#pragma unroll 1
+          for (int hf = 0; hf < 2; ++hf) {
+            float yh[8], yv[8];
+            load_yhat8(hf, yh);
+#pragma unroll
+            for (int d = 0; d < 8; ++d) yv[d] = Ys[(8 * hf + d) * 128 + tid];
+#pragma unroll
+            for (int d = 0; d < 8; ++d) seed_date(yv[d], c0, yh[d], wa, rend, hbytes);
+          }
+        }
+        release_yhat();
+        warp_arrive(a_yempty + 8 * ys);
+        yadvance();
+      }
+      // W = the window of rank nbar - 1 (ranks nbar-h .. nbar-1); the first
+      // monitoring step drops rank nbar - h, so W_0 = m^fst + r_nbar (L518)
+      float W = 0.f;
+      if (!deg)
+        for (uint32_t a = rbase; a < rend; a += C::RSLOT) W += lds_f32(a);
+
+      // ================= pass 3, monitoring (Alg. 1 l.6-12, Fig. 12 ker 9-10)
       float msum = 0.f, mfirst = 0.f;
       int brk = -1, first = -1;
       float mx = 0.f;  // max |W| over the valid monitoring dates so far
       cr = nbar;
       bool tie = false;
-      // largest 1-based rank with B == lambda (rank/nbar <= e), evaluated with
-      // the exact boundary formula around floor(e * nbar)
-      int rank_flat;
-      {
-        int r0 = (int)(2.718281828f * (float)nbar) - 2;
-        r0 = r0 < 0 ? 0 : r0;
-        rank_flat = r0;
-#pragma unroll
-        for (int q = 1; q <= 4; ++q)
-          if (nbar > 0 && boundary_f32(p.lambda, r0 + q, nbar) == p.lambda) rank_flat = r0 + q;
-      }
+      // a 1-based rank up to which B == lambda (rank/nbar <= e): floor(e nbar)
+      // - 3 keeps ln(rank/nbar) below 1 by more than f32 rounding for any nbar
+      const int rank_flat = max((int)(2.718281828f * (float)nbar) - 3, 0);
       const float lam = p.lambda;
       // thresholds on W: |m| > lambda (1 - tol)  <=>  |W| > lambda (1 - tol) scale
       float thr_lo = deg ? __int_as_float(0x7f800000) : lam * (1.0f - kTieTol) * scale;

@@ -24,7 +24,8 @@ def line_table(lib, kern):
     d = tempfile.mkdtemp()
     subprocess.run(["cuobjdump", "-xelf", "all", os.path.abspath(lib)], cwd=d, capture_output=True)
     cub = [f for f in os.listdir(d) if f.endswith(".cubin")][0]
-    dis = subprocess.run(["nvdisasm", "-g", "-c", os.path.join(d, cub)], capture_output=True, text=True).stdout
+    flag = "-gi" if os.environ.get("NCU_LINES_CALLSITE") else "-g"
+    dis = subprocess.run(["nvdisasm", flag, "-c", os.path.join(d, cub)], capture_output=True, text=True).stdout
     tab, cur, on = {}, None, False
     for ln in dis.splitlines():
         if ln.startswith(".text."):
@@ -32,9 +33,13 @@ def line_table(lib, kern):
             continue
         if not on:
             continue
-        m = re.search(r'//## File "([^"]+)", line (\d+)', ln)
+        m = re.search(r'//## File "([^"]+)", line (\d+)(?: inlined at "([^"]+)", line (\d+))?', ln)
         if m:
-            cur = (os.path.basename(m.group(1)), int(m.group(2)))
+            # NCU_LINES_CALLSITE=1: charge inlined helpers to their call site
+            if m.group(3):
+                cur = (os.path.basename(m.group(3)), int(m.group(4)))
+            else:
+                cur = (os.path.basename(m.group(1)), int(m.group(2)))
             continue
         m = re.match(r"\s+/\*([0-9a-f]{4,})\*/\s+(.*)", ln)
         if m:
