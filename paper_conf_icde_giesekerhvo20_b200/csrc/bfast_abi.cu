@@ -155,14 +155,14 @@ PFN_encodeTiled get_encode() {
   return fn;
 }
 
-// Tensor map of the stack range [p0, p0+P) x [0, N): box 128 px x 16 dates,
+// Tensor map of the stack range [p0, p0+P) x [0, N): box 128*kTcPx px x 16 dates,
 // out-of-bounds elements read as NaN (= missing).
 bool make_stack_map(CUtensorMap *m, const float *Y, int64_t ldY, int64_t P, int64_t N) {
   PFN_encodeTiled enc = get_encode();
   if (!enc) return false;
   cuuint64_t dims[2] = {(cuuint64_t)P, (cuuint64_t)N};
   cuuint64_t strides[1] = {(cuuint64_t)ldY * sizeof(float)};
-  cuuint32_t box[2] = {128, 16};
+  cuuint32_t box[2] = {128 * bfast::kTcPx, 16};
   cuuint32_t es[2] = {1, 1};
   return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void *)Y, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
              CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -194,8 +194,8 @@ inline size_t kmaj(int row, int k, int rows) { return sm100::kmajor_off(row, k, 
 // canonical K-major layout, fp64 values split into bf16 parts.
 //   tab1[c] (history chunk c, pass 1): F_hi | F_mid | F_lo ([NGn x 16] each,
 //           row q = moment function f_q (the last one the constant 1),
-//           column d = date 16c + d), then x_hi | x_mid | x_lo ([KBn x 16]
-//           each, row i = basis column i);
+//           column d = date 16c + d), then x_hi | x_mid ([KBn x 16]
+//           each, row i = basis column i; x_lo is only needed in pass 2);
 //   tab2[c] (history chunk c, pass 2): the yhat table [16 x KY] of its dates
 //           (row d = date, K index = 6 blocks of K: x_hi | x_mid | x_lo |
 //           x_hi | x_mid | x_hi, paired in the GEMM with beta hi | hi | hi |
@@ -243,12 +243,12 @@ void build_tc_tables(const bfast_plan &pl, std::vector<uint16_t> &tab, size_t &o
       for (int b = 0; b < 6; ++b) b3[kmaj(d, b * K + i, C::DC)] = blk[b];
     }
   };
-  auto put_bx = [&](uint16_t *bx, int d, const double *xv) {  // 3 x [KBn x 16]
+  auto put_bx = [&](uint16_t *bx, int d, const double *xv, int parts) {  // parts x [KBn x 16]
     for (int i = 0; i < K; ++i) {
       uint16_t h, m, l;
       split3(xv[i], h, m, l);
       const uint16_t prt[3] = {h, m, l};
-      for (int e = 0; e < 3; ++e) bx[e * C::BX_BYTES / 2 + kmaj(i, d, C::KBn)] = prt[e];
+      for (int e = 0; e < parts; ++e) bx[e * C::BX_BYTES / 2 + kmaj(i, d, C::KBn)] = prt[e];
     }
   };
   for (int c = 0; c < nch; ++c) {
@@ -265,9 +265,9 @@ void build_tc_tables(const bfast_plan &pl, std::vector<uint16_t> &tab, size_t &o
         const uint16_t prt[3] = {h, m, l};
         for (int e = 0; e < 3; ++e) bf[e * C::BF_BYTES / 2 + kmaj(q, d, C::NGn)] = prt[e];
       }
-      put_bx(bf + 3 * C::BF_BYTES / 2, d, x);
+      put_bx(bf + 3 * C::BF_BYTES / 2, d, x, 2);
       put_b3(t2, d, x);
-      put_bx(t2 + C::B3_BYTES / 2, d, x);
+      put_bx(t2 + C::B3_BYTES / 2, d, x, 3);
     }
   }
   for (int c = 0; c < ncm; ++c) {
@@ -349,7 +349,7 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
   int tc_sy = 2, tc_nop = 1, per_sm = 0;
   {
     const int cand[4][2] = {{2, 2}, {2, 1}, {3, 2}, {3, 1}};
-    const int reg_cap = 65536 / (bfast::kTcThreads * bfast::kTcLaunchRegs);
+    const int reg_cap = std::min(65536 / (bfast::kTcThreads * bfast::kTcLaunchRegs), bfast::kTcCtasPerSm);
     const int tmem_cap = 512 / TC::TMEM_COLS;
     for (auto &c : cand) {
       const size_t b = TC::smem_bytes(tc_hcap, pl.nch, c[0], c[1]);
@@ -367,7 +367,7 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
   }
   if (const char *lay = std::getenv("BFAST_TC_LAYOUT")) {  // experiments: "sy,nop,per_sm"
     int a = 0, b = 0, c = 0;
-    if (std::sscanf(lay, "%d,%d,%d", &a, &b, &c) == 3 && a >= 2 && a <= 4 && b >= 1 && b <= 2 && c >= 1 && c <= 3) {
+    if (std::sscanf(lay, "%d,%d,%d", &a, &b, &c) == 3 && a >= 2 && a <= 4 && b >= 1 && b <= 2 && c >= 1 && c <= 4) {
       tc_sy = a;
       tc_nop = b;
       per_sm = c;
@@ -382,7 +382,7 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
   CUtensorMap ymap, hmap;  // full stack; history only (dates >= n out of bounds)
   const bool tma_ok = tc_ok && make_stack_map(&ymap, prm.Y + prm.p0, prm.ldY, prm.P, pl.N) &&
                       make_stack_map(&hmap, prm.Y + prm.p0, prm.ldY, prm.P, pl.n);
-  const int64_t ntiles = tma_ok ? (prm.P + 127) / 128 : 0;
+  const int64_t ntiles = tma_ok ? (prm.P + TC::PIX - 1) / TC::PIX : 0;
   // the refit list/counter are plan scratch: order executions on any stream
   CUDA_TRY(cudaStreamWaitEvent(st, pl.scratch_free, 0));
   CUDA_TRY(cudaMemsetAsync(prm.refit_count, 0, sizeof(int32_t), st));

@@ -59,7 +59,16 @@ namespace bfast {
 // producers drop to kTcAuxRegs, the consumers rise to kTcConsumerRegs
 // (80*256 = 128*kTcAuxRegs + 128*kTcConsumerRegs).
 constexpr int kTcThreads = 256;
-constexpr int kTcLaunchRegs = 80;
+#ifndef BFAST_TC_PX
+#define BFAST_TC_PX 2
+#endif
+constexpr int kTcPx = BFAST_TC_PX;  // pixels per consumer thread (tile = 128 * kTcPx pixels)
+
+#ifndef BFAST_TC_CTAS
+#define BFAST_TC_CTAS (BFAST_TC_PX == 2 ? 2 : 3)
+#endif
+constexpr int kTcCtasPerSm = BFAST_TC_CTAS;               // register budget: CTAs per SM
+constexpr int kTcLaunchRegs = kTcCtasPerSm == 4 ? 64 : kTcCtasPerSm == 3 ? 80 : 128;
 #ifndef BFAST_TC_AUX_REGS
 #define BFAST_TC_AUX_REGS 32
 #endif
@@ -74,7 +83,7 @@ constexpr int kTcConsumerRegs = 2 * kTcLaunchRegs - kTcAuxRegs;
 #endif
 constexpr int kR0Parts = BFAST_R0_PARTS;
 
-template <int K>
+template <int K, int PX = kTcPx>
 struct TcCfg {
   static constexpr int k = (K - 2) / 2;
   static constexpr int NF = 2 + 6 * k;                     // masked moment functions
@@ -82,29 +91,37 @@ struct TcCfg {
   static constexpr int KBn = ((K + 15) / 16) * 16;         // moment GEMM N
   static constexpr int KY = ((6 * K + 15) / 16) * 16;      // yhat GEMM K
   static constexpr int DC = 16;                            // dates per chunk
-  // TMEM columns.  Pass 1: two accumulator sets [Gram | moment]; pass 2
-  // (after the solve has read them): two yhat slots, the beta operand (the A
-  // operand of the yhat GEMM, bf16 pairs) and the refinement moment.
+  static constexpr int PIX = 128 * PX;                     // pixels per tile
+  // TMEM columns (lane = consumer thread; a thread's PX pixels are the same
+  // lane of PX column groups).  Pass 1: two accumulator sets [Gram | moment]
+  // per pixel group; pass 2 (after the solve has read them): two yhat slots,
+  // the beta operand (the A operand of the yhat GEMM, bf16 pairs) and the
+  // refinement moment, per pixel group.
   static constexpr int SET = NGn + KBn;
-  static constexpr int COL_Y = 0, COL_A3 = 2 * DC, COL_DB = ((COL_A3 + KY / 2 + 15) / 16) * 16;
-  static constexpr int COLS_P1 = 2 * SET, COLS_P2 = COL_DB + KBn;
+  static constexpr int A3W = ((KY / 2 + 15) / 16) * 16;
+  static constexpr int COLS_P1 = 2 * PX * SET;
+  static constexpr __host__ __device__ int col_set(int s, int q) { return (s * PX + q) * SET; }
+  static constexpr __host__ __device__ int col_y(int slot, int q) { return (slot * PX + q) * DC; }
+  static constexpr __host__ __device__ int col_a3(int q) { return 2 * PX * DC + q * A3W; }
+  static constexpr __host__ __device__ int col_db(int q) { return 2 * PX * DC + PX * A3W + q * KBn; }
+  static constexpr int COLS_P2 = 2 * PX * DC + PX * A3W + PX * KBn;
   static constexpr int COLS_USED = COLS_P1 > COLS_P2 ? COLS_P1 : COLS_P2;
   static constexpr int TMEM_COLS = COLS_USED <= 32 ? 32 : COLS_USED <= 64 ? 64 : COLS_USED <= 128 ? 128
                                    : COLS_USED <= 256 ? 256 : 512;
   static constexpr int BF_BYTES = NGn * DC * 2;            // one part of the Gram table [NGn x 16]
   static constexpr int BX_BYTES = KBn * DC * 2;            // one part of x [KBn x 16]
   static constexpr int B3_BYTES = DC * KY * 2;             // yhat table [16 x KY]
-  static constexpr int TAB1 = 3 * BF_BYTES + 3 * BX_BYTES; // pass 1 (history): F parts, x parts
+  static constexpr int TAB1 = 3 * BF_BYTES + 2 * BX_BYTES; // pass 1 (history): F parts, x hi/mid
   static constexpr int TAB2 = B3_BYTES + 3 * BX_BYTES;     // pass 2 history: yhat table, x parts
   static constexpr int TABY = B3_BYTES;                    // pass 2 monitoring: yhat table
   static constexpr int TABMAX = TAB1 > TAB2 ? TAB1 : TAB2;
-  static constexpr int YBYTES = DC * 128 * 4;             // one [16 dates x 128 px] box
+  static constexpr int YBYTES = DC * PIX * 4;              // one [16 dates x PIX px] box
   static constexpr int TSTAGE = ((TABMAX + 127) / 128) * 128;
   static constexpr int SY_MAX = 4;                         // stack ring stages (released on read)
   static constexpr int ST = 3;                             // table ring stages (released by MMA commit)
-  static constexpr int ATILE = 128 * DC * 2;               // one [128 x 16] bf16 A tile
-  static constexpr int OPBUF = 3 * ATILE;                  // pass 1: mask, y'hi, y'lo; pass 2: r0hi, r0lo
-  static constexpr int RSLOT = 128 * 4;                    // ring slot: one residual per pixel
+  static constexpr int ATILE = 128 * DC * 2;               // one [128 x 16] bf16 A tile (one pixel group)
+  static constexpr int OPBUF = 3 * PX * ATILE;             // pass 1: mask, y'hi, y'lo; pass 2: r0 parts
+  static constexpr int RSLOT = PIX * 4;                    // ring slot: one residual per pixel
   // sy stack stages, nop operand buffers (2: the consumers fill one while the
   // MMA reads the other) and, in the same bytes, the MOSUM ring of hcap slots
   // (the operands are dead once the refinement moment is accumulated, the
@@ -190,6 +207,7 @@ __device__ __forceinline__ void p2h_date3(float y, float c0, float yh, float &s2
 // Seed date (history chunks re-read after the refinement): r = (y - c) -
 // yhat with the final beta; if r is a value it enters the per-pixel ring of
 // h slots at wa (wrap at rend back by hbytes).
+template <int RSLOT>
 __device__ __forceinline__ void seed_date(float y, float c0, float yh, uint32_t &wa, uint32_t rend, uint32_t hbytes) {
   asm volatile(
       "{\n\t.reg .pred p, q;\n\t.reg .f32 r;\n\t"
@@ -197,11 +215,11 @@ __device__ __forceinline__ void seed_date(float y, float c0, float yh, uint32_t 
       "sub.f32 r, r, %3;\n\t"
       "setp.num.f32 p, r, r;\n\t"
       "@p st.shared.f32 [%0], r;\n\t"
-      "@p add.u32 %0, %0, 512;\n\t"
+      "@p add.u32 %0, %0, %6;\n\t"
       "setp.ge.u32 q, %0, %4;\n\t"
       "@q sub.u32 %0, %0, %5;\n\t}"
       : "+r"(wa)
-      : "f"(y), "f"(c0), "f"(yh), "r"(rend), "r"(hbytes)
+      : "f"(y), "f"(c0), "f"(yh), "r"(rend), "r"(hbytes), "n"(RSLOT)
       : "memory");
 }
 // Cholesky factorisation (Alg. 1 l.3, an SPD Gram) in fp32 with hardware
@@ -262,6 +280,7 @@ __device__ __forceinline__ void chol_solve_rsq(const float (&L)[Tri<K>::kN], con
 // slot at wa holds rank cr - h (`old`); if r is a value it replaces it,
 // W += r - old, msum += W, cr += 1 and mx = max(mx, |W|).  r and old are
 // returned for the exact replay of a half-chunk in which mx crossed.
+template <int RSLOT>
 __device__ __forceinline__ void mon_date(float y, float c0, float yh, float &W, float &msum, float &mx, int &cr,
                                          uint32_t &wa, uint32_t rend, uint32_t hbytes, float &r, float &old) {
   asm volatile(
@@ -271,7 +290,7 @@ __device__ __forceinline__ void mon_date(float y, float c0, float yh, float &W, 
       "setp.num.f32 p, %5, %5;\n\t"
       "ld.shared.f32 %6, [%4];\n\t"
       "@p st.shared.f32 [%4], %5;\n\t"
-      "@p add.u32 %4, %4, 512;\n\t"
+      "@p add.u32 %4, %4, %12;\n\t"
       "setp.ge.u32 q, %4, %10;\n\t"
       "@q sub.u32 %4, %4, %11;\n\t"
       "@p add.s32 %3, %3, 1;\n\t"
@@ -281,7 +300,7 @@ __device__ __forceinline__ void mon_date(float y, float c0, float yh, float &W, 
       "abs.f32 t, %0;\n\t"
       "@p max.f32 %2, %2, t;\n\t}"
       : "+f"(W), "+f"(msum), "+f"(mx), "+r"(cr), "+r"(wa), "=f"(r), "=f"(old)
-      : "f"(y), "f"(c0), "f"(yh), "r"(rend), "r"(hbytes)
+      : "f"(y), "f"(c0), "f"(yh), "r"(rend), "r"(hbytes), "n"(RSLOT)
       : "memory");
 }
 // producer-side waits with back-off so a waiting producer does not steal
@@ -332,10 +351,11 @@ __device__ __forceinline__ float bf16_round(float v) {
 }
 
 template <int K>
-__global__ void __launch_bounds__(kTcThreads, 3)
+__global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
     monitor_tc_kernel(MonitorParams p, TcTables tb, const __grid_constant__ CUtensorMap ymap,
                       const __grid_constant__ CUtensorMap hmap) {
-  using C = TcCfg<K>;
+  constexpr int PX = kTcPx;
+  using C = TcCfg<K, PX>;
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ __align__(8) uint64_t yfull[C::SY_MAX], yempty[C::SY_MAX], tfull[C::ST], tempty[C::ST], opfull[2],
       opfree[2], yhfull[2], yhfree[2], accready, betaready, seedready;
@@ -378,12 +398,12 @@ __global__ void __launch_bounds__(kTcThreads, 3)
 
   if (warp >= NCW) {
     // producer warpgroup: three single-thread roles need few registers; hand
-    // them to the consumer warpgroup (3 CTAs per SM fit the register file)
+    // them to the consumer warpgroup
     sm100::setmaxnreg_dec<kTcAuxRegs>();
     if (warp == 4) {
       // ------------------------------------------------------------ stack producer
       if (lane == 0) {
-        // one 2-D TMA box [16 dates x 128 px] per chunk.  History chunks read
+        // one 2-D TMA box [16 dates x PIX px] per chunk.  History chunks read
         // through `hmap` (dates >= n are out of bounds), monitoring chunks
         // through `ymap`; out-of-bounds elements arrive as NaN = missing.
         sm100::prefetch_tmap(&ymap);
@@ -392,7 +412,7 @@ __global__ void __launch_bounds__(kTcThreads, 3)
         int ys = 0;
         uint32_t yph = 0, sph = 0;
         for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
-          const int x0 = (int)(tile * 128);
+          const int x0 = (int)(tile * C::PIX);
           // history twice (pass 1, pass 2: re-read from L2), then the seed
           // chunks [s0, nch) once the consumers have found s0, then monitoring
           int s0 = nch;
@@ -483,7 +503,7 @@ __global__ void __launch_bounds__(kTcThreads, 3)
           return ob;
         };
         // yhat of the chunk `ahead` chunks after the current one (its table
-        // stage starts with the [16 x KY] yhat table)
+        // stage starts with the [16 x KY] yhat table), for every pixel group
         auto issue_yhat = [&](int ahead) {
           uint32_t par;
           const int s = tslot(ahead, par);
@@ -493,9 +513,11 @@ __global__ void __launch_bounds__(kTcThreads, 3)
           sm100::tc_fence_after();
           const uint32_t b3 = tss + s * C::TSTAGE;
 #pragma unroll
-          for (int q = 0; q < C::KY / 16; ++q)
-            sm100::umma_bf16_ts(tbase + C::COL_Y + slot * C::DC, tbase + C::COL_A3 + 8 * q,
-                                sm100::smem_desc(b3 + q * 2 * 256, 256, 128), idY, q > 0);
+          for (int q = 0; q < PX; ++q)
+#pragma unroll
+            for (int j = 0; j < C::KY / 16; ++j)
+              sm100::umma_bf16_ts(tbase + C::col_y(slot, q), tbase + C::col_a3(q) + 8 * j,
+                                  sm100::smem_desc(b3 + j * 2 * 256, 256, 128), idY, j > 0);
           sm100::umma_commit(&yhfull[slot]);
           ++yissue;
         };
@@ -505,21 +527,24 @@ __global__ void __launch_bounds__(kTcThreads, 3)
             const uint32_t ob = opwait();
             mbar_wait_mma(&tfull[ts], tph);
             sm100::tc_fence_after();
-            const uint32_t am = aop + ob * C::OPBUF;  // mask, y' hi, y' lo tiles
             const uint32_t bf = tss + ts * C::TSTAGE, bx = bf + 3 * C::BF_BYTES;
-            const uint32_t dG = tbase + (c & 1) * C::SET, dB = dG + C::NGn;
             const uint32_t first = c >= 2 ? 1u : 0u;
 #pragma unroll
-            for (int e = 0; e < 3; ++e)
-              sm100::umma_bf16(dG, sm100::smem_desc(am, 2048, 128),
-                               sm100::smem_desc(bf + e * C::BF_BYTES, C::NGn * 16, 128), idG, first | (e > 0));
-            // y'hi x_hi, y'hi x_mid, y'lo x_hi
-            sm100::umma_bf16(dB, sm100::smem_desc(am + C::ATILE, 2048, 128), sm100::smem_desc(bx, C::KBn * 16, 128),
-                             idB, first);
-            sm100::umma_bf16(dB, sm100::smem_desc(am + C::ATILE, 2048, 128),
-                             sm100::smem_desc(bx + C::BX_BYTES, C::KBn * 16, 128), idB, 1);
-            sm100::umma_bf16(dB, sm100::smem_desc(am + 2 * C::ATILE, 2048, 128),
-                             sm100::smem_desc(bx, C::KBn * 16, 128), idB, 1);
+            for (int q = 0; q < PX; ++q) {
+              const uint32_t am = aop + ob * C::OPBUF + q * 3 * C::ATILE;  // mask, y' hi, y' lo tiles
+              const uint32_t dG = tbase + C::col_set(c & 1, q), dB = dG + C::NGn;
+#pragma unroll
+              for (int e = 0; e < 3; ++e)
+                sm100::umma_bf16(dG, sm100::smem_desc(am, 2048, 128),
+                                 sm100::smem_desc(bf + e * C::BF_BYTES, C::NGn * 16, 128), idG, first | (e > 0));
+              // y'hi x_hi, y'hi x_mid, y'lo x_hi
+              sm100::umma_bf16(dB, sm100::smem_desc(am + C::ATILE, 2048, 128),
+                               sm100::smem_desc(bx, C::KBn * 16, 128), idB, first);
+              sm100::umma_bf16(dB, sm100::smem_desc(am + C::ATILE, 2048, 128),
+                               sm100::smem_desc(bx + C::BX_BYTES, C::KBn * 16, 128), idB, 1);
+              sm100::umma_bf16(dB, sm100::smem_desc(am + 2 * C::ATILE, 2048, 128),
+                               sm100::smem_desc(bx, C::KBn * 16, 128), idB, 1);
+            }
             sm100::umma_commit(&opfree[ob]);
             sm100::umma_commit(&tempty[ts]);
             if (c == nch - 1) sm100::umma_commit(&accready);
@@ -534,17 +559,20 @@ __global__ void __launch_bounds__(kTcThreads, 3)
             const uint32_t ob = opwait();
             mbar_wait_mma(&tfull[ts], tph);
             sm100::tc_fence_after();
-            const uint32_t am = aop + ob * C::OPBUF;  // r0 hi, r0 lo tiles
             const uint32_t bx = tss + ts * C::TSTAGE + C::B3_BYTES;
-            const uint32_t dD = tbase + C::COL_DB;
-            // r0hi (x_hi + x_mid + x_lo) + r0lo (x_hi + x_mid) [+ r0lo2 x_hi]
 #pragma unroll
-            for (int e = 0; e < kR0Parts; ++e)
+            for (int q = 0; q < PX; ++q) {
+              const uint32_t am = aop + ob * C::OPBUF + q * 3 * C::ATILE;  // r0 parts
+              const uint32_t dD = tbase + C::col_db(q);
+              // r0hi (x_hi + x_mid + x_lo) + r0mid (x_hi + x_mid) + r0lo x_hi
 #pragma unroll
-              for (int q = 0; q < 3 - e; ++q)
-                sm100::umma_bf16(dD, sm100::smem_desc(am + e * C::ATILE, 2048, 128),
-                                 sm100::smem_desc(bx + q * C::BX_BYTES, C::KBn * 16, 128), idB,
-                                 (c > 0 || e > 0 || q > 0) ? 1u : 0u);
+              for (int e = 0; e < kR0Parts; ++e)
+#pragma unroll
+                for (int x = 0; x < 3 - e; ++x)
+                  sm100::umma_bf16(dD, sm100::smem_desc(am + e * C::ATILE, 2048, 128),
+                                   sm100::smem_desc(bx + x * C::BX_BYTES, C::KBn * 16, 128), idB,
+                                   (c > 0 || e > 0 || x > 0) ? 1u : 0u);
+            }
             sm100::umma_commit(&opfree[ob]);
             if (c + 2 < nch) issue_yhat(2);
             sm100::umma_commit(&tempty[ts]);
@@ -569,11 +597,15 @@ __global__ void __launch_bounds__(kTcThreads, 3)
     }  // warp 7 idles: it completes the producer warpgroup
   } else {
     // ------------------------------------------------------------ consumers
+    // Thread t owns pixels PX*t .. PX*t + PX-1 of the tile (adjacent: one
+    // 8-byte shared load per date reads both); pixel group q = t's q-th
+    // pixel, i.e. TMEM lane t of the column groups of q and row t of the A
+    // tiles of q.
     sm100::setmaxnreg_inc<kTcConsumerRegs>();
     const uint32_t lanebase = tbase + ((uint32_t)(32 * warp) << 16);
     const float qnan = __int_as_float(0x7fc00000);
-    // ring: slot s = 128 residuals f32, this thread's at rbase + s*RSLOT
-    const uint32_t rbase = sm100::smem_u32(ring) + 4 * tid;
+    // ring: slot s = PIX residuals f32, pixel q of this thread at rbase + 4q + s*RSLOT
+    const uint32_t rbase = sm100::smem_u32(ring) + 4 * PX * tid;
     int ys = 0;
     uint32_t yph = 0, opcnt = 0, yuse = 0, acnt = 0;
     // 32-bit shared addresses of the barriers this warp waits on / arrives at
@@ -605,32 +637,35 @@ __global__ void __launch_bounds__(kTcThreads, 3)
       warp_arrive(a_opfull + 8 * ob);
       ++opcnt;
     };
-    auto write_beta_operand = [&](const float (&bt)[K]) {
-      // A3 row (TMEM) = [bh | bh | bh | bm | bm | bl | 0...] (6 blocks of K, KY bf16)
-      float h[K], m[K], l[K];
+    // A3 rows (TMEM) = [bh | bh | bh | bm | bm | bl | 0...] (6 blocks of K, KY bf16) per pixel group
+    auto write_beta_operand = [&](const float (&bt)[PX][K]) {
 #pragma unroll
-      for (int i = 0; i < K; ++i) {
-        h[i] = bf16_round(bt[i]);
-        m[i] = bf16_round(bt[i] - h[i]);
-        l[i] = bt[i] - h[i] - m[i];
-      }
-      uint32_t w[C::KY / 2];
+      for (int q = 0; q < PX; ++q) {
+        float h[K], m[K], l[K];
 #pragma unroll
-      for (int j = 0; j < C::KY / 2; ++j) {
-        float e[2];
-#pragma unroll
-        for (int u = 0; u < 2; ++u) {
-          const int col = 2 * j + u, blk = col / K, i = col % K;
-          e[u] = col >= 6 * K ? 0.f : (blk < 3 ? h[i] : blk < 5 ? m[i] : l[i]);
+        for (int i = 0; i < K; ++i) {
+          h[i] = bf16_round(bt[q][i]);
+          m[i] = bf16_round(bt[q][i] - h[i]);
+          l[i] = bt[q][i] - h[i] - m[i];
         }
-        w[j] = sm100::pack_bf16x2(e[0], e[1]);
-      }
+        uint32_t w[C::KY / 2];
 #pragma unroll
-      for (int q = 0; q < C::KY / 16; ++q) {
-        uint32_t w8[8];
+        for (int j = 0; j < C::KY / 2; ++j) {
+          float e[2];
 #pragma unroll
-        for (int i = 0; i < 8; ++i) w8[i] = w[8 * q + i];
-        sm100::tmem_st8(lanebase + C::COL_A3 + 8 * q, w8);  // this pixel's row of the A operand
+          for (int u = 0; u < 2; ++u) {
+            const int col = 2 * j + u, blk = col / K, i = col % K;
+            e[u] = col >= 6 * K ? 0.f : (blk < 3 ? h[i] : blk < 5 ? m[i] : l[i]);
+          }
+          w[j] = sm100::pack_bf16x2(e[0], e[1]);
+        }
+#pragma unroll
+        for (int j = 0; j < C::KY / 16; ++j) {
+          uint32_t w8[8];
+#pragma unroll
+          for (int i = 0; i < 8; ++i) w8[i] = w[8 * j + i];
+          sm100::tmem_st8(lanebase + C::col_a3(q) + 8 * j, w8);  // this pixel's row of the A operand
+        }
       }
       sm100::tmem_st_wait();
       sm100::tc_fence_before();
@@ -640,8 +675,9 @@ __global__ void __launch_bounds__(kTcThreads, 3)
       sm100::mbar_wait_a(a_yhfull + 8 * (yuse & 1), (yuse >> 1) & 1);
       sm100::tc_fence_after();
     };
-    auto load_yhat8 = [&](int half, float (&yh)[8]) {
-      sm100::tmem_ld8(lanebase + C::COL_Y + (yuse & 1) * C::DC + 8 * half, yh);
+    auto load_yhat8 = [&](int half, float (&yh)[PX][8]) {
+#pragma unroll
+      for (int q = 0; q < PX; ++q) sm100::tmem_ld8(lanebase + C::col_y(yuse & 1, q) + 8 * half, yh[q]);
       sm100::tmem_ld_wait();
     };
     auto release_yhat = [&]() {
@@ -649,53 +685,84 @@ __global__ void __launch_bounds__(kTcThreads, 3)
       warp_arrive(a_yhfree + 8 * (yuse & 1));
       ++yuse;
     };
+    // the 8 dates of a half chunk for this thread's pixels: yv[q][d]
+    auto load_y8 = [&](const float *Ys, int hf, float (&yv)[PX][8]) {
+#pragma unroll
+      for (int d = 0; d < 8; ++d) {
+        if (PX == 2) {
+          const float2 v = *reinterpret_cast<const float2 *>(Ys + (8 * hf + d) * C::PIX + 2 * tid);
+          yv[0][d] = v.x;
+          yv[PX - 1][d] = v.y;
+        } else {
+          yv[0][d] = Ys[(8 * hf + d) * C::PIX + tid];
+        }
+      }
+    };
 
     for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
-      const int64_t pix = p.p0 + tile * 128 + tid;
+      const int64_t pix0 = p.p0 + tile * C::PIX + PX * tid;
       // the operand buffers reuse the ring's bytes: every consumer warp must
       // be done with the previous tile's monitoring before any writes them
       asm volatile("bar.sync 1, 128;" ::: "memory");
       // ================= pass 1: masked Gram + moment on the tensor cores
-      float c0 = qnan, ymax = 0.f;
-      bool have = false;
+      float c0[PX], ymax[PX];
+      bool have[PX];
+#pragma unroll
+      for (int q = 0; q < PX; ++q) {
+        c0[q] = qnan;
+        ymax[q] = 0.f;
+        have[q] = false;
+      }
       for (int c = 0; c < nch; ++c) {
         sm100::mbar_wait_a(a_yfull + 8 * ys, yph);
         const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
         // offset c = first valid value (warp-uniform pre-scan while a lane lacks it)
-        if (__any_sync(0xffffffffu, !have)) {
-          for (int d = 0; d < C::DC && !have; ++d) {
-            const float y = Ys[d * 128 + tid];
-            if (y == y) {
-              c0 = y;
-              have = true;
+        bool need = false;
+#pragma unroll
+        for (int q = 0; q < PX; ++q) need = need || !have[q];
+        if (__any_sync(0xffffffffu, need)) {
+#pragma unroll
+          for (int q = 0; q < PX; ++q)
+            for (int d = 0; d < C::DC && !have[q]; ++d) {
+              const float y = Ys[d * C::PIX + PX * tid + q];
+              if (y == y) {
+                c0[q] = y;
+                have[q] = true;
+              }
             }
-          }
         }
         uint8_t *ob = nullptr;
 #pragma unroll 1
         for (int hf = 0; hf < 2; ++hf) {  // two halves of 8 dates: half the hot code
-          float yv[8];
+          float yv[PX][8];
+          load_y8(Ys, hf, yv);  // dates >= n read as NaN (hmap)
+          uint32_t vm[PX][8];
+          float ph[PX][8], pl[PX][8];
 #pragma unroll
-          for (int d = 0; d < 8; ++d) yv[d] = Ys[(8 * hf + d) * 128 + tid];  // dates >= n read as NaN (hmap)
-          uint32_t vm[8];
-          float ph[8], pl[8];
+          for (int q = 0; q < PX; ++q)
 #pragma unroll
-          for (int d = 0; d < 8; ++d) {
-            ymax = fmaxf(ymax, fabsf(yv[d]));  // NaN ignored
-            p1_date(yv[d], c0, vm[d], ph[d], pl[d]);
-          }
+            for (int d = 0; d < 8; ++d) {
+              ymax[q] = fmaxf(ymax[q], fabsf(yv[q][d]));  // NaN ignored
+              p1_date(yv[q][d], c0[q], vm[q][d], ph[q][d], pl[q][d]);
+            }
           // the MMA of the previous chunk frees the operand buffer while the
           // first half is computed
           if (hf == 0) ob = opbuf_acquire();
           const uint32_t off = sm100::kmajor_off(tid, 8 * hf, 128);
-          // mask pair words: bf16 1.0 (0x3F80) in each half whose date is valid
-          *reinterpret_cast<uint4 *>(ob + off) =
-              make_uint4((vm[0] & 0x3F80u) | (vm[1] & 0x3F800000u), (vm[2] & 0x3F80u) | (vm[3] & 0x3F800000u),
-                         (vm[4] & 0x3F80u) | (vm[5] & 0x3F800000u), (vm[6] & 0x3F80u) | (vm[7] & 0x3F800000u));
-          *reinterpret_cast<uint4 *>(ob + C::ATILE + off) = make_uint4(
-              pack_hi16(ph[0], ph[1]), pack_hi16(ph[2], ph[3]), pack_hi16(ph[4], ph[5]), pack_hi16(ph[6], ph[7]));
-          *reinterpret_cast<uint4 *>(ob + 2 * C::ATILE + off) = make_uint4(
-              pack_hi16(pl[0], pl[1]), pack_hi16(pl[2], pl[3]), pack_hi16(pl[4], pl[5]), pack_hi16(pl[6], pl[7]));
+#pragma unroll
+          for (int q = 0; q < PX; ++q) {
+            uint8_t *oq = ob + q * 3 * C::ATILE;
+            // mask pair words: bf16 1.0 (0x3F80) in each half whose date is valid
+            *reinterpret_cast<uint4 *>(oq + off) = make_uint4(
+                (vm[q][0] & 0x3F80u) | (vm[q][1] & 0x3F800000u), (vm[q][2] & 0x3F80u) | (vm[q][3] & 0x3F800000u),
+                (vm[q][4] & 0x3F80u) | (vm[q][5] & 0x3F800000u), (vm[q][6] & 0x3F80u) | (vm[q][7] & 0x3F800000u));
+            *reinterpret_cast<uint4 *>(oq + C::ATILE + off) =
+                make_uint4(pack_hi16(ph[q][0], ph[q][1]), pack_hi16(ph[q][2], ph[q][3]),
+                           pack_hi16(ph[q][4], ph[q][5]), pack_hi16(ph[q][6], ph[q][7]));
+            *reinterpret_cast<uint4 *>(oq + 2 * C::ATILE + off) =
+                make_uint4(pack_hi16(pl[q][0], pl[q][1]), pack_hi16(pl[q][2], pl[q][3]),
+                           pack_hi16(pl[q][4], pl[q][5]), pack_hi16(pl[q][6], pl[q][7]));
+          }
         }
         warp_arrive(a_yempty + 8 * ys);  // every loaded value has been consumed
         opbuf_publish();
@@ -706,79 +773,83 @@ __global__ void __launch_bounds__(kTcThreads, 3)
       sm100::tc_fence_after();
 
       // ================= solve (Alg. 1 l.3-4): Gram from the masked moments
-      float A[Tri<K>::kN], b[K];
-      int nbar;
-      {
-        float G[C::NF + 1];  // moments, then the count of valid history dates
-#pragma unroll
-        for (int i = 0; i <= C::NF; ++i) G[i] = 0.f;
-#pragma unroll
-        for (int i = 0; i < K; ++i) b[i] = 0.f;
-#pragma unroll
-        for (int s = 0; s < 2; ++s) {
-          if (s == 1 && nch < 2) break;
-#pragma unroll
-          for (int q = 0; q < C::NGn / 16; ++q) {
-            float v16[16];
-            sm100::tmem_ld16(lanebase + s * C::SET + 16 * q, v16);
-            sm100::tmem_ld_wait();
-#pragma unroll
-            for (int i = 0; i < 16; ++i)
-              if (16 * q + i <= C::NF) G[16 * q + i] += v16[i];
-          }
-          {
-            float v16[16];
-            sm100::tmem_ld16(lanebase + s * C::SET + C::NGn, v16);
-            sm100::tmem_ld_wait();
-#pragma unroll
-            for (int i = 0; i < K; ++i) b[i] += v16[i];
-          }
-        }
-        nbar = (int)G[C::NF];  // exact: a sum of 0/1 products in fp32
-        const float nb = (float)nbar;
-        auto Cf = [&](int m) -> float { return m == 0 ? nb : G[2 + 2 * C::k + 2 * ((m < 0 ? -m : m) - 1) + 1]; };
-        auto Sf = [&](int m) -> float {
-          return m == 0 ? 0.f : (m < 0 ? -G[2 + 2 * C::k + 2 * (-m - 1)] : G[2 + 2 * C::k + 2 * (m - 1)]);
-        };
-        A[Tri<K>::idx(0, 0)] = nb;
-        A[Tri<K>::idx(0, 1)] = G[0];
-        A[Tri<K>::idx(1, 1)] = G[1];
-#pragma unroll
-        for (int j = 1; j <= C::k; ++j) {
-          A[Tri<K>::idx(0, 2 * j)] = Sf(j);
-          A[Tri<K>::idx(0, 2 * j + 1)] = Cf(j);
-          A[Tri<K>::idx(1, 2 * j)] = G[2 + 2 * (j - 1)];
-          A[Tri<K>::idx(1, 2 * j + 1)] = G[3 + 2 * (j - 1)];
-#pragma unroll
-          for (int jb = j; jb <= C::k; ++jb) {
-            A[Tri<K>::idx(2 * j, 2 * jb)] = 0.5f * (Cf(j - jb) - Cf(j + jb));          // s_j s_jb
-            A[Tri<K>::idx(2 * j + 1, 2 * jb + 1)] = 0.5f * (Cf(j - jb) + Cf(j + jb));  // c_j c_jb
-            A[Tri<K>::idx(2 * j, 2 * jb + 1)] = 0.5f * (Sf(j + jb) + Sf(j - jb));      // s_j c_jb
-            if (jb > j) A[Tri<K>::idx(2 * j + 1, 2 * jb)] = 0.5f * (Sf(jb + j) + Sf(jb - j));  // c_j s_jb
-          }
-        }
-      }
-      const int h = window_h(nbar, p.hf);
-      bool deg = (nbar < K + 1) || (h < 1);
-      float beta[K];
-      bool refit = false;
+      float A[PX][Tri<K>::kN], dinv[PX][K], beta[PX][K];
+      int nbar[PX], h[PX];
+      bool deg[PX], refit[PX];
 #ifdef BFAST_REFIT_WHY
-      uint32_t why = 0;  // diagnostics build: which trigger sent the pixel to the refit
-#define BFAST_WHY(b) why |= (b)
-#else
-#define BFAST_WHY(b)
-#endif
-      float dinv[K];
-      {
-        const float minratio = chol_factor_rsq<K>(A, dinv);
-        chol_solve_rsq<K>(A, dinv, b, beta);
-        if (!deg && !(minratio >= (float)kRefitRatio)) {
-          refit = true;
-          BFAST_WHY(0x10);
-        }
-        if (deg) {
+      uint32_t why[PX];  // diagnostics build: which trigger sent the pixel to the refit
 #pragma unroll
-          for (int i = 0; i < K; ++i) beta[i] = 0.f;
+      for (int q = 0; q < PX; ++q) why[q] = 0;
+#define BFAST_WHY(q, b) why[q] |= (b)
+#else
+#define BFAST_WHY(q, b)
+#endif
+#pragma unroll
+      for (int q = 0; q < PX; ++q) {
+        float b[K];
+        {
+          float G[C::NF + 1];  // moments, then the count of valid history dates
+#pragma unroll
+          for (int i = 0; i <= C::NF; ++i) G[i] = 0.f;
+#pragma unroll
+          for (int i = 0; i < K; ++i) b[i] = 0.f;
+#pragma unroll
+          for (int s = 0; s < 2; ++s) {
+            if (s == 1 && nch < 2) break;
+#pragma unroll
+            for (int j = 0; j < C::NGn / 16; ++j) {
+              float v16[16];
+              sm100::tmem_ld16(lanebase + C::col_set(s, q) + 16 * j, v16);
+              sm100::tmem_ld_wait();
+#pragma unroll
+              for (int i = 0; i < 16; ++i)
+                if (16 * j + i <= C::NF) G[16 * j + i] += v16[i];
+            }
+            {
+              float v16[16];
+              sm100::tmem_ld16(lanebase + C::col_set(s, q) + C::NGn, v16);
+              sm100::tmem_ld_wait();
+#pragma unroll
+              for (int i = 0; i < K; ++i) b[i] += v16[i];
+            }
+          }
+          nbar[q] = (int)G[C::NF];  // exact: a sum of 0/1 products in fp32
+          const float nb = (float)nbar[q];
+          auto Cf = [&](int m) -> float { return m == 0 ? nb : G[2 + 2 * C::k + 2 * ((m < 0 ? -m : m) - 1) + 1]; };
+          auto Sf = [&](int m) -> float {
+            return m == 0 ? 0.f : (m < 0 ? -G[2 + 2 * C::k + 2 * (-m - 1)] : G[2 + 2 * C::k + 2 * (m - 1)]);
+          };
+          float(&Aq)[Tri<K>::kN] = A[q];
+          Aq[Tri<K>::idx(0, 0)] = nb;
+          Aq[Tri<K>::idx(0, 1)] = G[0];
+          Aq[Tri<K>::idx(1, 1)] = G[1];
+#pragma unroll
+          for (int j = 1; j <= C::k; ++j) {
+            Aq[Tri<K>::idx(0, 2 * j)] = Sf(j);
+            Aq[Tri<K>::idx(0, 2 * j + 1)] = Cf(j);
+            Aq[Tri<K>::idx(1, 2 * j)] = G[2 + 2 * (j - 1)];
+            Aq[Tri<K>::idx(1, 2 * j + 1)] = G[3 + 2 * (j - 1)];
+#pragma unroll
+            for (int jb = j; jb <= C::k; ++jb) {
+              Aq[Tri<K>::idx(2 * j, 2 * jb)] = 0.5f * (Cf(j - jb) - Cf(j + jb));          // s_j s_jb
+              Aq[Tri<K>::idx(2 * j + 1, 2 * jb + 1)] = 0.5f * (Cf(j - jb) + Cf(j + jb));  // c_j c_jb
+              Aq[Tri<K>::idx(2 * j, 2 * jb + 1)] = 0.5f * (Sf(j + jb) + Sf(j - jb));      // s_j c_jb
+              if (jb > j) Aq[Tri<K>::idx(2 * j + 1, 2 * jb)] = 0.5f * (Sf(jb + j) + Sf(jb - j));  // c_j s_jb
+            }
+          }
+        }
+        h[q] = window_h(nbar[q], p.hf);
+        deg[q] = (nbar[q] < K + 1) || (h[q] < 1);
+        refit[q] = false;
+        const float minratio = chol_factor_rsq<K>(A[q], dinv[q]);
+        chol_solve_rsq<K>(A[q], dinv[q], b, beta[q]);
+        if (!deg[q] && !(minratio >= (float)kRefitRatio)) {
+          refit[q] = true;
+          BFAST_WHY(q, 0x10);
+        }
+        if (deg[q]) {
+#pragma unroll
+          for (int i = 0; i < K; ++i) beta[q][i] = 0.f;
         }
       }
       sm100::tc_fence_before();
@@ -788,58 +859,80 @@ __global__ void __launch_bounds__(kTcThreads, 3)
       // sigma-hat sums, the refinement moment operand; and which chunk holds
       // the oldest residual of the MOSUM seed (rank nbar - h: the window of
       // the first monitoring date reaches back to rank nbar - h + 1)
-      const int hh = deg ? 1 : h;
-      const int ring_from = nbar - hh;
-      float s2 = 0.f;
-      int cr = 0;       // valid history dates before the current chunk
-      int sc = nch;     // first chunk holding a rank >= ring_from (nch: no seed needed)
+      int hh[PX], ring_from[PX], cr[PX], sc[PX];
+      float s2[PX];
+#pragma unroll
+      for (int q = 0; q < PX; ++q) {
+        hh[q] = deg[q] ? 1 : h[q];
+        ring_from[q] = nbar[q] - hh[q];
+        s2[q] = 0.f;
+        cr[q] = 0;     // valid history dates before the current chunk
+        sc[q] = nch;   // first chunk holding a rank >= ring_from (nch: no seed needed)
+      }
       for (int c = 0; c < nch; ++c) {
         sm100::mbar_wait_a(a_yfull + 8 * ys, yph);
         wait_yhat();
         const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
         uint8_t *ob = nullptr;
-        uint32_t vb = 0;  // validity of the chunk's 16 dates
+        uint32_t vb[PX];  // validity of the chunk's 16 dates
+#pragma unroll
+        for (int q = 0; q < PX; ++q) vb[q] = 0;
 #pragma unroll 1
         for (int hf = 0; hf < 2; ++hf) {
-          float yh[8], yv[8];
+          float yh[PX][8], yv[PX][8];
           load_yhat8(hf, yh);
+          load_y8(Ys, hf, yv);  // dates >= n read as NaN (hmap)
+          float rh[PX][8], rm[PX][8], rl[PX][8];
 #pragma unroll
-          for (int d = 0; d < 8; ++d) yv[d] = Ys[(8 * hf + d) * 128 + tid];  // dates >= n read as NaN (hmap)
-          float rh[8], rm[8], rl[8];
-          uint32_t v8 = 0;
-          SFor<0, 8>::run([&](auto dc) {
-            constexpr int d = decltype(dc)::value;
-            if (kR0Parts == 3)
-              p2h_date3<d>(yv[d], c0, yh[d], s2, v8, rh[d], rm[d], rl[d]);
-            else
-              p2h_date<d>(yv[d], c0, yh[d], s2, v8, rh[d], rl[d]);
-          });
-          vb |= v8 << (8 * hf);
+          for (int q = 0; q < PX; ++q) {
+            uint32_t v8 = 0;
+            SFor<0, 8>::run([&](auto dc) {
+              constexpr int d = decltype(dc)::value;
+              if (kR0Parts == 3)
+                p2h_date3<d>(yv[q][d], c0[q], yh[q][d], s2[q], v8, rh[q][d], rm[q][d], rl[q][d]);
+              else
+                p2h_date<d>(yv[q][d], c0[q], yh[q][d], s2[q], v8, rh[q][d], rl[q][d]);
+            });
+            vb[q] |= v8 << (8 * hf);
+          }
           if (hf == 0) ob = opbuf_acquire();
           const uint32_t off = sm100::kmajor_off(tid, 8 * hf, 128);
-          *reinterpret_cast<uint4 *>(ob + off) = make_uint4(
-              pack_hi16(rh[0], rh[1]), pack_hi16(rh[2], rh[3]), pack_hi16(rh[4], rh[5]), pack_hi16(rh[6], rh[7]));
-          if (kR0Parts == 3) {
-            *reinterpret_cast<uint4 *>(ob + C::ATILE + off) = make_uint4(
-                pack_hi16(rm[0], rm[1]), pack_hi16(rm[2], rm[3]), pack_hi16(rm[4], rm[5]), pack_hi16(rm[6], rm[7]));
-            *reinterpret_cast<uint4 *>(ob + 2 * C::ATILE + off) = make_uint4(
-                pack_hi16(rl[0], rl[1]), pack_hi16(rl[2], rl[3]), pack_hi16(rl[4], rl[5]), pack_hi16(rl[6], rl[7]));
-          } else {
-            // r0 = hi (truncated, exact) + lo (rounded to nearest: unbiased)
-            *reinterpret_cast<uint4 *>(ob + C::ATILE + off) =
-                make_uint4(sm100::pack_bf16x2(rl[0], rl[1]), sm100::pack_bf16x2(rl[2], rl[3]),
-                           sm100::pack_bf16x2(rl[4], rl[5]), sm100::pack_bf16x2(rl[6], rl[7]));
+#pragma unroll
+          for (int q = 0; q < PX; ++q) {
+            uint8_t *oq = ob + q * 3 * C::ATILE;
+            *reinterpret_cast<uint4 *>(oq + off) =
+                make_uint4(pack_hi16(rh[q][0], rh[q][1]), pack_hi16(rh[q][2], rh[q][3]),
+                           pack_hi16(rh[q][4], rh[q][5]), pack_hi16(rh[q][6], rh[q][7]));
+            if (kR0Parts == 3) {
+              *reinterpret_cast<uint4 *>(oq + C::ATILE + off) =
+                  make_uint4(pack_hi16(rm[q][0], rm[q][1]), pack_hi16(rm[q][2], rm[q][3]),
+                             pack_hi16(rm[q][4], rm[q][5]), pack_hi16(rm[q][6], rm[q][7]));
+              *reinterpret_cast<uint4 *>(oq + 2 * C::ATILE + off) =
+                  make_uint4(pack_hi16(rl[q][0], rl[q][1]), pack_hi16(rl[q][2], rl[q][3]),
+                             pack_hi16(rl[q][4], rl[q][5]), pack_hi16(rl[q][6], rl[q][7]));
+            } else {
+              // r0 = hi (truncated, exact) + lo (rounded to nearest: unbiased)
+              *reinterpret_cast<uint4 *>(oq + C::ATILE + off) =
+                  make_uint4(sm100::pack_bf16x2(rl[q][0], rl[q][1]), sm100::pack_bf16x2(rl[q][2], rl[q][3]),
+                             sm100::pack_bf16x2(rl[q][4], rl[q][5]), sm100::pack_bf16x2(rl[q][6], rl[q][7]));
+            }
           }
         }
-        cr += __popc(vb);
-        if (sc == nch && !deg && cr > ring_from) sc = c;
+#pragma unroll
+        for (int q = 0; q < PX; ++q) {
+          cr[q] += __popc(vb[q]);
+          if (sc[q] == nch && !deg[q] && cr[q] > ring_from[q]) sc[q] = c;
+        }
         release_yhat();
         warp_arrive(a_yempty + 8 * ys);  // every loaded value has been consumed
         opbuf_publish();
         yadvance();
       }
       // the tile's seed chunks start at the smallest sc: publish this warp's
-      const int sw = __reduce_min_sync(0xffffffffu, sc);
+      int scm = sc[0];
+#pragma unroll
+      for (int q = 1; q < PX; ++q) scm = min(scm, sc[q]);
+      const int sw = __reduce_min_sync(0xffffffffu, scm);
       if (lane == 0) {
         seed_slot[warp] = sw;
         sm100::mbar_arrive_a(sm100::smem_u32(&seedready));
@@ -849,42 +942,43 @@ __global__ void __launch_bounds__(kTcThreads, 3)
       sm100::tc_fence_after();
 
       // ================= refinement: beta = beta0 + A^-1 db; sigma-hat
-      float sigma;
-      {
+      float sigma[PX], scale[PX], inv_scale[PX];
+#pragma unroll
+      for (int q = 0; q < PX; ++q) {
         float db[K], dbf[K];
         {
           float v16[16];
-          sm100::tmem_ld16(lanebase + C::COL_DB, v16);
+          sm100::tmem_ld16(lanebase + C::col_db(q), v16);
           sm100::tmem_ld_wait();
 #pragma unroll
           for (int i = 0; i < K; ++i) db[i] = v16[i];
         }
-        chol_solve_rsq<K>(A, dinv, db, dbf);
+        chol_solve_rsq<K>(A[q], dinv[q], db, dbf);
         float lin = 0.f;
 #pragma unroll
         for (int i = 0; i < K; ++i) {
-          if (deg) dbf[i] = 0.f;
+          if (deg[q]) dbf[i] = 0.f;
           lin = fmaf(dbf[i], db[i], lin);
-          beta[i] += dbf[i];
+          beta[q][i] += dbf[i];
         }
         // sigma^2 (nbar - K) = sum (r0 - x dbeta)^2 = s2 - dbeta . db (A dbeta = db)
-        sigma = sqrtf(fmaxf(s2 - lin, 0.f) / (float)(nbar - K));
+        sigma[q] = sqrtf(fmaxf(s2[q] - lin, 0.f) / (float)(nbar[q] - K));
         // sigma^2 cancels when the refinement step is large next to the
         // residual sum: the fp32 sigma-hat is then unreliable -> fp64 refit
-        if (!(lin <= 1e-2f * s2)) {
-          refit = true;
-          BFAST_WHY(0x20);
+        if (!(lin <= 1e-2f * s2[q])) {
+          refit[q] = true;
+          BFAST_WHY(q, 0x20);
         }
+        if (!deg[q] && !(sigma[q] > 1e-4f * ymax[q])) deg[q] = true;
+        // noise within 2e-3 of the signal scale: fp32 fitted values (~1e-7 |y|)
+        // are no longer negligible next to sigma-hat -> fp64 refit (R12)
+        if (!deg[q] && !(sigma[q] > 2e-3f * ymax[q])) {
+          refit[q] = true;
+          BFAST_WHY(q, 0x40);
+        }
+        scale[q] = sigma[q] * sqrtf((float)nbar[q]);  // MOSUM = W / scale (L524)
+        inv_scale[q] = 1.0f / scale[q];
       }
-      if (!deg && !(sigma > 1e-4f * ymax)) deg = true;
-      // noise within 2e-3 of the signal scale: fp32 fitted values (~1e-7 |y|)
-      // are no longer negligible next to sigma-hat -> fp64 refit (R12)
-      if (!deg && !(sigma > 2e-3f * ymax)) {
-        refit = true;
-        BFAST_WHY(0x40);
-      }
-      const float scale = sigma * sqrtf((float)nbar);  // MOSUM = W / scale (L524)
-      const float inv_scale = 1.0f / scale;
       sm100::tc_fence_before();
       write_beta_operand(beta);
 
@@ -893,8 +987,13 @@ __global__ void __launch_bounds__(kTcThreads, 3)
       // slot about to be written always holds rank cr - h; writing from any
       // rank <= nbar - h on leaves ranks nbar-h .. nbar-1 in the ring with the
       // write slot on rank nbar - h.  A warp starts at its own first chunk sw.
-      const uint32_t hbytes = (uint32_t)hh * C::RSLOT, rend = rbase + hbytes;
-      uint32_t wa = rbase;
+      uint32_t wa[PX], rend[PX], hbytes[PX];
+#pragma unroll
+      for (int q = 0; q < PX; ++q) {
+        wa[q] = rbase + 4 * q;
+        hbytes[q] = (uint32_t)hh[q] * C::RSLOT;
+        rend[q] = wa[q] + hbytes[q];
+      }
       // every consumer warp has published sw and written its last operands
       // (the ring overwrites them); the producers wait on seedready instead
       asm volatile("bar.sync 1, 128;" ::: "memory");
@@ -906,12 +1005,13 @@ __global__ void __launch_bounds__(kTcThreads, 3)
           const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
 #pragma unroll 1
           for (int hf = 0; hf < 2; ++hf) {
-            float yh[8], yv[8];
+            float yh[PX][8], yv[PX][8];
             load_yhat8(hf, yh);
+            load_y8(Ys, hf, yv);
 #pragma unroll
-            for (int d = 0; d < 8; ++d) yv[d] = Ys[(8 * hf + d) * 128 + tid];
+            for (int d = 0; d < 8; ++d)
 #pragma unroll
-            for (int d = 0; d < 8; ++d) seed_date(yv[d], c0, yh[d], wa, rend, hbytes);
+              for (int q = 0; q < PX; ++q) seed_date<C::RSLOT>(yv[q][d], c0[q], yh[q][d], wa[q], rend[q], hbytes[q]);
           }
         }
         release_yhat();
@@ -920,68 +1020,100 @@ __global__ void __launch_bounds__(kTcThreads, 3)
       }
       // W = the window of rank nbar - 1 (ranks nbar-h .. nbar-1); the first
       // monitoring step drops rank nbar - h, so W_0 = m^fst + r_nbar (L518)
-      float W = 0.f;
-      if (!deg)
-        for (uint32_t a = rbase; a < rend; a += C::RSLOT) W += lds_f32(a);
+      float W[PX];
+#pragma unroll
+      for (int q = 0; q < PX; ++q) {
+        W[q] = 0.f;
+        if (!deg[q])
+          for (uint32_t a = rbase + 4 * q; a < rend[q]; a += C::RSLOT) W[q] += lds_f32(a);
+      }
 
       // ================= pass 3, monitoring (Alg. 1 l.6-12, Fig. 12 ker 9-10)
-      float msum = 0.f, mfirst = 0.f;
-      int brk = -1, first = -1;
-      float mx = 0.f;  // max |W| over the valid monitoring dates so far
-      cr = nbar;
-      bool tie = false;
-      // a 1-based rank up to which B == lambda (rank/nbar <= e): floor(e nbar)
-      // - 3 keeps ln(rank/nbar) below 1 by more than f32 rounding for any nbar
-      const int rank_flat = max((int)(2.718281828f * (float)nbar) - 3, 0);
+      float msum[PX], mfirst[PX], mx[PX], thr_lo[PX];
+      int brk[PX], first[PX];
+      bool tie[PX];
+      bool anydeg = false;
+      int rank_flat_min = 0x7fffffff;
       const float lam = p.lambda;
-      // thresholds on W: |m| > lambda (1 - tol)  <=>  |W| > lambda (1 - tol) scale
-      float thr_lo = deg ? __int_as_float(0x7f800000) : lam * (1.0f - kTieTol) * scale;
+#pragma unroll
+      for (int q = 0; q < PX; ++q) {
+        msum[q] = 0.f;
+        mfirst[q] = 0.f;
+        mx[q] = 0.f;  // max |W| over the valid monitoring dates so far
+        brk[q] = -1;
+        first[q] = -1;
+        tie[q] = false;
+        cr[q] = nbar[q];
+        // a 1-based rank up to which B == lambda (rank/nbar <= e): floor(e nbar)
+        // - 3 keeps ln(rank/nbar) below 1 by more than f32 rounding for any nbar
+        const int rank_flat = max((int)(2.718281828f * (float)nbar[q]) - 3, 0);
+        // thresholds on W: |m| > lambda (1 - tol)  <=>  |W| > lambda (1 - tol) scale
+        thr_lo[q] = deg[q] ? __int_as_float(0x7f800000) : lam * (1.0f - kTieTol) * scale[q];
+        if (!deg[q]) rank_flat_min = min(rank_flat_min, rank_flat - nbar[q]);  // monitoring ranks with B == lambda
+        anydeg = anydeg || deg[q];
+      }
+      (void)anydeg;
       for (int c = 0; c < ncm; ++c) {
         sm100::mbar_wait_a(a_yfull + 8 * ys, yph);
         wait_yhat();
         const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
-        // B_j == lambda for every rank this chunk can reach (rank/nbar <= e):
-        // warp-uniform fast path without the out-of-line boundary evaluation
-        const bool fast = __all_sync(0xffffffffu, deg || cr + C::DC <= rank_flat);
+        // B_j == lambda for every rank this chunk can reach (rank/nbar <= e)
+        // for all of the thread's valid pixels: warp-uniform fast path without
+        // the out-of-line boundary evaluation
+        int crm = 0;
+#pragma unroll
+        for (int q = 0; q < PX; ++q) crm = max(crm, deg[q] ? 0 : cr[q] - nbar[q]);
+        const bool fast = __all_sync(0xffffffffu, crm + C::DC <= rank_flat_min);
 #pragma unroll 1
         for (int hf = 0; hf < 2; ++hf) {
-          float yh[8], yv[8];
+          float yh[PX][8], yv[PX][8];
           load_yhat8(hf, yh);
-#pragma unroll
-          for (int d = 0; d < 8; ++d) yv[d] = Ys[(8 * hf + d) * 128 + tid];  // dates >= N read as NaN (TMA OOB)
+          load_y8(Ys, hf, yv);  // dates >= N read as NaN (TMA OOB)
           if (fast) {
             // B_j == lambda here: the first |m| > lambda(1 - tol) decides (a
             // clear crossing is the break, a near tie goes to the fp64 refit).
             // The dates only track max |W|; a half in which it crossed
             // replays its 8 steps from the saved state (same arithmetic).
-            const float W0 = W;
-            float rr[8], oo[8];
+            float W0[PX], rr[PX][8], oo[PX][8];
+#pragma unroll
+            for (int q = 0; q < PX; ++q) W0[q] = W[q];
 #pragma unroll
             for (int d = 0; d < 8; ++d)
-              mon_date(yv[d], c0, yh[d], W, msum, mx, cr, wa, rend, hbytes, rr[d], oo[d]);
-            if (mx > thr_lo) {
-              float Wr = W0;
 #pragma unroll
-              for (int d = 0; d < 8; ++d) {
-                if (rr[d] == rr[d]) {
-                  Wr += rr[d] - oo[d];
-                  if (first < 0 && fabsf(Wr) > thr_lo) {
-                    first = c * C::DC + 8 * hf + d;
-                    mfirst = Wr;
+              for (int q = 0; q < PX; ++q)
+                mon_date<C::RSLOT>(yv[q][d], c0[q], yh[q][d], W[q], msum[q], mx[q], cr[q], wa[q], rend[q],
+                                   hbytes[q], rr[q][d], oo[q][d]);
+
+#pragma unroll
+            for (int q = 0; q < PX; ++q) {
+              if (mx[q] > thr_lo[q]) {
+                float Wr = W0[q];
+#pragma unroll
+                for (int d = 0; d < 8; ++d) {
+                  if (rr[q][d] == rr[q][d]) {
+                    Wr += rr[q][d] - oo[q][d];
+                    if (first[q] < 0 && fabsf(Wr) > thr_lo[q]) {
+                      first[q] = c * C::DC + 8 * hf + d;
+                      mfirst[q] = Wr;
+                    }
                   }
                 }
+                thr_lo[q] = __int_as_float(0x7f800000);
               }
-              thr_lo = __int_as_float(0x7f800000);
             }
           } else {
 #pragma unroll
             for (int d = 0; d < 8; ++d) {
-              float r, old;
-              mon_date(yv[d], c0, yh[d], W, msum, mx, cr, wa, rend, hbytes, r, old);
-              if (r == r && brk < 0 && !tie && first < 0 && fabsf(W) > thr_lo) {
-                const int code = boundary_rare(W * inv_scale, cr, nbar, lam);
-                tie = tie || (code >> 1);
-                brk = (code & 1) ? c * C::DC + 8 * hf + d : brk;
+#pragma unroll
+              for (int q = 0; q < PX; ++q) {
+                float r, old;
+                mon_date<C::RSLOT>(yv[q][d], c0[q], yh[q][d], W[q], msum[q], mx[q], cr[q], wa[q], rend[q], hbytes[q], r,
+                         old);
+                if (r == r && brk[q] < 0 && !tie[q] && first[q] < 0 && fabsf(W[q]) > thr_lo[q]) {
+                  const int code = boundary_rare(W[q] * inv_scale[q], cr[q], nbar[q], lam);
+                  tie[q] = tie[q] || (code >> 1);
+                  brk[q] = (code & 1) ? c * C::DC + 8 * hf + d : brk[q];
+                }
               }
             }
           }
@@ -989,38 +1121,51 @@ __global__ void __launch_bounds__(kTcThreads, 3)
         release_yhat();
         warp_arrive(a_yempty + 8 * ys);  // every loaded value has been consumed
         yadvance();
-        if (first >= 0 && brk < 0 && !tie) {  // resolve a fast-path candidate
-          if (fabsf(mfirst * inv_scale) > lam * (1.0f + kTieTol)) brk = first;
-          else tie = true;
-          thr_lo = __int_as_float(0x7f800000);
+#pragma unroll
+        for (int q = 0; q < PX; ++q) {
+          if (first[q] >= 0 && brk[q] < 0 && !tie[q]) {  // resolve a fast-path candidate
+            if (fabsf(mfirst[q] * inv_scale[q]) > lam * (1.0f + kTieTol)) brk[q] = first[q];
+            else tie[q] = true;
+            thr_lo[q] = __int_as_float(0x7f800000);
+          }
         }
       }
-      const int Nbar = cr;
-      if (Nbar - nbar < 1) deg = true;
 
       // ================= epilogue
-      const bool fit_ok = !((nbar < K + 1) || (h < 1) || (Nbar - nbar < 1));
-      const bool inside = pix < p.p0 + p.P;  // the last tile may be ragged
-      if (inside) {
-        p.out_break[pix] = deg ? -2 : brk;
-        p.out_mag[pix] = deg ? qnan : msum * inv_scale / (float)(Nbar - nbar);
-        if (p.out_sigma) p.out_sigma[pix] = fit_ok ? sigma : qnan;
-        if (p.out_nbar) p.out_nbar[pix] = nbar;
+      unsigned wantbits = 0;
+#pragma unroll
+      for (int q = 0; q < PX; ++q) {
+        const int64_t pix = pix0 + q;
+        const int Nbar = cr[q];
+        if (Nbar - nbar[q] < 1) deg[q] = true;
+        const bool fit_ok = !((nbar[q] < K + 1) || (h[q] < 1) || (Nbar - nbar[q] < 1));
+        const bool inside = pix < p.p0 + p.P;  // the last tile may be ragged
+        if (inside) {
+          p.out_break[pix] = deg[q] ? -2 : brk[q];
+          p.out_mag[pix] = deg[q] ? qnan : msum[q] * inv_scale[q] / (float)(Nbar - nbar[q]);
+          if (p.out_sigma) p.out_sigma[pix] = fit_ok ? sigma[q] : qnan;
+          if (p.out_nbar) p.out_nbar[pix] = nbar[q];
 #ifdef BFAST_REFIT_WHY
-        if (p.out_flags) p.out_flags[pix] = (deg ? 1u : 0u) | why | (tie ? 0x80u : 0u);
+          if (p.out_flags) p.out_flags[pix] = (deg[q] ? 1u : 0u) | why[q] | (tie[q] ? 0x80u : 0u);
 #else
-        if (p.out_flags) p.out_flags[pix] = deg ? 1u : 0u;
+          if (p.out_flags) p.out_flags[pix] = deg[q] ? 1u : 0u;
 #endif
-        store_beta<K, float>(p, pix, beta, c0, fit_ok);
+          store_beta<K, float>(p, pix, beta[q], c0[q], fit_ok);
+        }
+        if ((refit[q] || tie[q]) && fit_ok && inside) wantbits |= 1u << q;
       }
-      const bool want = (refit || tie) && fit_ok && inside;
-      const unsigned mask = __ballot_sync(0xffffffffu, want);
-      if (want) {
-        const int leader = __ffs(mask) - 1;
-        int base = 0;
-        if (lane == leader) base = atomicAdd(p.refit_count, __popc(mask));
-        base = __shfl_sync(mask, base, leader);
-        p.refit_list[base + __popc(mask & ((1u << lane) - 1))] = (int32_t)pix;
+      // append the pixels for the fp64 refit (warp-aggregated)
+#pragma unroll
+      for (int q = 0; q < PX; ++q) {
+        const bool want = (wantbits >> q) & 1u;
+        const unsigned mask = __ballot_sync(0xffffffffu, want);
+        if (want) {
+          const int leader = __ffs(mask) - 1;
+          int base = 0;
+          if (lane == leader) base = atomicAdd(p.refit_count, __popc(mask));
+          base = __shfl_sync(mask, base, leader);
+          p.refit_list[base + __popc(mask & ((1u << lane) - 1))] = (int32_t)(pix0 + q);
+        }
       }
     }
   }
