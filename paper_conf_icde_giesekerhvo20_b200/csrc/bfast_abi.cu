@@ -340,15 +340,15 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
   // shared-memory layout and CTAs per SM.  Co-resident CTAs hide each
   // other's latencies (1 -> 2 -> 3 CTAs/SM measured 1.5x, then 1.08x), so
   // take the layout that admits the most CTAs, preferring among equals the
-  // earlier entry: two stack stages already cover the HBM latency of this
-  // compute-bound kernel (2 and 4 stages time alike), double operand buffers
+  // earlier entry: a third stack stage is worth 1.5% on the Landsat scene
+  // (it absorbs the HBM latency of the history's first read), double operand buffers
   // let the consumers fill chunk c+1 while the MMA still reads chunk c.
   // Limits: registers (80 x 256 threads at launch -> 3 CTAs), shared memory
   // (228 KB per SM, 1 KB reserved + 1 KB static per CTA), TMEM (512 columns).
   // (The occupancy API is not used: it does not model setmaxnreg kernels.)
   int tc_sy = 2, tc_nop = 1, per_sm = 0;
   {
-    const int cand[4][2] = {{2, 2}, {2, 1}, {3, 2}, {3, 1}};
+    const int cand[4][2] = {{3, 2}, {2, 2}, {3, 1}, {2, 1}};
     const int reg_cap = std::min(65536 / (bfast::kTcThreads * bfast::kTcLaunchRegs), bfast::kTcCtasPerSm);
     const int tmem_cap = 512 / TC::TMEM_COLS;
     for (auto &c : cand) {

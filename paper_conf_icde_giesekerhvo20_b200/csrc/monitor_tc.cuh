@@ -82,6 +82,24 @@ constexpr int kTcConsumerRegs = 2 * kTcLaunchRegs - kTcAuxRegs;
 #define BFAST_R0_PARTS 3
 #endif
 constexpr int kR0Parts = BFAST_R0_PARTS;
+// release a chunk's stack stage and yhat slot as soon as the second half's
+// values are in registers (1), or after the chunk's arithmetic (0)
+#ifndef BFAST_EARLY_REL
+#define BFAST_EARLY_REL 1
+#endif
+constexpr bool kEarlyRelease = BFAST_EARLY_REL != 0;
+// TMEM slots for yhat = X beta of upcoming chunks (the MMA warp runs this
+// many chunks ahead of the consumers in passes 2 and 3)
+#ifndef BFAST_YS
+#define BFAST_YS 2
+#endif
+constexpr int kYhatSlots = BFAST_YS;
+// one producer thread issues both the stack boxes and the chunk tables (1)
+// or one thread each (0)
+#ifndef BFAST_MERGE_PROD
+#define BFAST_MERGE_PROD 1
+#endif
+constexpr bool kMergeProducers = BFAST_MERGE_PROD != 0;
 
 template <int K, int PX = kTcPx>
 struct TcCfg {
@@ -101,10 +119,11 @@ struct TcCfg {
   static constexpr int A3W = ((KY / 2 + 15) / 16) * 16;
   static constexpr int COLS_P1 = 2 * PX * SET;
   static constexpr __host__ __device__ int col_set(int s, int q) { return (s * PX + q) * SET; }
+  static constexpr int NYS = kYhatSlots;
   static constexpr __host__ __device__ int col_y(int slot, int q) { return (slot * PX + q) * DC; }
-  static constexpr __host__ __device__ int col_a3(int q) { return 2 * PX * DC + q * A3W; }
-  static constexpr __host__ __device__ int col_db(int q) { return 2 * PX * DC + PX * A3W + q * KBn; }
-  static constexpr int COLS_P2 = 2 * PX * DC + PX * A3W + PX * KBn;
+  static constexpr __host__ __device__ int col_a3(int q) { return NYS * PX * DC + q * A3W; }
+  static constexpr __host__ __device__ int col_db(int q) { return NYS * PX * DC + PX * A3W + q * KBn; }
+  static constexpr int COLS_P2 = NYS * PX * DC + PX * A3W + PX * KBn;
   static constexpr int COLS_USED = COLS_P1 > COLS_P2 ? COLS_P1 : COLS_P2;
   static constexpr int TMEM_COLS = COLS_USED <= 32 ? 32 : COLS_USED <= 64 ? 64 : COLS_USED <= 128 ? 128
                                    : COLS_USED <= 256 ? 256 : 512;
@@ -118,7 +137,7 @@ struct TcCfg {
   static constexpr int YBYTES = DC * PIX * 4;              // one [16 dates x PIX px] box
   static constexpr int TSTAGE = ((TABMAX + 127) / 128) * 128;
   static constexpr int SY_MAX = 4;                         // stack ring stages (released on read)
-  static constexpr int ST = 3;                             // table ring stages (released by MMA commit)
+  static constexpr int ST = NYS + 1 > 3 ? NYS + 1 : 3;     // table ring stages (released by MMA commit)
   static constexpr int ATILE = 128 * DC * 2;               // one [128 x 16] bf16 A tile (one pixel group)
   static constexpr int OPBUF = 3 * PX * ATILE;             // pass 1: mask, y'hi, y'lo; pass 2: r0 parts
   static constexpr int RSLOT = PIX * 4;                    // ring slot: one residual per pixel
@@ -358,7 +377,7 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
   using C = TcCfg<K, PX>;
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ __align__(8) uint64_t yfull[C::SY_MAX], yempty[C::SY_MAX], tfull[C::ST], tempty[C::ST], opfull[2],
-      opfree[2], yhfull[2], yhfree[2], accready, betaready, seedready;
+      opfree[2], yhfull[C::NYS], yhfree[C::NYS], accready, betaready, seedready;
   __shared__ uint32_t tmem_base_s;
   __shared__ int seed_slot[4];  // per consumer warp: first history chunk its MOSUM seed needs
   const int SY = tb.sy, NOP = tb.nop;
@@ -381,6 +400,8 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
     for (int i = 0; i < 2; ++i) {
       sm100::mbar_init(&opfull[i], NCW);
       sm100::mbar_init(&opfree[i], 1);
+    }
+    for (int i = 0; i < C::NYS; ++i) {
       sm100::mbar_init(&yhfull[i], 1);
       sm100::mbar_init(&yhfree[i], NCW);
     }
@@ -409,8 +430,8 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
         sm100::prefetch_tmap(&ymap);
         sm100::prefetch_tmap(&hmap);
         const uint64_t pol_first = sm100::policy_evict_first();
-        int ys = 0;
-        uint32_t yph = 0, sph = 0;
+        int ys = 0, ts = 0;
+        uint32_t yph = 0, tph = 0, sph = 0;
         for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
           const int x0 = (int)(tile * C::PIX);
           // history twice (pass 1, pass 2: re-read from L2), then the seed
@@ -436,11 +457,25 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
                 ys = 0;
                 yph ^= 1;
               }
+              if (kMergeProducers) {
+                // the chunk's B-operand tables (same chunk sequence as the stack)
+                const uint32_t tabbytes = phase == 0 ? C::TAB1 : phase == 1 ? C::TAB2 : C::TABY;
+                const uint32_t stride = phase == 0 ? C::TAB1 : phase < 3 ? C::TAB2 : C::TABY;
+                const uint8_t *tabsrc = phase == 0 ? tb.tab1 : phase < 3 ? tb.tab2 : tb.taby;
+                mbar_wait_sleep(&tempty[ts], tph ^ 1);
+                uint8_t *tst = tstages + ts * C::TSTAGE;
+                sm100::mbar_arrive_expect_tx(&tfull[ts], tabbytes);
+                sm100::bulk_g2s(tst, tabsrc + (size_t)c * stride, tabbytes, &tfull[ts]);
+                if (++ts == C::ST) {
+                  ts = 0;
+                  tph ^= 1;
+                }
+              }
             }
           }
         }
       }
-    } else if (warp == 5) {
+    } else if (warp == 5 && !kMergeProducers) {
       // ------------------------------------------------------------ table producer
       if (lane == 0) {
         int ts = 0;
@@ -507,8 +542,8 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
         auto issue_yhat = [&](int ahead) {
           uint32_t par;
           const int s = tslot(ahead, par);
-          const uint32_t slot = yissue & 1;
-          mbar_wait_mma(&yhfree[slot], ((yissue >> 1) & 1) ^ 1);  // consumers done with the slot
+          const uint32_t slot = yissue % C::NYS;
+          mbar_wait_mma(&yhfree[slot], ((yissue / C::NYS) & 1) ^ 1);  // consumers done with the slot
           mbar_wait_mma(&tfull[s], par);
           sm100::tc_fence_after();
           const uint32_t b3 = tss + s * C::TSTAGE;
@@ -554,7 +589,7 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
           // pass 2, history: yhat0 two chunks ahead, refinement moment per chunk
           mbar_wait_mma(&betaready, bcnt & 1);
           ++bcnt;
-          for (int a = 0; a < 2 && a < nch; ++a) issue_yhat(a);
+          for (int a = 0; a < C::NYS && a < nch; ++a) issue_yhat(a);
           for (int c = 0; c < nch; ++c) {
             const uint32_t ob = opwait();
             mbar_wait_mma(&tfull[ts], tph);
@@ -574,7 +609,7 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
                                    (c > 0 || e > 0 || x > 0) ? 1u : 0u);
             }
             sm100::umma_commit(&opfree[ob]);
-            if (c + 2 < nch) issue_yhat(2);
+            if (c + C::NYS < nch) issue_yhat(C::NYS);
             sm100::umma_commit(&tempty[ts]);
             if (c == nch - 1) sm100::umma_commit(&accready);
             ++opcnt;
@@ -586,9 +621,9 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
           ++bcnt;
           const int s0 = min(min(seed_slot[0], seed_slot[1]), min(seed_slot[2], seed_slot[3]));
           const int n3 = nch - s0 + ncm;
-          for (int a = 0; a < 2 && a < n3; ++a) issue_yhat(a);
+          for (int a = 0; a < C::NYS && a < n3; ++a) issue_yhat(a);
           for (int c = 0; c < n3; ++c) {
-            if (c + 2 < n3) issue_yhat(2);
+            if (c + C::NYS < n3) issue_yhat(C::NYS);
             sm100::umma_commit(&tempty[ts]);  // chunk c's table was read by its yhat MMA
             tadvance();
           }
@@ -672,17 +707,17 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
       warp_arrive(a_betaready);
     };
     auto wait_yhat = [&]() {
-      sm100::mbar_wait_a(a_yhfull + 8 * (yuse & 1), (yuse >> 1) & 1);
+      sm100::mbar_wait_a(a_yhfull + 8 * (yuse % C::NYS), (yuse / C::NYS) & 1);
       sm100::tc_fence_after();
     };
     auto load_yhat8 = [&](int half, float (&yh)[PX][8]) {
 #pragma unroll
-      for (int q = 0; q < PX; ++q) sm100::tmem_ld8(lanebase + C::col_y(yuse & 1, q) + 8 * half, yh[q]);
+      for (int q = 0; q < PX; ++q) sm100::tmem_ld8(lanebase + C::col_y(yuse % C::NYS, q) + 8 * half, yh[q]);
       sm100::tmem_ld_wait();
     };
     auto release_yhat = [&]() {
       sm100::tc_fence_before();
-      warp_arrive(a_yhfree + 8 * (yuse & 1));
+      warp_arrive(a_yhfree + 8 * (yuse % C::NYS));
       ++yuse;
     };
     // the 8 dates of a half chunk for this thread's pixels: yv[q][d]
@@ -736,6 +771,10 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
         for (int hf = 0; hf < 2; ++hf) {  // two halves of 8 dates: half the hot code
           float yv[PX][8];
           load_y8(Ys, hf, yv);  // dates >= n read as NaN (hmap)
+          if (kEarlyRelease && hf == 1) {  // the chunk's stack values are all in registers
+            warp_arrive(a_yempty + 8 * ys);
+            yadvance();
+          }
           uint32_t vm[PX][8];
           float ph[PX][8], pl[PX][8];
 #pragma unroll
@@ -764,9 +803,11 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
                            pack_hi16(pl[q][4], pl[q][5]), pack_hi16(pl[q][6], pl[q][7]));
           }
         }
-        warp_arrive(a_yempty + 8 * ys);  // every loaded value has been consumed
+        if (!kEarlyRelease) {
+          warp_arrive(a_yempty + 8 * ys);  // every loaded value has been consumed
+          yadvance();
+        }
         opbuf_publish();
-        yadvance();
       }
       sm100::mbar_wait_a(a_accready, acnt & 1);
       ++acnt;
@@ -882,6 +923,11 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
           float yh[PX][8], yv[PX][8];
           load_yhat8(hf, yh);
           load_y8(Ys, hf, yv);  // dates >= n read as NaN (hmap)
+          if (kEarlyRelease && hf == 1) {  // yhat slot and stack stage fully read
+            release_yhat();
+            warp_arrive(a_yempty + 8 * ys);
+            yadvance();
+          }
           float rh[PX][8], rm[PX][8], rl[PX][8];
 #pragma unroll
           for (int q = 0; q < PX; ++q) {
@@ -923,10 +969,12 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
           cr[q] += __popc(vb[q]);
           if (sc[q] == nch && !deg[q] && cr[q] > ring_from[q]) sc[q] = c;
         }
-        release_yhat();
-        warp_arrive(a_yempty + 8 * ys);  // every loaded value has been consumed
+        if (!kEarlyRelease) {
+          release_yhat();
+          warp_arrive(a_yempty + 8 * ys);  // every loaded value has been consumed
+          yadvance();
+        }
         opbuf_publish();
-        yadvance();
       }
       // the tile's seed chunks start at the smallest sc: publish this warp's
       int scm = sc[0];
@@ -1069,6 +1117,11 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
           float yh[PX][8], yv[PX][8];
           load_yhat8(hf, yh);
           load_y8(Ys, hf, yv);  // dates >= N read as NaN (TMA OOB)
+          if (kEarlyRelease && hf == 1) {
+            release_yhat();
+            warp_arrive(a_yempty + 8 * ys);
+            yadvance();
+          }
           if (fast) {
             // B_j == lambda here: the first |m| > lambda(1 - tol) decides (a
             // clear crossing is the break, a near tie goes to the fp64 refit).
@@ -1118,9 +1171,11 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
             }
           }
         }
-        release_yhat();
-        warp_arrive(a_yempty + 8 * ys);  // every loaded value has been consumed
-        yadvance();
+        if (!kEarlyRelease) {
+          release_yhat();
+          warp_arrive(a_yempty + 8 * ys);  // every loaded value has been consumed
+          yadvance();
+        }
 #pragma unroll
         for (int q = 0; q < PX; ++q) {
           if (first[q] >= 0 && brk[q] < 0 && !tie[q]) {  // resolve a fast-path candidate

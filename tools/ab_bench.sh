@@ -12,6 +12,8 @@ for i in $(seq 1 $R); do
     BFAST_TC_LAYOUT=$LAY BFAST_LIB=$L timeout 600 python bench.py --no-e2e --no-cpu-baseline $BENCH_ARGS > gpurun_out/ab.json 2> gpurun_out/ab.err
     python -c "
 import json,sys; d=json.load(open('gpurun_out/ab.json'))
-print('$(basename $L):$LAY', round(d['value']/1e6,1), round(d['roofline']['kernel_ms_avg'],3), d['clocks']['sm_mhz'])" || tail -3 gpurun_out/ab.err
+ps=d.get('parity_sample') or {}
+print('$(basename $L):$LAY', round(d['value']/1e6,1), round(d['roofline']['kernel_ms_avg'],3), d['clocks']['sm_mhz'],
+      'parity', ps.get('ok'), ps.get('break_mismatch'), ps.get('mag_max_scaled_err'))" || tail -3 gpurun_out/ab.err
   done
 done
