@@ -100,6 +100,12 @@ constexpr int kYhatSlots = BFAST_YS;
 #define BFAST_MERGE_PROD 1
 #endif
 constexpr bool kMergeProducers = BFAST_MERGE_PROD != 0;
+// k-indexed ring slots in the seed pass too (the monitoring fast path always
+// uses them when every pixel of the warp has h >= 8)
+#ifndef BFAST_SEEDK
+#define BFAST_SEEDK 1
+#endif
+constexpr bool kSeedK = BFAST_SEEDK != 0;
 
 template <int K, int PX = kTcPx>
 struct TcCfg {
@@ -241,6 +247,24 @@ __device__ __forceinline__ void seed_date(float y, float c0, float yh, uint32_t 
       : "f"(y), "f"(c0), "f"(yh), "r"(rend), "r"(hbytes), "n"(RSLOT)
       : "memory");
 }
+// seed_date with the k-indexed slot address of mon_date_k (below)
+template <int RSLOT>
+__device__ __forceinline__ void seed_date_k(float y, float c0, float yh, uint32_t &k, uint32_t wa, uint32_t jw,
+                                            uint32_t hbytes) {
+  asm volatile(
+      "{\n\t.reg .pred p, q;\n\t.reg .f32 r;\n\t.reg .u32 a;\n\t"
+      "sub.f32 r, %1, %2;\n\t"
+      "sub.f32 r, r, %3;\n\t"
+      "setp.num.f32 p, r, r;\n\t"
+      "mad.lo.u32 a, %0, %7, %4;\n\t"
+      "setp.ge.u32 q, %0, %5;\n\t"
+      "@q sub.u32 a, a, %6;\n\t"
+      "@p st.shared.f32 [a], r;\n\t"
+      "@p add.u32 %0, %0, 1;\n\t}"
+      : "+r"(k)
+      : "f"(y), "f"(c0), "f"(yh), "r"(wa), "r"(jw), "r"(hbytes), "n"(RSLOT)
+      : "memory");
+}
 // Cholesky factorisation (Alg. 1 l.3, an SPD Gram) in fp32 with hardware
 // reciprocal square roots: on return A holds L^T off the diagonal and dinv
 // the reciprocal pivots 1/l_jj.  Returns the smallest pivot ratio d_j / A_jj
@@ -320,6 +344,35 @@ __device__ __forceinline__ void mon_date(float y, float c0, float yh, float &W, 
       "@p max.f32 %2, %2, t;\n\t}"
       : "+f"(W), "+f"(msum), "+f"(mx), "+r"(cr), "+r"(wa), "=f"(r), "=f"(old)
       : "f"(y), "f"(c0), "f"(yh), "r"(rend), "r"(hbytes), "n"(RSLOT)
+      : "memory");
+}
+// mon_date with the slot addressed from the half's running count k instead
+// of a pointer advanced date by date: a = wa + k*RSLOT, wrapped once when k
+// reaches jw (slots left before the ring's end).  Only k += 1 is carried
+// from date to date; every date's address is a fresh value, so a store does
+// not hold up the next date's pointer arithmetic (write-after-read on the
+// address register).  Needs h >= 8 (at most one wrap per 8-date half).
+template <int RSLOT>
+__device__ __forceinline__ void mon_date_k(float y, float c0, float yh, float &W, float &msum, float &mx, uint32_t &k,
+                                           uint32_t wa, uint32_t jw, uint32_t hbytes, float &r, float &old) {
+  asm volatile(
+      "{\n\t.reg .pred p, q;\n\t.reg .f32 t;\n\t.reg .u32 a;\n\t"
+      "sub.f32 %4, %6, %7;\n\t"
+      "sub.f32 %4, %4, %8;\n\t"
+      "setp.num.f32 p, %4, %4;\n\t"
+      "mad.lo.u32 a, %3, %12, %9;\n\t"
+      "setp.ge.u32 q, %3, %10;\n\t"
+      "@q sub.u32 a, a, %11;\n\t"
+      "ld.shared.f32 %5, [a];\n\t"
+      "@p st.shared.f32 [a], %4;\n\t"
+      "@p add.u32 %3, %3, 1;\n\t"
+      "sub.f32 t, %4, %5;\n\t"
+      "@p add.f32 %0, %0, t;\n\t"
+      "@p add.f32 %1, %1, %0;\n\t"
+      "abs.f32 t, %0;\n\t"
+      "@p max.f32 %2, %2, t;\n\t}"
+      : "+f"(W), "+f"(msum), "+f"(mx), "+r"(k), "=f"(r), "=f"(old)
+      : "f"(y), "f"(c0), "f"(yh), "r"(wa), "r"(jw), "r"(hbytes), "n"(RSLOT)
       : "memory");
 }
 // producer-side waits with back-off so a waiting producer does not steal
@@ -904,7 +957,7 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
       float s2[PX];
 #pragma unroll
       for (int q = 0; q < PX; ++q) {
-        hh[q] = deg[q] ? 1 : h[q];
+        hh[q] = deg[q] ? min(8, p.hcap) : h[q];  // a degenerate pixel's ring is never read
         ring_from[q] = nbar[q] - hh[q];
         s2[q] = 0.f;
         cr[q] = 0;     // valid history dates before the current chunk
@@ -1042,6 +1095,17 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
         hbytes[q] = (uint32_t)hh[q] * C::RSLOT;
         rend[q] = wa[q] + hbytes[q];
       }
+      // k-indexed ring slots (mon_date_k) need at most one wrap per 8-date
+      // half: h >= 8 for every pixel of the warp
+      bool r8 = true;
+#pragma unroll
+      for (int q = 0; q < PX; ++q) r8 = r8 && hh[q] >= 8;
+#ifdef BFAST_FORCE_RING8
+      const bool ring8 = true;  // experiments only: wrong for pixels with h < 8
+      (void)r8;
+#else
+      const bool ring8 = __all_sync(0xffffffffu, r8);
+#endif
       // every consumer warp has published sw and written its last operands
       // (the ring overwrites them); the producers wait on seedready instead
       asm volatile("bar.sync 1, 128;" ::: "memory");
@@ -1056,10 +1120,30 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
             float yh[PX][8], yv[PX][8];
             load_yhat8(hf, yh);
             load_y8(Ys, hf, yv);
+            if (kSeedK && ring8) {
+              uint32_t kk[PX], jw[PX];
 #pragma unroll
-            for (int d = 0; d < 8; ++d)
+              for (int q = 0; q < PX; ++q) {
+                kk[q] = 0;
+                jw[q] = (rend[q] - wa[q]) / C::RSLOT;
+              }
 #pragma unroll
-              for (int q = 0; q < PX; ++q) seed_date<C::RSLOT>(yv[q][d], c0[q], yh[q][d], wa[q], rend[q], hbytes[q]);
+              for (int q = 0; q < PX; ++q)
+#pragma unroll
+                for (int d = 0; d < 8; ++d)
+                  seed_date_k<C::RSLOT>(yv[q][d], c0[q], yh[q][d], kk[q], wa[q], jw[q], hbytes[q]);
+#pragma unroll
+              for (int q = 0; q < PX; ++q) {
+                const uint32_t a = wa[q] + kk[q] * C::RSLOT;
+                wa[q] = a >= rend[q] ? a - hbytes[q] : a;
+              }
+            } else {
+#pragma unroll
+              for (int d = 0; d < 8; ++d)
+#pragma unroll
+                for (int q = 0; q < PX; ++q)
+                  seed_date<C::RSLOT>(yv[q][d], c0[q], yh[q][d], wa[q], rend[q], hbytes[q]);
+            }
           }
         }
         release_yhat();
@@ -1130,12 +1214,35 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
             float W0[PX], rr[PX][8], oo[PX][8];
 #pragma unroll
             for (int q = 0; q < PX; ++q) W0[q] = W[q];
+            if (ring8) {
+              // slot addresses from the half's running count (mon_date_k);
+              // pixel-major order: each pixel's 8 loads issue back to back
+              uint32_t kk[PX], jw[PX];
 #pragma unroll
-            for (int d = 0; d < 8; ++d)
+              for (int q = 0; q < PX; ++q) {
+                kk[q] = 0;
+                jw[q] = (rend[q] - wa[q]) / C::RSLOT;
+              }
 #pragma unroll
               for (int q = 0; q < PX; ++q)
-                mon_date<C::RSLOT>(yv[q][d], c0[q], yh[q][d], W[q], msum[q], mx[q], cr[q], wa[q], rend[q],
-                                   hbytes[q], rr[q][d], oo[q][d]);
+#pragma unroll
+                for (int d = 0; d < 8; ++d)
+                  mon_date_k<C::RSLOT>(yv[q][d], c0[q], yh[q][d], W[q], msum[q], mx[q], kk[q], wa[q], jw[q],
+                                       hbytes[q], rr[q][d], oo[q][d]);
+#pragma unroll
+              for (int q = 0; q < PX; ++q) {
+                cr[q] += (int)kk[q];
+                const uint32_t a = wa[q] + kk[q] * C::RSLOT;
+                wa[q] = a >= rend[q] ? a - hbytes[q] : a;
+              }
+            } else {
+#pragma unroll
+              for (int d = 0; d < 8; ++d)
+#pragma unroll
+                for (int q = 0; q < PX; ++q)
+                  mon_date<C::RSLOT>(yv[q][d], c0[q], yh[q][d], W[q], msum[q], mx[q], cr[q], wa[q], rend[q],
+                                     hbytes[q], rr[q][d], oo[q][d]);
+            }
 
 #pragma unroll
             for (int q = 0; q < PX; ++q) {
