@@ -94,12 +94,6 @@ constexpr bool kEarlyRelease = BFAST_EARLY_REL != 0;
 #define BFAST_YS 2
 #endif
 constexpr int kYhatSlots = BFAST_YS;
-// one producer thread issues both the stack boxes and the chunk tables (1)
-// or one thread each (0)
-#ifndef BFAST_MERGE_PROD
-#define BFAST_MERGE_PROD 1
-#endif
-constexpr bool kMergeProducers = BFAST_MERGE_PROD != 0;
 // k-indexed ring slots in the seed pass too (the monitoring fast path always
 // uses them when every pixel of the warp has h >= 8)
 #ifndef BFAST_SEEDK
@@ -387,21 +381,21 @@ __device__ __forceinline__ void mon_date_k(float y, float c0, float yh, float &W
 #define BFAST_MMA_WAIT 32
 #endif
 template <int MODE>
-__device__ __forceinline__ void mbar_wait_mode(uint64_t *bar, uint32_t parity) {
+__device__ __forceinline__ void mbar_wait_mode(uint32_t bar, uint32_t parity) {
   if (MODE == 0) {
-    while (!sm100::mbar_try_wait_suspend(bar, parity, 1000000u)) {
+    while (!sm100::mbar_try_wait_a_hint(bar, parity, 1000000u)) {
     }
   } else if (MODE == 1) {
-    while (!sm100::mbar_try_wait(bar, parity)) {
+    while (!sm100::mbar_try_wait_a(bar, parity)) {
     }
   } else {
-    while (!sm100::mbar_try_wait(bar, parity)) __nanosleep(MODE);
+    while (!sm100::mbar_try_wait_a(bar, parity)) __nanosleep(MODE);
   }
 }
-__device__ __forceinline__ void mbar_wait_sleep(uint64_t *bar, uint32_t parity) {
+__device__ __forceinline__ void mbar_wait_sleep(uint32_t bar, uint32_t parity) {
   mbar_wait_mode<BFAST_AUX_WAIT>(bar, parity);
 }
-__device__ __forceinline__ void mbar_wait_mma(uint64_t *bar, uint32_t parity) {
+__device__ __forceinline__ void mbar_wait_mma(uint32_t bar, uint32_t parity) {
   mbar_wait_mode<BFAST_MMA_WAIT>(bar, parity);
 }
 // the rare branch of the boundary test (Alg. 1 l.10-12), kept out of line
@@ -471,11 +465,12 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
   const int n = p.n, nch = tb.nch, ncm = tb.ncm;
 
   if (warp >= NCW) {
-    // producer warpgroup: three single-thread roles need few registers; hand
-    // them to the consumer warpgroup
+    // producer warpgroup: two single-thread roles (warp 4: stack boxes and
+    // chunk tables; warp 6: MMA issue) need few registers; hand them to the
+    // consumer warpgroup
     sm100::setmaxnreg_dec<kTcAuxRegs>();
     if (warp == 4) {
-      // ------------------------------------------------------------ stack producer
+      // ------------------------------------------------------------ producer
       if (lane == 0) {
         // one 2-D TMA box [16 dates x PIX px] per chunk.  History chunks read
         // through `hmap` (dates >= n are out of bounds), monitoring chunks
@@ -483,61 +478,26 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
         sm100::prefetch_tmap(&ymap);
         sm100::prefetch_tmap(&hmap);
         const uint64_t pol_first = sm100::policy_evict_first();
+        // barrier and stage addresses held in registers (sm100::opaque)
+        const uint32_t A_yfull = sm100::opaque(sm100::smem_u32(&yfull[0]));
+        const uint32_t A_yempty = sm100::opaque(sm100::smem_u32(&yempty[0]));
+        const uint32_t A_tfull = sm100::opaque(sm100::smem_u32(&tfull[0]));
+        const uint32_t A_tempty = sm100::opaque(sm100::smem_u32(&tempty[0]));
+        const uint32_t A_seed = sm100::opaque(sm100::smem_u32(&seedready));
+        const uint32_t A_ys = sm100::opaque(sm100::smem_u32(ystages));
+        const uint32_t A_ts = sm100::opaque(sm100::smem_u32(tstages));
         int ys = 0, ts = 0;
         uint32_t yph = 0, tph = 0, sph = 0;
         for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
           const int x0 = (int)(tile * C::PIX);
           // history twice (pass 1, pass 2: re-read from L2), then the seed
-          // chunks [s0, nch) once the consumers have found s0, then monitoring
+          // chunks [s0, nch) once the consumers have found s0, then monitoring;
+          // each chunk's stack box and its B-operand tables (the two rings
+          // advance over the same chunk sequence)
           int s0 = nch;
           for (int phase = 0; phase < 4; ++phase) {
             if (phase == 2) {
-              mbar_wait_sleep(&seedready, sph);
-              sph ^= 1;
-              s0 = min(min(seed_slot[0], seed_slot[1]), min(seed_slot[2], seed_slot[3]));
-            }
-            const int cb = phase == 2 ? s0 : 0, ce = phase < 3 ? nch : ncm;
-            for (int c = cb; c < ce; ++c) {
-              mbar_wait_sleep(&yempty[ys], yph ^ 1);
-              uint8_t *yst = ystages + ys * C::YBYTES;
-              sm100::mbar_arrive_expect_tx(&yfull[ys], C::YBYTES);
-              if (phase < 2)
-                sm100::tma_load_2d(yst, &hmap, x0, c * C::DC, &yfull[ys]);  // read again later (L2)
-              else
-                sm100::tma_load_2d_hint(yst, phase == 2 ? &hmap : &ymap, x0, (phase == 2 ? 0 : n) + c * C::DC,
-                                        &yfull[ys], pol_first);  // last use
-              if (++ys == SY) {
-                ys = 0;
-                yph ^= 1;
-              }
-              if (kMergeProducers) {
-                // the chunk's B-operand tables (same chunk sequence as the stack)
-                const uint32_t tabbytes = phase == 0 ? C::TAB1 : phase == 1 ? C::TAB2 : C::TABY;
-                const uint32_t stride = phase == 0 ? C::TAB1 : phase < 3 ? C::TAB2 : C::TABY;
-                const uint8_t *tabsrc = phase == 0 ? tb.tab1 : phase < 3 ? tb.tab2 : tb.taby;
-                mbar_wait_sleep(&tempty[ts], tph ^ 1);
-                uint8_t *tst = tstages + ts * C::TSTAGE;
-                sm100::mbar_arrive_expect_tx(&tfull[ts], tabbytes);
-                sm100::bulk_g2s(tst, tabsrc + (size_t)c * stride, tabbytes, &tfull[ts]);
-                if (++ts == C::ST) {
-                  ts = 0;
-                  tph ^= 1;
-                }
-              }
-            }
-          }
-        }
-      }
-    } else if (warp == 5 && !kMergeProducers) {
-      // ------------------------------------------------------------ table producer
-      if (lane == 0) {
-        int ts = 0;
-        uint32_t tph = 0, sph = 0;
-        for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
-          int s0 = nch;
-          for (int phase = 0; phase < 4; ++phase) {
-            if (phase == 2) {
-              mbar_wait_sleep(&seedready, sph);
+              mbar_wait_sleep(A_seed, sph);
               sph ^= 1;
               s0 = min(min(seed_slot[0], seed_slot[1]), min(seed_slot[2], seed_slot[3]));
             }
@@ -547,10 +507,22 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
             const uint32_t stride = phase == 0 ? C::TAB1 : phase < 3 ? C::TAB2 : C::TABY;
             const uint8_t *tabsrc = phase == 0 ? tb.tab1 : phase < 3 ? tb.tab2 : tb.taby;
             for (int c = cb; c < ce; ++c) {
-              mbar_wait_sleep(&tempty[ts], tph ^ 1);
-              uint8_t *tst = tstages + ts * C::TSTAGE;
-              sm100::mbar_arrive_expect_tx(&tfull[ts], tabbytes);
-              sm100::bulk_g2s(tst, tabsrc + (size_t)c * stride, tabbytes, &tfull[ts]);
+              mbar_wait_sleep(A_yempty + 8 * ys, yph ^ 1);
+              const uint32_t yst = A_ys + ys * C::YBYTES, yb = A_yfull + 8 * ys;
+              sm100::mbar_arrive_expect_tx_a(yb, C::YBYTES);
+              if (phase < 2)
+                sm100::tma_load_2d_a(yst, &hmap, x0, c * C::DC, yb);  // read again later (L2)
+              else
+                sm100::tma_load_2d_hint_a(yst, phase == 2 ? &hmap : &ymap, x0, (phase == 2 ? 0 : n) + c * C::DC,
+                                          yb, pol_first);  // last use
+              if (++ys == SY) {
+                ys = 0;
+                yph ^= 1;
+              }
+              mbar_wait_sleep(A_tempty + 8 * ts, tph ^ 1);
+              const uint32_t tb_ = A_tfull + 8 * ts;
+              sm100::mbar_arrive_expect_tx_a(tb_, tabbytes);
+              sm100::bulk_g2s_a(A_ts + ts * C::TSTAGE, tabsrc + (size_t)c * stride, tabbytes, tb_);
               if (++ts == C::ST) {
                 ts = 0;
                 tph ^= 1;
@@ -565,7 +537,15 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
         const uint32_t idG = sm100::idesc_bf16_f32(128, C::NGn);
         const uint32_t idB = sm100::idesc_bf16_f32(128, C::KBn);
         const uint32_t idY = sm100::idesc_bf16_f32(128, C::DC);
-        const uint32_t aop = sm100::smem_u32(opb), tss = sm100::smem_u32(tstages);
+        const uint32_t aop = sm100::opaque(sm100::smem_u32(opb)), tss = sm100::opaque(sm100::smem_u32(tstages));
+        const uint32_t A_tfull = sm100::opaque(sm100::smem_u32(&tfull[0]));
+        const uint32_t A_tempty = sm100::opaque(sm100::smem_u32(&tempty[0]));
+        const uint32_t A_opfull = sm100::opaque(sm100::smem_u32(&opfull[0]));
+        const uint32_t A_opfree = sm100::opaque(sm100::smem_u32(&opfree[0]));
+        const uint32_t A_yhfull = sm100::opaque(sm100::smem_u32(&yhfull[0]));
+        const uint32_t A_yhfree = sm100::opaque(sm100::smem_u32(&yhfree[0]));
+        const uint32_t A_acc = sm100::opaque(sm100::smem_u32(&accready));
+        const uint32_t A_beta = sm100::opaque(sm100::smem_u32(&betaready));
         int ts = 0;
         uint32_t tph = 0, opcnt = 0, yissue = 0, bcnt = 0;
         auto tslot = [&](int ahead, uint32_t &par) {
@@ -587,7 +567,7 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
         auto opwait = [&]() -> uint32_t {
           const uint32_t ob = NOP == 2 ? (opcnt & 1) : 0;
           const uint32_t par = NOP == 2 ? ((opcnt >> 1) & 1) : (opcnt & 1);
-          mbar_wait_mma(&opfull[ob], par);
+          mbar_wait_mma(A_opfull + 8 * ob, par);
           return ob;
         };
         // yhat of the chunk `ahead` chunks after the current one (its table
@@ -596,8 +576,8 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
           uint32_t par;
           const int s = tslot(ahead, par);
           const uint32_t slot = yissue % C::NYS;
-          mbar_wait_mma(&yhfree[slot], ((yissue / C::NYS) & 1) ^ 1);  // consumers done with the slot
-          mbar_wait_mma(&tfull[s], par);
+          mbar_wait_mma(A_yhfree + 8 * slot, ((yissue / C::NYS) & 1) ^ 1);  // consumers done with the slot
+          mbar_wait_mma(A_tfull + 8 * s, par);
           sm100::tc_fence_after();
           const uint32_t b3 = tss + s * C::TSTAGE;
 #pragma unroll
@@ -606,14 +586,14 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
             for (int j = 0; j < C::KY / 16; ++j)
               sm100::umma_bf16_ts(tbase + C::col_y(slot, q), tbase + C::col_a3(q) + 8 * j,
                                   sm100::smem_desc(b3 + j * 2 * 256, 256, 128), idY, j > 0);
-          sm100::umma_commit(&yhfull[slot]);
+          sm100::umma_commit_a(A_yhfull + 8 * slot);
           ++yissue;
         };
         for (int64_t tile = blockIdx.x; tile < tb.ntiles; tile += gridDim.x) {
           // pass 1: Gram + moment per chunk, accumulator set c & 1
           for (int c = 0; c < nch; ++c) {
             const uint32_t ob = opwait();
-            mbar_wait_mma(&tfull[ts], tph);
+            mbar_wait_mma(A_tfull + 8 * ts, tph);
             sm100::tc_fence_after();
             const uint32_t bf = tss + ts * C::TSTAGE, bx = bf + 3 * C::BF_BYTES;
             const uint32_t first = c >= 2 ? 1u : 0u;
@@ -633,19 +613,19 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
               sm100::umma_bf16(dB, sm100::smem_desc(am + 2 * C::ATILE, 2048, 128),
                                sm100::smem_desc(bx, C::KBn * 16, 128), idB, 1);
             }
-            sm100::umma_commit(&opfree[ob]);
-            sm100::umma_commit(&tempty[ts]);
-            if (c == nch - 1) sm100::umma_commit(&accready);
+            sm100::umma_commit_a(A_opfree + 8 * ob);
+            sm100::umma_commit_a(A_tempty + 8 * ts);
+            if (c == nch - 1) sm100::umma_commit_a(A_acc);
             ++opcnt;
             tadvance();
           }
           // pass 2, history: yhat0 two chunks ahead, refinement moment per chunk
-          mbar_wait_mma(&betaready, bcnt & 1);
+          mbar_wait_mma(A_beta, bcnt & 1);
           ++bcnt;
           for (int a = 0; a < C::NYS && a < nch; ++a) issue_yhat(a);
           for (int c = 0; c < nch; ++c) {
             const uint32_t ob = opwait();
-            mbar_wait_mma(&tfull[ts], tph);
+            mbar_wait_mma(A_tfull + 8 * ts, tph);
             sm100::tc_fence_after();
             const uint32_t bx = tss + ts * C::TSTAGE + C::B3_BYTES;
 #pragma unroll
@@ -661,23 +641,23 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
                                    sm100::smem_desc(bx + x * C::BX_BYTES, C::KBn * 16, 128), idB,
                                    (c > 0 || e > 0 || x > 0) ? 1u : 0u);
             }
-            sm100::umma_commit(&opfree[ob]);
+            sm100::umma_commit_a(A_opfree + 8 * ob);
             if (c + C::NYS < nch) issue_yhat(C::NYS);
-            sm100::umma_commit(&tempty[ts]);
-            if (c == nch - 1) sm100::umma_commit(&accready);
+            sm100::umma_commit_a(A_tempty + 8 * ts);
+            if (c == nch - 1) sm100::umma_commit_a(A_acc);
             ++opcnt;
             tadvance();
           }
           // pass 3, seed chunks + monitoring: yhat with the refined beta, two
           // chunks ahead (the consumers published s0 before betaready)
-          mbar_wait_mma(&betaready, bcnt & 1);
+          mbar_wait_mma(A_beta, bcnt & 1);
           ++bcnt;
           const int s0 = min(min(seed_slot[0], seed_slot[1]), min(seed_slot[2], seed_slot[3]));
           const int n3 = nch - s0 + ncm;
           for (int a = 0; a < C::NYS && a < n3; ++a) issue_yhat(a);
           for (int c = 0; c < n3; ++c) {
             if (c + C::NYS < n3) issue_yhat(C::NYS);
-            sm100::umma_commit(&tempty[ts]);  // chunk c's table was read by its yhat MMA
+            sm100::umma_commit_a(A_tempty + 8 * ts);  // chunk c's table was read by its yhat MMA
             tadvance();
           }
         }
@@ -693,14 +673,20 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
     const uint32_t lanebase = tbase + ((uint32_t)(32 * warp) << 16);
     const float qnan = __int_as_float(0x7fc00000);
     // ring: slot s = PIX residuals f32, pixel q of this thread at rbase + 4q + s*RSLOT
-    const uint32_t rbase = sm100::smem_u32(ring) + 4 * PX * tid;
+    const uint32_t rbase = sm100::opaque(sm100::smem_u32(ring) + 4 * PX * tid);
     int ys = 0;
     uint32_t yph = 0, opcnt = 0, yuse = 0, acnt = 0;
     // 32-bit shared addresses of the barriers this warp waits on / arrives at
-    const uint32_t a_yfull = sm100::smem_u32(&yfull[0]), a_yempty = sm100::smem_u32(&yempty[0]);
-    const uint32_t a_opfull = sm100::smem_u32(&opfull[0]), a_opfree = sm100::smem_u32(&opfree[0]);
-    const uint32_t a_yhfull = sm100::smem_u32(&yhfull[0]), a_yhfree = sm100::smem_u32(&yhfree[0]);
-    const uint32_t a_accready = sm100::smem_u32(&accready), a_betaready = sm100::smem_u32(&betaready);
+    // (sm100::opaque: kept in registers, not recomputed from the CTA's cluster rank)
+    const uint32_t a_yfull = sm100::opaque(sm100::smem_u32(&yfull[0]));
+    const uint32_t a_yempty = sm100::opaque(sm100::smem_u32(&yempty[0]));
+    const uint32_t a_opfull = sm100::opaque(sm100::smem_u32(&opfull[0]));
+    const uint32_t a_opfree = sm100::opaque(sm100::smem_u32(&opfree[0]));
+    const uint32_t a_yhfull = sm100::opaque(sm100::smem_u32(&yhfull[0]));
+    const uint32_t a_yhfree = sm100::opaque(sm100::smem_u32(&yhfree[0]));
+    const uint32_t a_accready = sm100::opaque(sm100::smem_u32(&accready));
+    const uint32_t a_betaready = sm100::opaque(sm100::smem_u32(&betaready));
+    const uint32_t a_ystages = sm100::opaque(sm100::smem_u32(ystages));
 
     auto yadvance = [&]() {
       if (++ys == SY) {
@@ -774,15 +760,18 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
       ++yuse;
     };
     // the 8 dates of a half chunk for this thread's pixels: yv[q][d]
-    auto load_y8 = [&](const float *Ys, int hf, float (&yv)[PX][8]) {
+    // Ys = shared address of the stage (a register, see a_yfull)
+    auto load_y8 = [&](uint32_t Ys, int hf, float (&yv)[PX][8]) {
+      const uint32_t a = Ys + 4 * (8 * hf * C::PIX + PX * tid);
 #pragma unroll
       for (int d = 0; d < 8; ++d) {
         if (PX == 2) {
-          const float2 v = *reinterpret_cast<const float2 *>(Ys + (8 * hf + d) * C::PIX + 2 * tid);
-          yv[0][d] = v.x;
-          yv[PX - 1][d] = v.y;
+          asm volatile("ld.shared.v2.f32 {%0, %1}, [%2];"
+                       : "=f"(yv[0][d]), "=f"(yv[PX - 1][d])
+                       : "r"(a + 4 * d * C::PIX)
+                       : "memory");
         } else {
-          yv[0][d] = Ys[(8 * hf + d) * C::PIX + tid];
+          yv[0][d] = lds_f32(a + 4 * d * C::PIX);
         }
       }
     };
@@ -803,7 +792,7 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
       }
       for (int c = 0; c < nch; ++c) {
         sm100::mbar_wait_a(a_yfull + 8 * ys, yph);
-        const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
+        const uint32_t Ys = a_ystages + ys * C::YBYTES;
         // offset c = first valid value (warp-uniform pre-scan while a lane lacks it)
         bool need = false;
 #pragma unroll
@@ -812,7 +801,7 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
 #pragma unroll
           for (int q = 0; q < PX; ++q)
             for (int d = 0; d < C::DC && !have[q]; ++d) {
-              const float y = Ys[d * C::PIX + PX * tid + q];
+              const float y = lds_f32(Ys + 4 * (d * C::PIX + PX * tid + q));
               if (y == y) {
                 c0[q] = y;
                 have[q] = true;
@@ -966,7 +955,7 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
       for (int c = 0; c < nch; ++c) {
         sm100::mbar_wait_a(a_yfull + 8 * ys, yph);
         wait_yhat();
-        const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
+        const uint32_t Ys = a_ystages + ys * C::YBYTES;
         uint8_t *ob = nullptr;
         uint32_t vb[PX];  // validity of the chunk's 16 dates
 #pragma unroll
@@ -1114,7 +1103,7 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
         sm100::mbar_wait_a(a_yfull + 8 * ys, yph);
         wait_yhat();
         if (c >= sw) {
-          const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
+          const uint32_t Ys = a_ystages + ys * C::YBYTES;
 #pragma unroll 1
           for (int hf = 0; hf < 2; ++hf) {
             float yh[PX][8], yv[PX][8];
@@ -1188,7 +1177,7 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
       for (int c = 0; c < ncm; ++c) {
         sm100::mbar_wait_a(a_yfull + 8 * ys, yph);
         wait_yhat();
-        const float *Ys = reinterpret_cast<const float *>(ystages + ys * C::YBYTES);
+        const uint32_t Ys = a_ystages + ys * C::YBYTES;
         // B_j == lambda for every rank this chunk can reach (rank/nbar <= e)
         // for all of the thread's valid pixels: warp-uniform fast path without
         // the out-of-line boundary evaluation
