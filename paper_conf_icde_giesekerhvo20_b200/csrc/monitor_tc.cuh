@@ -346,26 +346,29 @@ __device__ __forceinline__ void mon_date(float y, float c0, float yh, float &W, 
 // from date to date; every date's address is a fresh value, so a store does
 // not hold up the next date's pointer arithmetic (write-after-read on the
 // address register).  Needs h >= 8 (at most one wrap per 8-date half).
+// wv = W after a valid date, 0 after a missing one (the crossing scan of a
+// half reads these instead of replaying the half).
 template <int RSLOT>
 __device__ __forceinline__ void mon_date_k(float y, float c0, float yh, float &W, float &msum, float &mx, uint32_t &k,
-                                           uint32_t wa, uint32_t jw, uint32_t hbytes, float &r, float &old) {
+                                           uint32_t wa, uint32_t jw, uint32_t hbytes, float &wv) {
   asm volatile(
-      "{\n\t.reg .pred p, q;\n\t.reg .f32 t;\n\t.reg .u32 a;\n\t"
-      "sub.f32 %4, %6, %7;\n\t"
-      "sub.f32 %4, %4, %8;\n\t"
-      "setp.num.f32 p, %4, %4;\n\t"
-      "mad.lo.u32 a, %3, %12, %9;\n\t"
-      "setp.ge.u32 q, %3, %10;\n\t"
-      "@q sub.u32 a, a, %11;\n\t"
-      "ld.shared.f32 %5, [a];\n\t"
-      "@p st.shared.f32 [a], %4;\n\t"
+      "{\n\t.reg .pred p, q;\n\t.reg .f32 r, o, t;\n\t.reg .u32 a;\n\t"
+      "sub.f32 r, %5, %6;\n\t"
+      "sub.f32 r, r, %7;\n\t"
+      "setp.num.f32 p, r, r;\n\t"
+      "mad.lo.u32 a, %3, %11, %8;\n\t"
+      "setp.ge.u32 q, %3, %9;\n\t"
+      "@q sub.u32 a, a, %10;\n\t"
+      "ld.shared.f32 o, [a];\n\t"
+      "@p st.shared.f32 [a], r;\n\t"
       "@p add.u32 %3, %3, 1;\n\t"
-      "sub.f32 t, %4, %5;\n\t"
+      "sub.f32 t, r, o;\n\t"
       "@p add.f32 %0, %0, t;\n\t"
       "@p add.f32 %1, %1, %0;\n\t"
       "abs.f32 t, %0;\n\t"
-      "@p max.f32 %2, %2, t;\n\t}"
-      : "+f"(W), "+f"(msum), "+f"(mx), "+r"(k), "=f"(r), "=f"(old)
+      "@p max.f32 %2, %2, t;\n\t"
+      "selp.f32 %4, %0, 0f00000000, p;\n\t}"
+      : "+f"(W), "+f"(msum), "+f"(mx), "+r"(k), "=f"(wv)
       : "f"(y), "f"(c0), "f"(yh), "r"(wa), "r"(jw), "r"(hbytes), "n"(RSLOT)
       : "memory");
 }
@@ -1198,11 +1201,10 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
           if (fast) {
             // B_j == lambda here: the first |m| > lambda(1 - tol) decides (a
             // clear crossing is the break, a near tie goes to the fp64 refit).
-            // The dates only track max |W|; a half in which it crossed
-            // replays its 8 steps from the saved state (same arithmetic).
-            float W0[PX], rr[PX][8], oo[PX][8];
-#pragma unroll
-            for (int q = 0; q < PX; ++q) W0[q] = W[q];
+            // The dates only track max |W| and keep W at each valid date
+            // (wv); a half in which max |W| crossed is scanned for the first
+            // crossing date.
+            float wv[PX][8];
             if (ring8) {
               // slot addresses from the half's running count (mon_date_k);
               // pixel-major order: each pixel's 8 loads issue back to back
@@ -1217,7 +1219,7 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
 #pragma unroll
                 for (int d = 0; d < 8; ++d)
                   mon_date_k<C::RSLOT>(yv[q][d], c0[q], yh[q][d], W[q], msum[q], mx[q], kk[q], wa[q], jw[q],
-                                       hbytes[q], rr[q][d], oo[q][d]);
+                                       hbytes[q], wv[q][d]);
 #pragma unroll
               for (int q = 0; q < PX; ++q) {
                 cr[q] += (int)kk[q];
@@ -1228,25 +1230,27 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
 #pragma unroll
               for (int d = 0; d < 8; ++d)
 #pragma unroll
-                for (int q = 0; q < PX; ++q)
+                for (int q = 0; q < PX; ++q) {
+                  float r, old;
                   mon_date<C::RSLOT>(yv[q][d], c0[q], yh[q][d], W[q], msum[q], mx[q], cr[q], wa[q], rend[q],
-                                     hbytes[q], rr[q][d], oo[q][d]);
+                                     hbytes[q], r, old);
+                  wv[q][d] = r == r ? W[q] : 0.f;
+                }
             }
 
 #pragma unroll
             for (int q = 0; q < PX; ++q) {
-              if (mx[q] > thr_lo[q]) {
-                float Wr = W0[q];
+              if (mx[q] > thr_lo[q]) {  // first[q] < 0 while thr_lo is finite
+                int fd = 7;
+                float fw = wv[q][7];
 #pragma unroll
-                for (int d = 0; d < 8; ++d) {
-                  if (rr[q][d] == rr[q][d]) {
-                    Wr += rr[q][d] - oo[q][d];
-                    if (first[q] < 0 && fabsf(Wr) > thr_lo[q]) {
-                      first[q] = c * C::DC + 8 * hf + d;
-                      mfirst[q] = Wr;
-                    }
+                for (int d = 6; d >= 0; --d)
+                  if (fabsf(wv[q][d]) > thr_lo[q]) {
+                    fd = d;
+                    fw = wv[q][d];
                   }
-                }
+                first[q] = c * C::DC + 8 * hf + fd;
+                mfirst[q] = fw;
                 thr_lo[q] = __int_as_float(0x7f800000);
               }
             }
