@@ -94,6 +94,24 @@ constexpr bool kEarlyRelease = BFAST_EARLY_REL != 0;
 #define BFAST_YS 2
 #endif
 constexpr int kYhatSlots = BFAST_YS;
+// unroll factors of the two 8-date halves of a chunk per sweep (1 keeps one
+// copy of the hot code per sweep: instruction-cache footprint)
+#ifndef BFAST_UNROLL_P1
+#define BFAST_UNROLL_P1 1
+#endif
+constexpr int kUnrollP1 = BFAST_UNROLL_P1;
+#ifndef BFAST_UNROLL_P2
+#define BFAST_UNROLL_P2 2
+#endif
+constexpr int kUnrollP2 = BFAST_UNROLL_P2;
+#ifndef BFAST_UNROLL_SEED
+#define BFAST_UNROLL_SEED 1
+#endif
+constexpr int kUnrollSeed = BFAST_UNROLL_SEED;
+#ifndef BFAST_UNROLL_MON
+#define BFAST_UNROLL_MON 1
+#endif
+constexpr int kUnrollMon = BFAST_UNROLL_MON;
 // k-indexed ring slots in the seed pass too (the monitoring fast path always
 // uses them when every pixel of the warp has h >= 8)
 #ifndef BFAST_SEEDK
@@ -812,7 +830,7 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
             }
         }
         uint8_t *ob = nullptr;
-#pragma unroll 1
+#pragma unroll kUnrollP1
         for (int hf = 0; hf < 2; ++hf) {  // two halves of 8 dates: half the hot code
           float yv[PX][8];
           load_y8(Ys, hf, yv);  // dates >= n read as NaN (hmap)
@@ -963,7 +981,7 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
         uint32_t vb[PX];  // validity of the chunk's 16 dates
 #pragma unroll
         for (int q = 0; q < PX; ++q) vb[q] = 0;
-#pragma unroll 1
+#pragma unroll kUnrollP2
         for (int hf = 0; hf < 2; ++hf) {
           float yh[PX][8], yv[PX][8];
           load_yhat8(hf, yh);
@@ -1107,7 +1125,7 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
         wait_yhat();
         if (c >= sw) {
           const uint32_t Ys = a_ystages + ys * C::YBYTES;
-#pragma unroll 1
+#pragma unroll kUnrollSeed
           for (int hf = 0; hf < 2; ++hf) {
             float yh[PX][8], yv[PX][8];
             load_yhat8(hf, yh);
@@ -1188,7 +1206,7 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
 #pragma unroll
         for (int q = 0; q < PX; ++q) crm = max(crm, deg[q] ? 0 : cr[q] - nbar[q]);
         const bool fast = __all_sync(0xffffffffu, crm + C::DC <= rank_flat_min);
-#pragma unroll 1
+#pragma unroll kUnrollMon
         for (int hf = 0; hf < 2; ++hf) {
           float yh[PX][8], yv[PX][8];
           load_yhat8(hf, yh);
