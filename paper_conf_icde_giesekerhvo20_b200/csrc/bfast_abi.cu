@@ -155,14 +155,14 @@ PFN_encodeTiled get_encode() {
   return fn;
 }
 
-// Tensor map of the stack range [p0, p0+P) x [0, N): box 128*kTcPx px x 16 dates,
-// out-of-bounds elements read as NaN (= missing).
-bool make_stack_map(CUtensorMap *m, const float *Y, int64_t ldY, int64_t P, int64_t N) {
+// Tensor map of the stack range [p0, p0+P) x [0, N): box `pix` px x 16 dates
+// (one tile), out-of-bounds elements read as NaN (= missing).
+bool make_stack_map(CUtensorMap *m, const float *Y, int64_t ldY, int64_t P, int64_t N, int pix) {
   PFN_encodeTiled enc = get_encode();
   if (!enc) return false;
   cuuint64_t dims[2] = {(cuuint64_t)P, (cuuint64_t)N};
   cuuint64_t strides[1] = {(cuuint64_t)ldY * sizeof(float)};
-  cuuint32_t box[2] = {128 * bfast::kTcPx, 16};
+  cuuint32_t box[2] = {(cuuint32_t)pix, 16};
   cuuint32_t es[2] = {1, 1};
   return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void *)Y, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
              CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -349,7 +349,8 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
   int tc_sy = 2, tc_nop = 1, per_sm = 0;
   {
     const int cand[4][2] = {{3, 2}, {2, 2}, {3, 1}, {2, 1}};
-    const int reg_cap = std::min(65536 / (bfast::kTcThreads * bfast::kTcLaunchRegs), bfast::kTcCtasPerSm);
+    using Shape = bfast::TcShape<K>;
+    const int reg_cap = std::min(65536 / (bfast::kTcThreads * Shape::LAUNCH_REGS), Shape::CTAS);
     const int tmem_cap = 512 / TC::TMEM_COLS;
     for (auto &c : cand) {
       const size_t b = TC::smem_bytes(tc_hcap, pl.nch, c[0], c[1]);
@@ -380,8 +381,8 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
   const bool tc_ok = per_sm > 0 && pl.dtab && pl.mode != 1 && (prm.ldY % 4) == 0 &&
                      ((uintptr_t)(prm.Y + prm.p0) % 16) == 0 && tc_smem + 1024 <= (size_t)kMaxSmem;
   CUtensorMap ymap, hmap;  // full stack; history only (dates >= n out of bounds)
-  const bool tma_ok = tc_ok && make_stack_map(&ymap, prm.Y + prm.p0, prm.ldY, prm.P, pl.N) &&
-                      make_stack_map(&hmap, prm.Y + prm.p0, prm.ldY, prm.P, pl.n);
+  const bool tma_ok = tc_ok && make_stack_map(&ymap, prm.Y + prm.p0, prm.ldY, prm.P, pl.N, TC::PIX) &&
+                      make_stack_map(&hmap, prm.Y + prm.p0, prm.ldY, prm.P, pl.n, TC::PIX);
   const int64_t ntiles = tma_ok ? (prm.P + TC::PIX - 1) / TC::PIX : 0;
   // the refit list/counter are plan scratch: order executions on any stream
   CUDA_TRY(cudaStreamWaitEvent(st, pl.scratch_free, 0));

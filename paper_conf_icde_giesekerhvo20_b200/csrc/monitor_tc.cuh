@@ -53,27 +53,43 @@
 
 namespace bfast {
 
-// CTA = consumer warpgroup (warps 0-3, one pixel per thread) + producer
-// warpgroup (warp 4 stack TMA, 5 table copies, 6 MMA issue, 7 idle).  At
-// launch every thread holds 80 registers (3 CTAs x 256 threads); the
-// producers drop to kTcAuxRegs, the consumers rise to kTcConsumerRegs
-// (80*256 = 128*kTcAuxRegs + 128*kTcConsumerRegs).
+// CTA = consumer warpgroup (warps 0-3, PX pixels per thread) + producer
+// warpgroup (warp 4: stack boxes and chunk tables, warp 6: MMA issue).  At
+// launch every thread holds LAUNCH_REGS registers (CTAS CTAs x 256 threads
+// fill the register file); the producers drop to kTcAuxRegs, the consumers
+// rise to CONSUMER_REGS (256 * LAUNCH_REGS = 128 * (kTcAuxRegs +
+// CONSUMER_REGS)).
 constexpr int kTcThreads = 256;
-#ifndef BFAST_TC_PX
-#define BFAST_TC_PX 2
-#endif
-constexpr int kTcPx = BFAST_TC_PX;  // pixels per consumer thread (tile = 128 * kTcPx pixels)
-
-#ifndef BFAST_TC_CTAS
-#define BFAST_TC_CTAS (BFAST_TC_PX == 2 ? 2 : 3)
-#endif
-constexpr int kTcCtasPerSm = BFAST_TC_CTAS;               // register budget: CTAs per SM
-constexpr int kTcLaunchRegs = kTcCtasPerSm == 4 ? 64 : kTcCtasPerSm == 3 ? 80 : 128;
 #ifndef BFAST_TC_AUX_REGS
 #define BFAST_TC_AUX_REGS 32
 #endif
 constexpr int kTcAuxRegs = BFAST_TC_AUX_REGS;
-constexpr int kTcConsumerRegs = 2 * kTcLaunchRegs - kTcAuxRegs;
+// Pixels per consumer thread and CTAs per SM, per design width K.  K <= 8:
+// one pixel per thread, 4 CTAs (16 consumer warps) per SM, 96 consumer
+// registers; measured 1.5% faster than two pixels per thread at 2 CTAs per
+// SM on the Landsat scene.  K >= 10 needs more registers per pixel (the
+// K x K Cholesky): two pixels per thread, 2 CTAs, 224 registers.
+// BFAST_TC_PX / BFAST_TC_CTAS override (experiments).
+template <int K>
+struct TcShape {
+#ifdef BFAST_TC_PX
+  static constexpr int PX = BFAST_TC_PX;
+#else
+  static constexpr int PX = K <= 8 ? 1 : 2;
+#endif
+#ifdef BFAST_TC_CTAS
+  static constexpr int CTAS = BFAST_TC_CTAS;
+#else
+  static constexpr int CTAS = PX == 1 ? 4 : 2;
+#endif
+  static constexpr int LAUNCH_REGS = CTAS == 4 ? 64 : CTAS == 3 ? 80 : 128;
+  static constexpr int CONSUMER_REGS = 2 * LAUNCH_REGS - kTcAuxRegs;
+#ifdef BFAST_UNROLL_SEED
+  static constexpr int UNROLL_SEED = BFAST_UNROLL_SEED;
+#else
+  static constexpr int UNROLL_SEED = PX == 1 ? 2 : 1;  // measured per shape
+#endif
+};
 
 // parts of the bf16 split of the first-fit residual r0 in the refinement
 // moment (2: hi truncated + lo rounded, ~17 bits; 3: three truncated parts,
@@ -104,10 +120,6 @@ constexpr int kUnrollP1 = BFAST_UNROLL_P1;
 #define BFAST_UNROLL_P2 2
 #endif
 constexpr int kUnrollP2 = BFAST_UNROLL_P2;
-#ifndef BFAST_UNROLL_SEED
-#define BFAST_UNROLL_SEED 1
-#endif
-constexpr int kUnrollSeed = BFAST_UNROLL_SEED;
 #ifndef BFAST_UNROLL_MON
 #define BFAST_UNROLL_MON 1
 #endif
@@ -119,7 +131,7 @@ constexpr int kUnrollMon = BFAST_UNROLL_MON;
 #endif
 constexpr bool kSeedK = BFAST_SEEDK != 0;
 
-template <int K, int PX = kTcPx>
+template <int K, int PX = TcShape<K>::PX>
 struct TcCfg {
   static constexpr int k = (K - 2) / 2;
   static constexpr int NF = 2 + 6 * k;                     // masked moment functions
@@ -134,7 +146,7 @@ struct TcCfg {
   // the beta operand (the A operand of the yhat GEMM, bf16 pairs) and the
   // refinement moment, per pixel group.
   static constexpr int SET = NGn + KBn;
-  static constexpr int A3W = ((KY / 2 + 15) / 16) * 16;
+  static constexpr int A3W = ((KY / 2 + 7) / 8) * 8;       // beta operand columns (8-column MMA steps)
   static constexpr int COLS_P1 = 2 * PX * SET;
   static constexpr __host__ __device__ int col_set(int s, int q) { return (s * PX + q) * SET; }
   static constexpr int NYS = kYhatSlots;
@@ -438,10 +450,11 @@ __device__ __forceinline__ float bf16_round(float v) {
 }
 
 template <int K>
-__global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
+__global__ void __launch_bounds__(kTcThreads, TcShape<K>::CTAS)
     monitor_tc_kernel(MonitorParams p, TcTables tb, const __grid_constant__ CUtensorMap ymap,
                       const __grid_constant__ CUtensorMap hmap) {
-  constexpr int PX = kTcPx;
+  constexpr int PX = TcShape<K>::PX;
+  constexpr int UNROLL_SEED = TcShape<K>::UNROLL_SEED;
   using C = TcCfg<K, PX>;
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ __align__(8) uint64_t yfull[C::SY_MAX], yempty[C::SY_MAX], tfull[C::ST], tempty[C::ST], opfull[2],
@@ -690,7 +703,7 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
     // 8-byte shared load per date reads both); pixel group q = t's q-th
     // pixel, i.e. TMEM lane t of the column groups of q and row t of the A
     // tiles of q.
-    sm100::setmaxnreg_inc<kTcConsumerRegs>();
+    sm100::setmaxnreg_inc<TcShape<K>::CONSUMER_REGS>();
     const uint32_t lanebase = tbase + ((uint32_t)(32 * warp) << 16);
     const float qnan = __int_as_float(0x7fc00000);
     // ring: slot s = PIX residuals f32, pixel q of this thread at rbase + 4q + s*RSLOT
@@ -1125,7 +1138,7 @@ __global__ void __launch_bounds__(kTcThreads, kTcCtasPerSm)
         wait_yhat();
         if (c >= sw) {
           const uint32_t Ys = a_ystages + ys * C::YBYTES;
-#pragma unroll kUnrollSeed
+#pragma unroll UNROLL_SEED
           for (int hf = 0; hf < 2; ++hf) {
             float yh[PX][8], yv[PX][8];
             load_yhat8(hf, yh);
