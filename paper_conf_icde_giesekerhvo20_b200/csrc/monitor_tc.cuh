@@ -110,6 +110,13 @@ constexpr bool kEarlyRelease = BFAST_EARLY_REL != 0;
 #define BFAST_YS 2
 #endif
 constexpr int kYhatSlots = BFAST_YS;
+// MMA A operands (mask / y' parts, r0 parts) written by the consumers into
+// Tensor Memory with tcgen05.st (1) instead of shared memory (0), where the
+// layout fits the CTA's TMEM allocation (one accumulator set then)
+#ifndef BFAST_TMEM_OPS
+#define BFAST_TMEM_OPS 1
+#endif
+constexpr bool kTmemOpsWanted = BFAST_TMEM_OPS != 0;
 // unroll factors of the two 8-date halves of a chunk per sweep (1 keeps one
 // copy of the hot code per sweep: instruction-cache footprint)
 #ifndef BFAST_UNROLL_P1
@@ -147,16 +154,28 @@ struct TcCfg {
   // refinement moment, per pixel group.
   static constexpr int SET = NGn + KBn;
   static constexpr int A3W = ((KY / 2 + 7) / 8) * 8;       // beta operand columns (8-column MMA steps)
-  static constexpr int COLS_P1 = 2 * PX * SET;
-  static constexpr __host__ __device__ int col_set(int s, int q) { return (s * PX + q) * SET; }
   static constexpr int NYS = kYhatSlots;
+  static constexpr int OPC = 3 * DC / 2;                   // three [128 x 16] bf16 A tiles, 8 columns each
+  static constexpr int P2B = NYS * PX * DC + PX * A3W + PX * KBn;
+  static constexpr __host__ __device__ int pow2cols(int c) {
+    return c <= 32 ? 32 : c <= 64 ? 64 : c <= 128 ? 128 : c <= 256 ? 256 : 512;
+  }
+  // shared-memory operands: two accumulator sets; TMEM operands: one set and
+  // two operand buffers per pass, taken only where that fits the allocation
+  static constexpr int COLS_SMEM = pow2cols(2 * PX * SET > P2B ? 2 * PX * SET : P2B);
+  static constexpr int P1T = PX * SET + 2 * PX * OPC, P2T = P2B + 2 * PX * OPC;
+  static constexpr bool TOPS = kTmemOpsWanted && pow2cols(P1T > P2T ? P1T : P2T) <= COLS_SMEM;
+  static constexpr int NSET = TOPS ? 1 : 2;
+  static constexpr int COLS_P1 = TOPS ? P1T : 2 * PX * SET;
+  static constexpr __host__ __device__ int col_set(int s, int q) { return (s * PX + q) * SET; }
+  static constexpr __host__ __device__ int col_op1(int b, int q) { return PX * SET + (b * PX + q) * OPC; }
   static constexpr __host__ __device__ int col_y(int slot, int q) { return (slot * PX + q) * DC; }
   static constexpr __host__ __device__ int col_a3(int q) { return NYS * PX * DC + q * A3W; }
   static constexpr __host__ __device__ int col_db(int q) { return NYS * PX * DC + PX * A3W + q * KBn; }
-  static constexpr int COLS_P2 = NYS * PX * DC + PX * A3W + PX * KBn;
+  static constexpr __host__ __device__ int col_op2(int b, int q) { return P2B + (b * PX + q) * OPC; }
+  static constexpr int COLS_P2 = TOPS ? P2T : P2B;
   static constexpr int COLS_USED = COLS_P1 > COLS_P2 ? COLS_P1 : COLS_P2;
-  static constexpr int TMEM_COLS = COLS_USED <= 32 ? 32 : COLS_USED <= 64 ? 64 : COLS_USED <= 128 ? 128
-                                   : COLS_USED <= 256 ? 256 : 512;
+  static constexpr int TMEM_COLS = pow2cols(COLS_USED);
   static constexpr int BF_BYTES = NGn * DC * 2;            // one part of the Gram table [NGn x 16]
   static constexpr int BX_BYTES = KBn * DC * 2;            // one part of x [KBn x 16]
   static constexpr int B3_BYTES = DC * KY * 2;             // yhat table [16 x KY]
@@ -176,7 +195,7 @@ struct TcCfg {
   // (the operands are dead once the refinement moment is accumulated, the
   // ring is dead once the tile's monitoring is done)
   static constexpr size_t smem_bytes(int hcap, int nch, int sy, int nop) {
-    const size_t ob = (size_t)nop * OPBUF, rg = (size_t)hcap * RSLOT;
+    const size_t ob = TOPS ? 0 : (size_t)nop * OPBUF, rg = (size_t)hcap * RSLOT;
     return (size_t)sy * YBYTES + (size_t)ST * TSTAGE + ((ob > rg ? ob : rg) + 127) / 128 * 128 + 0 * nch;
   }
 };
@@ -461,7 +480,7 @@ __global__ void __launch_bounds__(kTcThreads, TcShape<K>::CTAS)
       opfree[2], yhfull[C::NYS], yhfree[C::NYS], accready, betaready, seedready;
   __shared__ uint32_t tmem_base_s;
   __shared__ int seed_slot[4];  // per consumer warp: first history chunk its MOSUM seed needs
-  const int SY = tb.sy, NOP = tb.nop;
+  const int SY = tb.sy, NOP = C::TOPS ? 2 : tb.nop;
   uint8_t *ystages = smem;
   uint8_t *tstages = ystages + SY * C::YBYTES;
   uint8_t *opb = tstages + C::ST * C::TSTAGE;
@@ -630,11 +649,22 @@ __global__ void __launch_bounds__(kTcThreads, TcShape<K>::CTAS)
             mbar_wait_mma(A_tfull + 8 * ts, tph);
             sm100::tc_fence_after();
             const uint32_t bf = tss + ts * C::TSTAGE, bx = bf + 3 * C::BF_BYTES;
-            const uint32_t first = c >= 2 ? 1u : 0u;
+            const uint32_t first = c >= C::NSET ? 1u : 0u;
 #pragma unroll
             for (int q = 0; q < PX; ++q) {
+              const uint32_t dG = tbase + C::col_set(C::NSET == 2 ? (c & 1) : 0, q), dB = dG + C::NGn;
+              if (C::TOPS) {
+                const uint32_t at = tbase + C::col_op1(ob, q);  // mask, y' hi, y' lo tiles (TMEM)
+#pragma unroll
+                for (int e = 0; e < 3; ++e)
+                  sm100::umma_bf16_ts(dG, at, sm100::smem_desc(bf + e * C::BF_BYTES, C::NGn * 16, 128), idG,
+                                      first | (e > 0));
+                sm100::umma_bf16_ts(dB, at + 8, sm100::smem_desc(bx, C::KBn * 16, 128), idB, first);
+                sm100::umma_bf16_ts(dB, at + 8, sm100::smem_desc(bx + C::BX_BYTES, C::KBn * 16, 128), idB, 1);
+                sm100::umma_bf16_ts(dB, at + 16, sm100::smem_desc(bx, C::KBn * 16, 128), idB, 1);
+                continue;
+              }
               const uint32_t am = aop + ob * C::OPBUF + q * 3 * C::ATILE;  // mask, y' hi, y' lo tiles
-              const uint32_t dG = tbase + C::col_set(c & 1, q), dB = dG + C::NGn;
 #pragma unroll
               for (int e = 0; e < 3; ++e)
                 sm100::umma_bf16(dG, sm100::smem_desc(am, 2048, 128),
@@ -665,15 +695,20 @@ __global__ void __launch_bounds__(kTcThreads, TcShape<K>::CTAS)
 #pragma unroll
             for (int q = 0; q < PX; ++q) {
               const uint32_t am = aop + ob * C::OPBUF + q * 3 * C::ATILE;  // r0 parts
+              const uint32_t at = tbase + C::col_op2(ob, q);                // (TMEM)
               const uint32_t dD = tbase + C::col_db(q);
               // r0hi (x_hi + x_mid + x_lo) + r0mid (x_hi + x_mid) + r0lo x_hi
 #pragma unroll
               for (int e = 0; e < kR0Parts; ++e)
 #pragma unroll
-                for (int x = 0; x < 3 - e; ++x)
-                  sm100::umma_bf16(dD, sm100::smem_desc(am + e * C::ATILE, 2048, 128),
-                                   sm100::smem_desc(bx + x * C::BX_BYTES, C::KBn * 16, 128), idB,
-                                   (c > 0 || e > 0 || x > 0) ? 1u : 0u);
+                for (int x = 0; x < 3 - e; ++x) {
+                  const uint64_t bd = sm100::smem_desc(bx + x * C::BX_BYTES, C::KBn * 16, 128);
+                  const uint32_t acc = (c > 0 || e > 0 || x > 0) ? 1u : 0u;
+                  if (C::TOPS)
+                    sm100::umma_bf16_ts(dD, at + 8 * e, bd, idB, acc);
+                  else
+                    sm100::umma_bf16(dD, sm100::smem_desc(am + e * C::ATILE, 2048, 128), bd, idB, acc);
+                }
             }
             sm100::umma_commit_a(A_opfree + 8 * ob);
             if (c + C::NYS < nch) issue_yhat(C::NYS);
@@ -741,9 +776,20 @@ __global__ void __launch_bounds__(kTcThreads, TcShape<K>::CTAS)
     };
     auto opbuf_publish = [&]() {
       const uint32_t ob = NOP == 2 ? (opcnt & 1) : 0;
-      sm100::fence_proxy_async_smem();
+      if (C::TOPS) {
+        sm100::tmem_st_wait();  // this warp's operand rows are in TMEM
+        sm100::tc_fence_before();
+      } else {
+        sm100::fence_proxy_async_smem();
+      }
       warp_arrive(a_opfull + 8 * ob);
       ++opcnt;
+    };
+    // this thread's row of the three operand tiles of buffer `opcnt & 1`,
+    // dates 8 hf .. 8 hf + 7 (4 columns of bf16 pairs per tile)
+    auto tmem_ops = [&](uint32_t col, int hf, const uint32_t (&w)[3][4]) {
+#pragma unroll
+      for (int e = 0; e < 3; ++e) sm100::tmem_st4(lanebase + col + 8 * e + 4 * hf, w[e][0], w[e][1], w[e][2], w[e][3]);
     };
     // A3 rows (TMEM) = [bh | bh | bh | bm | bm | bl | 0...] (6 blocks of K, KY bf16) per pixel group
     auto write_beta_operand = [&](const float (&bt)[PX][K]) {
@@ -814,7 +860,7 @@ __global__ void __launch_bounds__(kTcThreads, TcShape<K>::CTAS)
       const int64_t pix0 = p.p0 + tile * C::PIX + PX * tid;
       // the operand buffers reuse the ring's bytes: every consumer warp must
       // be done with the previous tile's monitoring before any writes them
-      asm volatile("bar.sync 1, 128;" ::: "memory");
+      if (!C::TOPS) asm volatile("bar.sync 1, 128;" ::: "memory");
       // ================= pass 1: masked Gram + moment on the tensor cores
       float c0[PX], ymax[PX];
       bool have[PX];
@@ -863,6 +909,20 @@ __global__ void __launch_bounds__(kTcThreads, TcShape<K>::CTAS)
           // the MMA of the previous chunk frees the operand buffer while the
           // first half is computed
           if (hf == 0) ob = opbuf_acquire();
+          if (C::TOPS) {
+#pragma unroll
+            for (int q = 0; q < PX; ++q) {
+              const uint32_t w[3][4] = {
+                  {(vm[q][0] & 0x3F80u) | (vm[q][1] & 0x3F800000u), (vm[q][2] & 0x3F80u) | (vm[q][3] & 0x3F800000u),
+                   (vm[q][4] & 0x3F80u) | (vm[q][5] & 0x3F800000u), (vm[q][6] & 0x3F80u) | (vm[q][7] & 0x3F800000u)},
+                  {pack_hi16(ph[q][0], ph[q][1]), pack_hi16(ph[q][2], ph[q][3]), pack_hi16(ph[q][4], ph[q][5]),
+                   pack_hi16(ph[q][6], ph[q][7])},
+                  {pack_hi16(pl[q][0], pl[q][1]), pack_hi16(pl[q][2], pl[q][3]), pack_hi16(pl[q][4], pl[q][5]),
+                   pack_hi16(pl[q][6], pl[q][7])}};
+              tmem_ops(C::col_op1(opcnt & 1, q), hf, w);
+            }
+            continue;
+          }
           const uint32_t off = sm100::kmajor_off(tid, 8 * hf, 128);
 #pragma unroll
           for (int q = 0; q < PX; ++q) {
@@ -911,7 +971,7 @@ __global__ void __launch_bounds__(kTcThreads, TcShape<K>::CTAS)
 #pragma unroll
           for (int i = 0; i < K; ++i) b[i] = 0.f;
 #pragma unroll
-          for (int s = 0; s < 2; ++s) {
+          for (int s = 0; s < C::NSET; ++s) {
             if (s == 1 && nch < 2) break;
 #pragma unroll
             for (int j = 0; j < C::NGn / 16; ++j) {
@@ -1018,6 +1078,21 @@ __global__ void __launch_bounds__(kTcThreads, TcShape<K>::CTAS)
             vb[q] |= v8 << (8 * hf);
           }
           if (hf == 0) ob = opbuf_acquire();
+          if (C::TOPS) {
+            static_assert(!C::TOPS || kR0Parts == 3, "TMEM operands carry the 3-way r0 split");
+#pragma unroll
+            for (int q = 0; q < PX; ++q) {
+              const uint32_t w[3][4] = {
+                  {pack_hi16(rh[q][0], rh[q][1]), pack_hi16(rh[q][2], rh[q][3]), pack_hi16(rh[q][4], rh[q][5]),
+                   pack_hi16(rh[q][6], rh[q][7])},
+                  {pack_hi16(rm[q][0], rm[q][1]), pack_hi16(rm[q][2], rm[q][3]), pack_hi16(rm[q][4], rm[q][5]),
+                   pack_hi16(rm[q][6], rm[q][7])},
+                  {pack_hi16(rl[q][0], rl[q][1]), pack_hi16(rl[q][2], rl[q][3]), pack_hi16(rl[q][4], rl[q][5]),
+                   pack_hi16(rl[q][6], rl[q][7])}};
+              tmem_ops(C::col_op2(opcnt & 1, q), hf, w);
+            }
+            continue;
+          }
           const uint32_t off = sm100::kmajor_off(tid, 8 * hf, 128);
 #pragma unroll
           for (int q = 0; q < PX; ++q) {
