@@ -87,7 +87,7 @@ struct TcShape {
 #ifdef BFAST_UNROLL_SEED
   static constexpr int UNROLL_SEED = BFAST_UNROLL_SEED;
 #else
-  static constexpr int UNROLL_SEED = PX == 1 ? 2 : 1;  // measured per shape
+  static constexpr int UNROLL_SEED = 1;  // measured (2 was better before the TMEM operands)
 #endif
 };
 
@@ -423,11 +423,12 @@ __device__ __forceinline__ void mon_date_k(float y, float c0, float yh, float &W
 }
 // producer-side waits with back-off so a waiting producer does not steal
 // issue slots from the consumer warps of its SM sub-partition: MODE 0 =
-// try_wait with a suspend hint, 1 = poll, N > 1 = poll with an N-ns sleep.
-// Measured on the Landsat config (tools/ab_bench.sh): stack/table producers
-// 256 ns and the MMA issuer 32 ns are 8% faster than polling.
+// try_wait with a suspend hint, 1 = poll, N > 1 = poll with an N-ns sleep
+// (__nanosleep(N) sleeps ~2N ns).  Measured on the Landsat config
+// (tools/ab_bench.sh): producer 128 ns and MMA issuer 32 ns; polling and
+// suspended waits are slower, longer producer sleeps delay the stack boxes.
 #ifndef BFAST_AUX_WAIT
-#define BFAST_AUX_WAIT 256
+#define BFAST_AUX_WAIT 128
 #endif
 #ifndef BFAST_MMA_WAIT
 #define BFAST_MMA_WAIT 32
