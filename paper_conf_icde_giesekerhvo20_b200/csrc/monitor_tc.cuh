@@ -161,10 +161,12 @@ struct TcCfg {
     return c <= 32 ? 32 : c <= 64 ? 64 : c <= 128 ? 128 : c <= 256 ? 256 : 512;
   }
   // shared-memory operands: two accumulator sets; TMEM operands: one set and
-  // two operand buffers per pass, taken only where that fits the allocation
+  // two operand buffers per pass, taken where that fits the CTA's budget
   static constexpr int COLS_SMEM = pow2cols(2 * PX * SET > P2B ? 2 * PX * SET : P2B);
   static constexpr int P1T = PX * SET + 2 * PX * OPC, P2T = P2B + 2 * PX * OPC;
-  static constexpr bool TOPS = kTmemOpsWanted && pow2cols(P1T > P2T ? P1T : P2T) <= COLS_SMEM;
+  // (the TMEM budget per CTA: 128 columns at 4 CTAs/SM for PX = 1, 256 at 2)
+  static constexpr int TCAP = COLS_SMEM > 128 * PX ? COLS_SMEM : 128 * PX;
+  static constexpr bool TOPS = kTmemOpsWanted && pow2cols(P1T > P2T ? P1T : P2T) <= TCAP;
   static constexpr int NSET = TOPS ? 1 : 2;
   static constexpr int COLS_P1 = TOPS ? P1T : 2 * PX * SET;
   static constexpr __host__ __device__ int col_set(int s, int q) { return (s * PX + q) * SET; }
