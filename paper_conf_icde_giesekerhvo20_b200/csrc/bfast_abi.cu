@@ -430,7 +430,12 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
   const int rwarps = 4;
   const size_t rsmem = (size_t)rwarps * bfast::refit_warp_doubles((int)pl.N) * sizeof(double);
   if (rsmem > (size_t)kMaxSmem) return fail(BFAST_EUNSUPPORTED, "refit smem too large");
-  bfast::refit_fp64_kernel<K><<<sms * 8, rwarps * 32, rsmem, st>>>(prm);
+  // one resident wave: each warp walks its items with the next column in
+  // flight, so extra (waiting) blocks would only break that pipeline
+  int rblocks = 0;
+  CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&rblocks, bfast::refit_fp64_kernel<K>, rwarps * 32,
+                                                         rsmem));
+  bfast::refit_fp64_kernel<K><<<sms * std::max(rblocks, 1), rwarps * 32, rsmem, st>>>(prm);
   CUDA_TRY(cudaGetLastError());
   CUDA_TRY(cudaEventRecord(pl.scratch_free, st));
   g_launches = launches + 1;

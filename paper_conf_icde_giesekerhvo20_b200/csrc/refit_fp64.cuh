@@ -26,45 +26,55 @@ __device__ __forceinline__ double warp_sum(double v) {
   return v;
 }
 
-// shared memory per warp, in doubles: prefix sums [N + 1] + column [N] f32
-__host__ __device__ constexpr size_t refit_warp_doubles(int N) { return (size_t)(N + 1) + ((size_t)N + 1) / 2; }
+// shared memory per warp, in doubles: prefix sums [N + 1] + two column
+// buffers [N] f32 (the current pixel's and the next one's, in flight)
+__host__ __device__ constexpr size_t refit_warp_doubles(int N) { return (size_t)(N + 1) + (size_t)N; }
+
+// one 4-byte global -> shared copy through the LSU's asynchronous path
+// (cp.async, no register staging); completion tracked per thread by groups
+__device__ __forceinline__ void cp_async4(float *dst, const float *src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"((uint32_t)__cvta_generic_to_shared(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_prev() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
+
+// the pixel's column is N strided 4-byte reads (one DRAM burst each): every
+// lane issues its N/32 copies at once, straight into shared memory
+__device__ __forceinline__ void refit_fetch_column(float *Yc, const float *Y, int64_t pix, int N, int64_t ldY,
+                                                   int lane) {
+  const float *ycol = Y + pix;
+  for (int t = lane; t < N; t += 32) cp_async4(Yc + t, ycol + (int64_t)t * ldY);
+}
 
 template <int K>
 __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
-  // per warp: [N + 1] compacted residual prefix sums (fp64), then the
-  // pixel's column [N] (fp32), staged once so every pass reads shared memory
+  // per warp: [N + 1] compacted residual prefix sums (fp64), then two
+  // column buffers [N] (fp32): the column of item i is used while the
+  // column of item i + stride is being copied in (software pipeline over
+  // the warp's items, so only the first column's latency is exposed)
   extern __shared__ double rbuf_all[];
   const int lane = threadIdx.x & 31;
   const int wib = threadIdx.x >> 5;
   const int wpb = blockDim.x >> 5;
   double *S = rbuf_all + (size_t)wib * refit_warp_doubles(p.N);
-  float *Yc = reinterpret_cast<float *>(S + p.N + 1);
+  float *Ybuf = reinterpret_cast<float *>(S + p.N + 1);
   const int count = *p.refit_count;
   const int n = p.n, N = p.N;
   const int64_t ldY = p.ldY;
   const double qnan = __longlong_as_double(0x7ff8000000000000ll);
+  const int stride = gridDim.x * wpb;
 
-  for (int item = blockIdx.x * wpb + wib; item < count; item += gridDim.x * wpb) {
+  int item = blockIdx.x * wpb + wib;
+  if (item < count) refit_fetch_column(Ybuf, p.Y, p.refit_list[item], N, ldY, lane);
+  cp_async_commit();
+  for (int buf = 0; item < count; item += stride, buf ^= 1) {
     const int64_t pix = p.refit_list[item];  // absolute pixel index
-    {
-      // the column is N strided loads (one sector each): issue them all
-      // before any is used, so the pixel pays one memory latency, not N/32
-      const float *ycol = p.Y + pix;
-      float v4[4];
-      for (int t0 = 0; t0 < N; t0 += 128) {
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          const int t = t0 + 32 * u + lane;
-          v4[u] = t < N ? __ldcs(ycol + (int64_t)t * ldY) : 0.f;
-        }
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          const int t = t0 + 32 * u + lane;
-          if (t < N) Yc[t] = v4[u];
-        }
-      }
-      __syncwarp();
-    }
+    const int next = item + stride;
+    if (next < count) refit_fetch_column(Ybuf + (buf ^ 1) * N, p.Y, p.refit_list[next], N, ldY, lane);
+    cp_async_commit();
+    cp_async_wait_prev();  // this lane's copies of the current column landed
+    __syncwarp();          // ... and every other lane's
+    const float *Yc = Ybuf + buf * N;
     // ---- history: offset, Gram, moment (fp64)
     double A[Tri<K>::kN], b[K];
 #pragma unroll
