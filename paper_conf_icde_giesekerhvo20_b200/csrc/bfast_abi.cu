@@ -427,7 +427,10 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
     g_prof.emplace_back(e0, e1);
   }
   // fp64 refit of flagged pixels; exits at once when the list is empty
-  const int rwarps = 4;
+#ifndef BFAST_REFIT_WARPS
+#define BFAST_REFIT_WARPS 4
+#endif
+  const int rwarps = BFAST_REFIT_WARPS;
   const size_t rsmem = (size_t)rwarps * bfast::refit_warp_doubles((int)pl.N) * sizeof(double);
   if (rsmem > (size_t)kMaxSmem) return fail(BFAST_EUNSUPPORTED, "refit smem too large");
   // one resident wave: each warp walks its items with the next column in
