@@ -193,6 +193,25 @@ def test_landsat_full_size_sampled_parity(mode):
     torch.cuda.empty_cache()
 
 
+@pytest.mark.slow
+def test_landsat_every_refitted_pixel_matches_oracle(mode):
+    """configs[1] at full size: every pixel the fused kernel handed to the
+    fp64 refit (flags bit 1; ~0.1% of the scene, so each refit warp walks
+    several items with the next column in flight) against the oracle."""
+    spec = synth.CONFIGS["landsat"]
+    Y, dates = synth.generate(spec, DEV)
+    out = binding.bfast_monitor_ex(Y, dates, spec.n_hist, spec.k, spec.hf, spec.lam, diagnostics=True)
+    torch.cuda.synchronize()
+    it = torch.nonzero((out["flags"].to(torch.int32) & 2) != 0).flatten()
+    assert 1000 < it.numel() < spec.P // 100, it.numel()
+    Ys = Y.index_select(1, it).cpu().numpy()
+    orc = oracle.monitor(Ys, dates, spec.n_hist, spec.k, spec.hf, spec.lam)
+    gpu = {key: v.index_select(0, it).cpu().numpy() for key, v in out.items() if torch.is_tensor(v)}
+    _assert_parity(gpu, orc, dates, spec.n_hist, spec.k)
+    del Y
+    torch.cuda.empty_cache()
+
+
 def test_tc_and_simt_paths_agree_closely(monkeypatch):
     """The two kernels compute the same definitions with different fp32
     contraction orders: breaks equal up to near ties, magnitudes within the
