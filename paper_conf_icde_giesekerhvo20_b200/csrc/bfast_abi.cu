@@ -430,8 +430,10 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
 #ifndef BFAST_REFIT_WARPS
 #define BFAST_REFIT_WARPS 4
 #endif
-  const int rwarps = BFAST_REFIT_WARPS;
-  const size_t rsmem = (size_t)rwarps * bfast::refit_warp_doubles((int)pl.N) * sizeof(double);
+  int rwarps = BFAST_REFIT_WARPS;  // fewer warps per CTA where a long series needs the room
+  const size_t rwsmem = bfast::refit_warp_doubles((int)pl.N) * sizeof(double);
+  while (rwarps > 1 && (size_t)rwarps * rwsmem > (size_t)kMaxSmem) rwarps >>= 1;
+  const size_t rsmem = (size_t)rwarps * rwsmem;
   if (rsmem > (size_t)kMaxSmem) return fail(BFAST_EUNSUPPORTED, "refit smem too large");
   // one resident wave: each warp walks its items with the next column in
   // flight, so extra (waiting) blocks would only break that pipeline
@@ -629,7 +631,7 @@ int bfast_plan_create(bfast_plan **out, int device, int64_t N, const double *dat
   if (simt_smem(*pl, 32) > (size_t)kMaxSmem)
     return fail(BFAST_EUNSUPPORTED, "N=%lld with window %d exceeds shared memory", (long long)N,
                 pl->hcap);
-  if ((size_t)4 * (N + 1) * sizeof(double) > (size_t)kMaxSmem)
+  if (bfast::refit_warp_doubles((int)N) * sizeof(double) > (size_t)kMaxSmem)
     return fail(BFAST_EUNSUPPORTED, "N=%lld too large for the refit kernel", (long long)N);
   {
     const char *mode = std::getenv("BFAST_KERNEL");

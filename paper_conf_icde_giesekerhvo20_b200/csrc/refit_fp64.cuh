@@ -26,9 +26,12 @@ __device__ __forceinline__ double warp_sum(double v) {
   return v;
 }
 
-// shared memory per warp, in doubles: prefix sums [N + 1] + two column
-// buffers [N] f32 (the current pixel's and the next one's, in flight)
-__host__ __device__ constexpr size_t refit_warp_doubles(int N) { return (size_t)(N + 1) + (size_t)N; }
+// shared memory per warp, in doubles: prefix sums [N + 1], two column
+// buffers [N] f32 (the current pixel's and the next one's, in flight) and
+// the compacted date list Ic [N] u16
+__host__ __device__ constexpr size_t refit_warp_doubles(int N) {
+  return (size_t)(N + 1) + (size_t)N + ((size_t)N + 3) / 4;
+}
 
 // one 4-byte global -> shared copy through the LSU's asynchronous path
 // (cp.async, no register staging); completion tracked per thread by groups
@@ -58,6 +61,7 @@ __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
   const int wpb = blockDim.x >> 5;
   double *S = rbuf_all + (size_t)wib * refit_warp_doubles(p.N);
   float *Ybuf = reinterpret_cast<float *>(S + p.N + 1);
+  uint16_t *Ic = reinterpret_cast<uint16_t *>(Ybuf + 2 * p.N);
   const int count = *p.refit_count;
   const int n = p.n, N = p.N;
   const int64_t ldY = p.ldY;
@@ -75,40 +79,45 @@ __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
     cp_async_wait_prev();  // this lane's copies of the current column landed
     __syncwarp();          // ... and every other lane's
     const float *Yc = Ybuf + buf * N;
-    // ---- history: offset, Gram, moment (fp64)
+    // ---- order-preserving compaction (filterNaNsWKeys, L483-L490): Ic[c]
+    // = date of the c-th valid value, c < Nbar; the ranks are the popc
+    // prefix of the validity ballot, so every later loop runs over the
+    // N̄ valid dates only, all lanes busy
+    int cr = 0, nbar = 0;
+#pragma unroll 1
+    for (int t0 = 0; t0 < N; t0 += 32) {
+      const int t = t0 + lane;
+      const bool v = t < N && Yc[t] == Yc[t];
+      const unsigned bal = __ballot_sync(0xffffffffu, v);
+      if (v) Ic[cr + __popc(bal & ((1u << lane) - 1))] = (uint16_t)t;
+      if (t0 < n) nbar += __popc(bal & (t0 + 32 <= n ? 0xffffffffu : ((1u << (n - t0)) - 1u)));
+      cr += __popc(bal);
+    }
+    const int Nbar = cr;
+    __syncwarp();  // Ic is read across lanes below
+    // ---- history: offset c0 = first valid history value, Gram, moment (fp64)
     double A[Tri<K>::kN], b[K];
 #pragma unroll
     for (int i = 0; i < Tri<K>::kN; ++i) A[i] = 0.0;
 #pragma unroll
     for (int i = 0; i < K; ++i) b[i] = 0.0;
-    double c0 = 0.0;
-    bool have = false;
-    int nbar = 0;
+    const double c0 = nbar > 0 ? (double)Yc[Ic[0]] : 0.0;
     double ymax = 0.0;
-    for (int t0 = 0; t0 < n; t0 += 32) {
-      const int t = t0 + lane;
-      const float yf = t < n ? Yc[t] : __int_as_float(0x7fc00000);
-      const bool v = (yf == yf);
-      const unsigned bal = __ballot_sync(0xffffffffu, v);
-      if (!bal) continue;
-      if (!have) {
-        c0 = (double)__shfl_sync(0xffffffffu, yf, __ffs(bal) - 1);
-        have = true;
-      }
-      nbar += __popc(bal);
-      if (v) {
-        const double y = (double)yf - c0;
-        ymax = fmax(ymax, fabs((double)yf));
-        const double *x = p.X64 + (size_t)t * K;
-        double xr[K];
+#pragma unroll 1
+    for (int c = lane; c < nbar; c += 32) {
+      const int t = Ic[c];
+      const float yf = Yc[t];
+      const double y = (double)yf - c0;
+      ymax = fmax(ymax, fabs((double)yf));
+      const double *x = p.X64 + (size_t)t * K;
+      double xr[K];
 #pragma unroll
-        for (int i = 0; i < K; ++i) xr[i] = x[i];
+      for (int i = 0; i < K; ++i) xr[i] = x[i];
 #pragma unroll
-        for (int i = 0; i < K; ++i) {
+      for (int i = 0; i < K; ++i) {
 #pragma unroll
-          for (int j = i; j < K; ++j) A[Tri<K>::idx(i, j)] = fma(xr[i], xr[j], A[Tri<K>::idx(i, j)]);
-          b[i] = fma(y, xr[i], b[i]);
-        }
+        for (int j = i; j < K; ++j) A[Tri<K>::idx(i, j)] = fma(xr[i], xr[j], A[Tri<K>::idx(i, j)]);
+        b[i] = fma(y, xr[i], b[i]);
       }
     }
 #pragma unroll
@@ -124,40 +133,35 @@ __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
     const int h = window_h(nbar, p.hf);
     bool deg = !(minratio > 1e-9);  // rank test (reading R4)
 
-    // ---- residuals of all dates, compacted in order, as prefix sums S
+    // ---- residuals of the valid dates in compacted order, as prefix sums S
     double s2 = 0.0;
-    int cr = 0;
     if (lane == 0) S[0] = 0.0;
     __syncwarp();  // S[0] is read by every lane below
-    for (int t0 = 0; t0 < N; t0 += 32) {
-      const int t = t0 + lane;
-      const float yf = t < N ? Yc[t] : __int_as_float(0x7fc00000);
-      const bool v = (yf == yf);
-      const unsigned bal = __ballot_sync(0xffffffffu, v);
+#pragma unroll 1
+    for (int c0i = 0; c0i < Nbar; c0i += 32) {
+      const int c = c0i + lane;
       double r = 0.0;
-      if (v) {
+      if (c < Nbar) {
+        const int t = Ic[c];
         const double *x = p.X64 + (size_t)t * K;
         double yhat = 0.0;
 #pragma unroll
         for (int i = 0; i < K; ++i) yhat = fma(x[i], beta[i], yhat);
-        r = ((double)yf - c0) - yhat;
+        r = ((double)Yc[t] - c0) - yhat;
       }
-      if (t < n) s2 += r * r;
-      // inclusive warp scan of r over valid lanes (invalid lanes carry 0)
+      if (c < nbar) s2 += r * r;
+      // inclusive warp scan of r (lanes past N̄ carry 0)
       double sc = r;
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
         double up = __shfl_up_sync(0xffffffffu, sc, o);
         if (lane >= o) sc += up;
       }
-      const double base = S[cr];
+      const double base = S[c0i];
       __syncwarp();
-      const int rank = cr + __popc(bal & ((1u << lane) - 1));
-      if (v) S[rank + 1] = base + sc;
-      cr += __popc(bal);
+      if (c < Nbar) S[c + 1] = base + sc;
       __syncwarp();
     }
-    const int Nbar = cr;
     s2 = warp_sum(s2);
     const double sigma = sqrt(s2 / (double)(nbar - K));
     if (!(sigma > 1e-4 * ymax)) deg = true;
@@ -181,23 +185,7 @@ __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
     }
     msum = warp_sum(msum);
     // original date index of compacted rank nbar + jstar (REMAPINDICES)
-    int brk = -1;
-    if (jstar >= 0) {
-      int target = nbar + jstar, seen = 0;
-      for (int t0 = 0; t0 < N; t0 += 32) {
-        const int t = t0 + lane;
-        const float yf = t < N ? Yc[t] : __int_as_float(0x7fc00000);
-        const unsigned bal = __ballot_sync(0xffffffffu, yf == yf);
-        const int c = __popc(bal);
-        if (seen + c > target) {
-          unsigned bb = bal;
-          for (int q = 0; q < target - seen; ++q) bb &= bb - 1;
-          brk = t0 + __ffs(bb) - 1 - n;
-          break;
-        }
-        seen += c;
-      }
-    }
+    const int brk = jstar >= 0 ? (int)Ic[nbar + jstar] - n : -1;
     if (lane == 0) {
       p.out_break[pix] = deg ? -2 : brk;
       p.out_mag[pix] = deg ? (float)qnan : (float)(msum / (double)J);
