@@ -114,6 +114,26 @@ def test_edge_cases_degenerate_pixels(mode):
     assert gpu["break"][2] != -2 and gpu["break"][6] == -2 and gpu["break"][7] == 0
 
 
+@pytest.mark.parametrize("N", [1000, 3600])
+def test_refit_of_long_series(N, mode):
+    """Pixels pushed towards the fp64 refit (an offset of 20 under noise
+    0.01-0.05: the fp32 fit's cancellation triggers fire for a share of
+    them, none is degenerate by reading R4), on series long enough that the refit
+    CTA narrows to fit its per-warp buffers (N = 3600: 2 warps per CTA),
+    several per refit warp; compared with the oracle."""
+    spec = synth.StackSpec(P=65536, N=N, n_hist=N // 2, k=2, miss=0.5, seed=71)
+    Y, dates = synth.generate(spec, DEV)
+    Y[:, ::3] += 20.0                            # every third pixel
+    try:
+        gpu, orc = _run_both(Y, dates, spec.n_hist, spec.k, spec.hf, spec.lam)
+    except binding.BfastError as e:             # a series the fused kernels cannot hold
+        assert e.status == binding.BFAST_EUNSUPPORTED and N > 1000, str(e)
+        pytest.skip(str(e))
+    assert int(((gpu["flags"][::3] & 2) != 0).sum()) > spec.P // 60   # ~10% measured at N = 1000
+    assert int((gpu["break"][::3] == -2).sum()) == 0
+    _assert_parity(gpu, orc, dates, spec.n_hist, spec.k)
+
+
 def test_empty_input_is_a_noop():
     Y = torch.empty((10, 0), device=DEV)
     out = binding.bfast_monitor_ex(Y, synth.make_dates(10), 5, 1, 0.25, 1.65)
