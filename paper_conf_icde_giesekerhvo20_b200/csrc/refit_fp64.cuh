@@ -26,11 +26,15 @@ __device__ __forceinline__ double warp_sum(double v) {
   return v;
 }
 
-// shared memory per warp, in doubles: prefix sums [N + 1], two column
-// buffers [N] f32 (the current pixel's and the next one's, in flight) and
-// the compacted date list Ic [N] u16
+// shared memory per warp, in doubles: prefix sums [N + 1], kRefitBufs
+// column buffers [N] f32 (the current pixel's and the next ones', in
+// flight) and the compacted date list Ic [N] u16
+#ifndef BFAST_REFIT_BUFS
+#define BFAST_REFIT_BUFS 2
+#endif
+constexpr int kRefitBufs = BFAST_REFIT_BUFS;
 __host__ __device__ constexpr size_t refit_warp_doubles(int N) {
-  return (size_t)(N + 1) + (size_t)N + ((size_t)N + 3) / 4;
+  return (size_t)(N + 1) + ((size_t)kRefitBufs * N + 1) / 2 + ((size_t)N + 3) / 4;
 }
 
 // one 4-byte global -> shared copy through the LSU's asynchronous path
@@ -39,7 +43,9 @@ __device__ __forceinline__ void cp_async4(float *dst, const float *src) {
   asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"((uint32_t)__cvta_generic_to_shared(dst)), "l"(src) : "memory");
 }
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-__device__ __forceinline__ void cp_async_wait_prev() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_prev() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(kRefitBufs - 1) : "memory");
+}
 
 // the pixel's column is N strided 4-byte reads (one DRAM burst each): every
 // lane issues its N/32 copies at once, straight into shared memory
@@ -51,17 +57,17 @@ __device__ __forceinline__ void refit_fetch_column(float *Yc, const float *Y, in
 
 template <int K>
 __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
-  // per warp: [N + 1] compacted residual prefix sums (fp64), then two
-  // column buffers [N] (fp32): the column of item i is used while the
-  // column of item i + stride is being copied in (software pipeline over
-  // the warp's items, so only the first column's latency is exposed)
+  // per warp: [N + 1] compacted residual prefix sums (fp64), then
+  // kRefitBufs column buffers [N] (fp32): the column of item i is used
+  // while the columns of the next kRefitBufs - 1 items are being copied in
+  // (software pipeline over the warp's items), then the date list Ic
   extern __shared__ double rbuf_all[];
   const int lane = threadIdx.x & 31;
   const int wib = threadIdx.x >> 5;
   const int wpb = blockDim.x >> 5;
   double *S = rbuf_all + (size_t)wib * refit_warp_doubles(p.N);
   float *Ybuf = reinterpret_cast<float *>(S + p.N + 1);
-  uint16_t *Ic = reinterpret_cast<uint16_t *>(Ybuf + 2 * p.N);
+  uint16_t *Ic = reinterpret_cast<uint16_t *>(Ybuf + kRefitBufs * p.N);
   const int count = *p.refit_count;
   const int n = p.n, N = p.N;
   const int64_t ldY = p.ldY;
@@ -69,12 +75,19 @@ __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
   const int stride = gridDim.x * wpb;
 
   int item = blockIdx.x * wpb + wib;
-  if (item < count) refit_fetch_column(Ybuf, p.Y, p.refit_list[item], N, ldY, lane);
-  cp_async_commit();
-  for (int buf = 0; item < count; item += stride, buf ^= 1) {
+#pragma unroll
+  for (int q = 0; q < kRefitBufs - 1; ++q) {  // prologue: the first kRefitBufs - 1 columns
+    const int it = item + q * stride;
+    if (it < count) refit_fetch_column(Ybuf + q * N, p.Y, p.refit_list[it], N, ldY, lane);
+    cp_async_commit();
+  }
+  for (int buf = 0; item < count; item += stride, buf = buf + 1 == kRefitBufs ? 0 : buf + 1) {
     const int64_t pix = p.refit_list[item];  // absolute pixel index
-    const int next = item + stride;
-    if (next < count) refit_fetch_column(Ybuf + (buf ^ 1) * N, p.Y, p.refit_list[next], N, ldY, lane);
+    const int ahead = item + (kRefitBufs - 1) * stride;
+    // the buffer this column goes to was read by the previous item (whose
+    // trailing __syncwarp ordered those reads before these copies)
+    const int abuf = buf == 0 ? kRefitBufs - 1 : buf - 1;
+    if (ahead < count) refit_fetch_column(Ybuf + abuf * N, p.Y, p.refit_list[ahead], N, ldY, lane);
     cp_async_commit();
     cp_async_wait_prev();  // this lane's copies of the current column landed
     __syncwarp();          // ... and every other lane's
