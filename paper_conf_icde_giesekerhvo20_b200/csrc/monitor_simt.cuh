@@ -57,6 +57,9 @@ constexpr double kRefitRatio = 3e-2;   // worse conditioning -> fp64 refit
 // |m_j|/B_j within kTieTol of 1 at some j <= j* -> the break decision is
 // re-taken in fp64 by the refit kernel
 constexpr float kTieTol = 1e-4f;
+// reading R4: sigma-hat <= kSigmaTol * max|y_hist| is an exact fit
+// (fp64 rounding residue), decided in fp64 by the refit kernel only
+constexpr double kSigmaTol = 1e-10;
 
 __device__ __forceinline__ float ld_keep(const float *p) {
   // history values are read twice: keep them in L2 (default policy)
@@ -341,9 +344,9 @@ __global__ void __launch_bounds__(128, 4) monitor_simt_kernel(MonitorParams p) {
     // the residual sum: the fp32 sigma-hat is then unreliable -> fp64 refit
     if (!(lin <= 1e-2f * s2)) refit = true;
   }
-  if (!deg && !(sigma > 1e-4f * ymax)) deg = true;
   // noise within 2e-3 of the signal scale: fp32 fitted values (~1e-7 |y|)
-  // are no longer negligible next to sigma-hat -> fp64 refit (R12)
+  // are no longer negligible next to sigma-hat -> fp64 refit (R12), which
+  // also takes the sigma-hat ~ 0 decision of reading R4 in fp64
   if (!deg && !(sigma > 2e-3f * ymax)) refit = true;
   const float inv_scale = 1.0f / (sigma * sqrtf((float)nbar));
   // MOSUM seed: the last h-1 history residuals (ranks nbar-h+1 .. nbar-1),

@@ -1171,7 +1171,6 @@ __global__ void __launch_bounds__(kTcThreads, TcShape<K>::CTAS)
           refit[q] = true;
           BFAST_WHY(q, 0x20);
         }
-        if (!deg[q] && !(sigma[q] > 1e-4f * ymax[q])) deg[q] = true;
         // noise within 2e-3 of the signal scale: fp32 fitted values (~1e-7 |y|)
         // are no longer negligible next to sigma-hat -> fp64 refit (R12)
         if (!deg[q] && !(sigma[q] > 2e-3f * ymax[q])) {

@@ -177,7 +177,9 @@ __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
     }
     s2 = warp_sum(s2);
     const double sigma = sqrt(s2 / (double)(nbar - K));
-    if (!(sigma > 1e-4 * ymax)) deg = true;
+    // reading R4: sigma-hat at fp64 rounding level of an exact fit (the
+    // oracle's ORACLE_SIGMA_TOL rule; PAPER.md L515/L524 divide by it)
+    if (!(sigma > kSigmaTol * ymax)) deg = true;
     // ---- MOSUM by prefix differences, first break, mean
     const double scale = sigma * sqrt((double)nbar);
     double msum = 0.0;

@@ -55,6 +55,69 @@ def test_p1_worked_example(golden_dir):
     m = oracle.mosum(r, 3, 6, 2, exp["sigma"])
     np.testing.assert_allclose(m, exp["mosum"], rtol=1e-12)
     assert [oracle.boundary(1.5, 3, j) for j in range(3)] == exp["boundary"]
+    # the parity diagnostics (oracle/parity.py's excuse rules): max_j |m_j|/B_j
+    # over the whole monitoring period and the refined near-tie flag
+    assert out["max_ratio"][0] == pytest.approx(exp["max_ratio"], rel=1e-12)
+    assert out["near_tie"][0] == exp["near_tie"]
+
+
+def test_p9_near_tie_before_the_break():
+    """Hand-built pixel (P1's history and its last two monitoring values):
+    the first monitoring value is chosen so that m_0 = 1.49925, i.e.
+    |m_0|/B_0 = 0.9995, within 1e-3 of 1 but no break; m_1 then crosses
+    (j* = 1), m_2 is P1's -20.830952.  So near_tie = 1 (a tie at j = 0 <= j*)
+    while the literal rule's max ratio is P1's 13.887301, far from 1: the
+    pixel the refined rule excuses and the literal one does not.  A max taken
+    over j <= j* only would give |m_1|/1.5 = 2.54 instead."""
+    s14 = math.sqrt(3.0 / 14.0)                      # sigma sqrt(nbar) of P1
+    r_hist_last = -1.0 / 14.0                        # residual of rank 2 (t = 4)
+    r3 = 1.49925 * s14 - r_hist_last                 # m_0 = (r_2 + r_3) / s14
+    y6 = r3 + (-0.5 + 23.0 * 6.0 / 14.0)             # + yhat(6) of P1's fit
+    y = np.array([1.0, 3.0, np.nan, 6.0, np.nan, y6, 12.0, 2.0], np.float32)[:, None]
+    out = oracle.monitor(y, np.arange(1.0, 9.0), 4, 0, 0.75, 1.5)
+    assert out["near_tie"][0] == 1
+    assert out["break"][0] == 2                      # rank nbar + 1 -> t = 7 -> 6 - n
+    assert out["max_ratio"][0] == pytest.approx(135 * math.sqrt(14 / 3) / 21, rel=1e-12)
+    r3f = float(y[5, 0]) - (-0.5 + 23.0 * 6.0 / 14.0)   # the fp32 input's residual
+    m = np.array([r_hist_last + r3f, r3f + 1.0, 1.0 - 149.0 / 14.0]) / s14
+    assert abs(m[0]) / 1.5 == pytest.approx(0.9995, abs=1e-6)
+    assert out["magnitude"][0] == pytest.approx(m.mean(), rel=1e-9)
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_p9_max_ratio_and_near_tie_brute_force(seed):
+    """max_ratio / near_tie against a brute-force recomputation on tiny
+    inputs where the boundary is NOT flat (n = N/4, 60% missing: (nbar+1+j)/
+    nbar passes e): numpy lstsq residuals, direct window sums, and the
+    boundary of the P2 table (lambda sqrt(max(1, ln x)), pinned there)."""
+    rng = np.random.default_rng(90 + seed)
+    N, n, k, P, hf, lam = 64, 16, 1, 48, 0.5, 0.9
+    Y, dates = _rand_stack(rng, N, P, k, miss=0.6, noise=0.05)
+    out = oracle.monitor(Y, dates, n, k, hf, lam)
+    X = _design(dates, k)
+    checked = flat = 0
+    for p in range(P):
+        if out["deg_reason"][p] != 0:
+            continue
+        ok = ~np.isnan(Y[:, p])
+        I = np.nonzero(ok)[0]
+        nbar = int((I < n).sum())
+        beta = np.linalg.lstsq(X[I[:nbar]], Y[I[:nbar], p].astype(np.float64), rcond=None)[0]
+        r = Y[I, p].astype(np.float64) - X[I] @ beta
+        sig = math.sqrt((r[:nbar] ** 2).sum() / (nbar - X.shape[1]))
+        h = int(np.float32(nbar) * np.float32(hf))
+        J = len(I) - nbar
+        m = np.array([r[nbar + j - h + 1: nbar + j + 1].sum() for j in range(J)]) / (sig * math.sqrt(nbar))
+        x = (nbar + 1 + np.arange(J)) / nbar
+        B = lam * np.sqrt(np.maximum(1.0, np.log(x)))
+        flat += int((x > math.e).any())
+        ratio = np.abs(m) / B
+        hit = np.nonzero(np.abs(m) > B)[0]
+        jstar = hit[0] if hit.size else J - 1
+        assert out["max_ratio"][p] == pytest.approx(ratio.max(), rel=1e-6)
+        assert out["near_tie"][p] == int((np.abs(ratio[:jstar + 1] - 1) <= 1e-3).any())
+        checked += 1
+    assert checked >= 20 and flat >= 10
 
 
 # ---------------------------------------------------------------- P2
@@ -273,8 +336,13 @@ def test_p7_degenerate_table():
     y = clean.copy(); y[:n][4:] = np.nan; add(y, 1)          # nbar = K
     y = clean.copy(); y[:n][5:] = np.nan; add(y, 0)          # nbar = K+1, h = 1
     y = clean.copy(); y[n:] = np.nan; add(y, 3)              # no monitoring data
-    exact = (X @ np.array([0.25, 0.0, 0.125, 0.0])).astype(np.float32)
-    add(exact, 5)                                            # noise-free: sigma ~ 0
+    # an exact fit: the constant 0.5 is in the model, sigma-hat is fp64
+    # rounding residue (reading R4: <= 1e-10 max|y| -> invalid)
+    add(np.full(N, 0.5, np.float32), 5)
+    # noise-free but fp32-rounded: sigma-hat ~ 3e-8 max|y| is a value, the
+    # pixel is valid (R4 is a rule on exactness, not on fp32 resolution)
+    rounded = (X @ np.array([0.25, 0.0, 0.125, 0.0])).astype(np.float32)
+    add(rounded, 0)
     # rank deficiency: valid history dates congruent mod 23 -> sin/cos constant
     N2 = 23 * 12
     dates2 = 2000.0 + np.arange(1, N2 + 1) / 23.0
@@ -287,6 +355,9 @@ def test_p7_degenerate_table():
     Y = np.stack(cols, axis=1)
     out = oracle.monitor(Y, dates, n, k, 0.25, 1.65)
     assert list(out["deg_reason"]) == want
+    ymax = float(np.nanmax(np.abs(rounded[:n])))
+    assert out["sigma"][4] <= 1e-10 * 0.5
+    assert 1e-9 * ymax < out["sigma"][5] < 1e-6 * ymax
     for i, w in enumerate(want):
         if w:
             assert out["break"][i] == -2 and np.isnan(out["magnitude"][i])
