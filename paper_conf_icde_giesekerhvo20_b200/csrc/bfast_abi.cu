@@ -20,6 +20,7 @@
 #include "../../include/bfast.h"
 #include "monitor_simt.cuh"
 #include "monitor_tc.cuh"
+#include "monitor_fused.cuh"
 #include "refit_fp64.cuh"
 
 namespace {
@@ -89,14 +90,17 @@ struct bfast_plan {
   float *dX = nullptr;      // [N][KP] fp32
   double *dX64 = nullptr;   // [N][K] fp64
   int32_t *dcount = nullptr;
-  int32_t *dlist = nullptr;
+  int64_t *dlist = nullptr;
   int64_t list_cap = 0;
   cudaEvent_t scratch_free = nullptr;  // orders executions sharing the refit scratch
   // tensor-core path: per-chunk B-operand tables (monitor_tc.cuh)
   uint8_t *dtab = nullptr;
   size_t tab2_off = 0, taby_off = 0;
+  // fused kernel (monitor_fused.cuh): per-chunk tables of passes A, B, C
+  uint8_t *dtabf = nullptr;
+  size_t tabfB_off = 0, tabfC_off = 0;
   int nch = 0, ncm = 0;
-  int mode = 0;  // 0 auto, 1 force SIMT, 2 force tensor cores (BFAST_KERNEL env at plan creation)
+  int mode = 0;  // 0 auto (fused), 1 SIMT, 2 round-1 tensor-core kernel (BFAST_KERNEL=simt|tc1 at plan creation)
   std::mutex mu;
   ~bfast_plan() {
     int prev = -1;
@@ -107,6 +111,7 @@ struct bfast_plan {
     cudaFree(dcount);
     cudaFree(dlist);
     cudaFree(dtab);
+    cudaFree(dtabf);
     if (scratch_free) cudaEventDestroy(scratch_free);
     if (prev >= 0) cudaSetDevice(prev);
   }
@@ -157,12 +162,12 @@ PFN_encodeTiled get_encode() {
 
 // Tensor map of the stack range [p0, p0+P) x [0, N): box `pix` px x 16 dates
 // (one tile), out-of-bounds elements read as NaN (= missing).
-bool make_stack_map(CUtensorMap *m, const float *Y, int64_t ldY, int64_t P, int64_t N, int pix) {
+bool make_stack_map(CUtensorMap *m, const float *Y, int64_t ldY, int64_t P, int64_t N, int pix, int dates = 16) {
   PFN_encodeTiled enc = get_encode();
   if (!enc) return false;
   cuuint64_t dims[2] = {(cuuint64_t)P, (cuuint64_t)N};
   cuuint64_t strides[1] = {(cuuint64_t)ldY * sizeof(float)};
-  cuuint32_t box[2] = {(cuuint32_t)pix, 16};
+  cuuint32_t box[2] = {(cuuint32_t)pix, (cuuint32_t)dates};
   cuuint32_t es[2] = {1, 1};
   return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void *)Y, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
              CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -303,8 +308,190 @@ int build_tc(bfast_plan &pl) {
   return BFAST_OK;
 }
 
+// Chunk tables of the fused kernel (monitor_fused.cuh), B operands in the
+// canonical K-major layout, fp64 values split into bf16 parts:
+//   A[c] (history chunk c, pass A): F_hi | F_mid | F_lo ([NGn x 16] each;
+//        row q = moment function f_q, the last one the constant 1; column d
+//        = date 16c + d) | x_hi | x_mid ([KBn x 16] each, the first moment);
+//   B[c] (history chunk c, pass B): the yhat table [16 x KY] (row d = date;
+//        K index = 6 blocks of K: x_hi | x_mid | x_lo | x_hi | x_mid | x_hi,
+//        paired in the GEMM with beta hi | hi | hi | mid | mid | lo) | x_hi |
+//        x_mid | x_lo ([KBn x 16] each, the refinement moment);
+//   C[c] (monitoring chunk c): the yhat table of dates n + 16c + d.
+template <int K>
+void build_fz_tables(const bfast_plan &pl, std::vector<uint16_t> &tab, size_t &offB, size_t &offC) {
+  using C = bfast::FzCfg<K>;
+  const int k = pl.k, n = pl.n, N = (int)pl.N, DC = C::DC;
+  const int nch = (n + DC - 1) / DC, ncm = (N - n + DC - 1) / DC;
+  const double two_pi = 6.283185307179586476925286766559;
+  auto xrow = [&](int t, double *x) {
+    const double tau = ((double)(t + 1) - pl.tc) / pl.ts, th = two_pi * pl.dates[t];
+    x[0] = 1.0;
+    x[1] = tau;
+    for (int j = 1; j <= k; ++j) {
+      x[2 * j] = std::sin(j * th);
+      x[2 * j + 1] = std::cos(j * th);
+    }
+  };
+  auto frow = [&](int t, double *f) {  // tau, tau^2, tau sin_j, tau cos_j, sin_m, cos_m, 1
+    const double tau = ((double)(t + 1) - pl.tc) / pl.ts, th = two_pi * pl.dates[t];
+    f[0] = tau;
+    f[1] = tau * tau;
+    for (int j = 1; j <= k; ++j) {
+      f[2 + 2 * (j - 1)] = tau * std::sin(j * th);
+      f[3 + 2 * (j - 1)] = tau * std::cos(j * th);
+    }
+    for (int m = 1; m <= 2 * k; ++m) {
+      f[2 + 2 * k + 2 * (m - 1)] = std::sin(m * th);
+      f[3 + 2 * k + 2 * (m - 1)] = std::cos(m * th);
+    }
+    f[C::NF] = 1.0;  // the constant function: its masked moment is nbar
+  };
+  const size_t TA = C::TABA / 2, TB = C::TABB / 2, TC = C::TABC / 2;
+  tab.assign((size_t)nch * (TA + TB) + (size_t)ncm * TC, 0);
+  offB = (size_t)nch * TA;
+  offC = offB + (size_t)nch * TB;
+  double x[2 + 2 * BFAST_K_MAX_HARMONICS], f[3 + 6 * BFAST_K_MAX_HARMONICS];
+  auto put_b3 = [&](uint16_t *b3, int d, const double *xv) {  // [16 x KY]: xh|xm|xl|xh|xm|xh
+    for (int i = 0; i < K; ++i) {
+      uint16_t h, m, l;
+      split3(xv[i], h, m, l);
+      const uint16_t blk[6] = {h, m, l, h, m, h};
+      for (int b = 0; b < 6; ++b) b3[kmaj(d, b * K + i, C::DC)] = blk[b];
+    }
+  };
+  auto put_bx = [&](uint16_t *bx, int d, const double *xv, int parts) {  // parts x [KBn x 16]
+    for (int i = 0; i < K; ++i) {
+      uint16_t h, m, l;
+      split3(xv[i], h, m, l);
+      const uint16_t prt[3] = {h, m, l};
+      for (int e = 0; e < parts; ++e) bx[e * C::BX_BYTES / 2 + kmaj(i, d, C::KBn)] = prt[e];
+    }
+  };
+  for (int c = 0; c < nch; ++c) {
+    uint16_t *ta = tab.data() + (size_t)c * TA;
+    uint16_t *tb = tab.data() + offB + (size_t)c * TB;
+    for (int d = 0; d < DC; ++d) {
+      const int t = c * DC + d;
+      if (t >= n) continue;
+      xrow(t, x);
+      frow(t, f);
+      for (int q = 0; q <= C::NF; ++q) {
+        uint16_t h, m, l;
+        split3(f[q], h, m, l);
+        const uint16_t prt[3] = {h, m, l};
+        for (int e = 0; e < 3; ++e) ta[e * C::BF_BYTES / 2 + kmaj(q, d, C::NGn)] = prt[e];
+      }
+      put_bx(ta + 3 * C::BF_BYTES / 2, d, x, 2);
+      put_b3(tb, d, x);
+      put_bx(tb + C::B3_BYTES / 2, d, x, 3);
+    }
+  }
+  for (int c = 0; c < ncm; ++c) {
+    uint16_t *tcp = tab.data() + offC + (size_t)c * TC;
+    for (int d = 0; d < DC; ++d) {
+      const int t = n + c * DC + d;
+      if (t >= N) continue;
+      xrow(t, x);
+      put_b3(tcp, d, x);
+    }
+  }
+}
+
+int build_fz(bfast_plan &pl) {
+  std::vector<uint16_t> tab;
+  size_t ob = 0, oc = 0;
+  switch (pl.k) {
+    case 0: build_fz_tables<2>(pl, tab, ob, oc); break;
+    case 1: build_fz_tables<4>(pl, tab, ob, oc); break;
+    case 2: build_fz_tables<6>(pl, tab, ob, oc); break;
+    case 3: build_fz_tables<8>(pl, tab, ob, oc); break;
+    case 4: build_fz_tables<10>(pl, tab, ob, oc); break;
+    case 5: build_fz_tables<12>(pl, tab, ob, oc); break;
+    case 6: build_fz_tables<14>(pl, tab, ob, oc); break;
+    default: return BFAST_EUNSUPPORTED;
+  }
+  pl.tabfB_off = ob * 2;
+  pl.tabfC_off = oc * 2;
+  CUDA_TRY(cudaMalloc(&pl.dtabf, tab.size() * 2));
+  CUDA_TRY(cudaMemcpy(pl.dtabf, tab.data(), tab.size() * 2, cudaMemcpyHostToDevice));
+  return BFAST_OK;
+}
+
 size_t simt_smem(const bfast_plan &pl, int bp) {
   return (size_t)pl.N * pl.KP * sizeof(float) + (size_t)pl.hcap * bp * (sizeof(float) + sizeof(int16_t));
+}
+
+// The fused kernel (monitor_fused.cuh): T tiles of 128 pixels per CTA, the
+// largest T whose shared memory fits (the MOSUM ring grows with the window
+// hcap = floor(hf * n)), as many CTAs per SM as shared memory, TMEM and
+// registers admit, and a persistent grid over the tile groups.
+// Returns BFAST_OK with `done` = false when the stack cannot be read by TMA
+// (row pitch not a multiple of 16 bytes): the caller falls back to SIMT.
+template <int K>
+int launch_fused(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t st, bool &done) {
+  using C = bfast::FzCfg<K>;
+  done = false;
+  static thread_local int configured_dev = -1;
+  cudaFuncAttributes fa{};
+  CUDA_TRY(cudaFuncGetAttributes(&fa, bfast::monitor_fused_kernel<K>));
+  const int static_smem = (int)fa.sharedSizeBytes;
+  if (configured_dev != pl.device) {
+    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_fused_kernel<K>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  kMaxSmem - static_smem));
+    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_fused_kernel<K>, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                  (int)cudaSharedmemCarveoutMaxShared));
+    configured_dev = pl.device;
+  }
+  if (!pl.dtabf || (prm.ldY % 4) != 0 || ((uintptr_t)(prm.Y + prm.p0) % 16) != 0) return BFAST_OK;
+  // tiles per CTA and stack stages: the most tiles that fit with 3 stack
+  // stages, else with 2
+  int T = C::TMAX, sc = C::SCMAX;
+  if (const char *e = std::getenv("BFAST_FZ_T")) T = std::max(1, std::min(C::TMAX, std::atoi(e)));
+  if (const char *e = std::getenv("BFAST_FZ_SC")) sc = std::max(2, std::min(C::SCMAX, std::atoi(e)));
+  auto fits = [&](int t, int c) { return C::smem_bytes(t, pl.hcap, c) + static_smem <= (size_t)kMaxSmem; };
+  while (T > 1 && !fits(T, 2)) --T;
+  if (!fits(T, sc)) sc = 2;
+  const size_t smem = C::smem_bytes(T, pl.hcap, sc);
+  if (smem + static_smem > (size_t)kMaxSmem)
+    return fail(BFAST_EUNSUPPORTED, "fused kernel: shared memory %zu B for window %d", smem, pl.hcap);
+  int sms = 148;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, pl.device);
+  // CTAs per SM: shared memory (228 KB per SM, 1 KB reserved per CTA), TMEM
+  // (512 columns), registers, threads
+  const int threads = 128 * (T + 1);  // T consumer warpgroups + the control warpgroup
+  const int by_smem = (int)(kSmemPerSM / (smem + static_smem + 1024));
+  const int by_tmem = 512 / C::pow2cols(T * C::TCOLS);
+  const int by_regs = 65536 / (threads * std::max(fa.numRegs, 1));
+  const int by_thr = 2048 / threads;
+  const int per_sm = std::max(1, std::min(std::min(by_smem, by_tmem), std::min(by_regs, by_thr)));
+  // full stack; history only (dates >= n out of bounds -> NaN); L2 prefetch boxes
+  CUtensorMap ymap, hmap, pmap;
+  if (!make_stack_map(&ymap, prm.Y + prm.p0, prm.ldY, prm.P, pl.N, 128, 16) ||
+      !make_stack_map(&hmap, prm.Y + prm.p0, prm.ldY, prm.P, pl.n, 128, 16) ||
+      !make_stack_map(&pmap, prm.Y + prm.p0, prm.ldY, prm.P, pl.N, 128, C::PFB))
+    return BFAST_OK;
+  int pfd = 128;
+  if (const char *e = std::getenv("BFAST_FZ_PFD")) pfd = std::max(0, std::atoi(e)) / C::PFB * C::PFB;
+  bfast::FzTables tb;
+  tb.tabA = pl.dtabf;
+  tb.tabB = pl.dtabf + pl.tabfB_off;
+  tb.tabC = pl.dtabf + pl.tabfC_off;
+  tb.nch = pl.nch;
+  tb.ncm = pl.ncm;
+  tb.T = T;
+  tb.hcap = pl.hcap;
+  tb.pfd = pfd;
+  tb.sc = sc;
+  tb.ntg = (prm.P + 128 * T - 1) / (128 * T);
+  const int64_t grid = std::min<int64_t>(tb.ntg, (int64_t)sms * per_sm);
+  if (std::getenv("BFAST_VERBOSE"))
+    std::fprintf(stderr, "bfast: fused k=%d T=%d sc=%d smem=%zu+%d regs=%d per_sm=%d grid=%lld tile groups=%lld\n",
+                 pl.k, T, sc, smem, static_smem, fa.numRegs, per_sm, (long long)grid, (long long)tb.ntg);
+  bfast::monitor_fused_kernel<K><<<(unsigned)grid, threads, smem, st>>>(prm, tb, ymap, hmap, pmap);
+  CUDA_TRY(cudaGetLastError());
+  done = true;
+  return BFAST_OK;
 }
 
 template <int K>
@@ -378,7 +565,7 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
   if (std::getenv("BFAST_VERBOSE"))
     std::fprintf(stderr, "bfast: tc layout k=%d hcap=%d nch=%d sy=%d nop=%d smem=%zu per_sm=%d tmem_cols=%d\n", pl.k,
                  tc_hcap, pl.nch, tc_sy, tc_nop, tc_smem, per_sm, TC::TMEM_COLS);
-  const bool tc_ok = per_sm > 0 && pl.dtab && pl.mode != 1 && (prm.ldY % 4) == 0 &&
+  const bool tc_ok = per_sm > 0 && pl.dtab && pl.mode == 2 && (prm.ldY % 4) == 0 &&
                      ((uintptr_t)(prm.Y + prm.p0) % 16) == 0 && tc_smem + 1024 <= (size_t)kMaxSmem;
   CUtensorMap ymap, hmap;  // full stack; history only (dates >= n out of bounds)
   const bool tma_ok = tc_ok && make_stack_map(&ymap, prm.Y + prm.p0, prm.ldY, prm.P, pl.N, TC::PIX) &&
@@ -394,6 +581,12 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
     CUDA_TRY(cudaEventRecord(e0, st));
   }
   int launches = 0;
+  bool fused = false;
+  if (pl.mode == 0) {
+    const int rc = launch_fused<K>(pl, prm, st, fused);
+    if (rc) return rc;
+    launches += fused ? 1 : 0;
+  }
   if (ntiles > 0) {
     bfast::TcTables tb;
     tb.tab1 = pl.dtab;
@@ -411,10 +604,10 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
     CUDA_TRY(cudaGetLastError());
     ++launches;
   }
-  const int64_t rest = ntiles > 0 ? 0 : prm.P;
+  // SIMT kernel: forced (BFAST_KERNEL=simt) or a stack TMA cannot read
+  const int64_t rest = (fused || ntiles > 0) ? 0 : prm.P;
   if (rest > 0) {
     bfast::MonitorParams q = prm;
-    q.p0 = prm.p0 + ntiles * 128;
     q.P = rest;
     const int64_t blocks = (rest + bp - 1) / bp;
     if (blocks > 0x7fffffff) return fail(BFAST_EUNSUPPORTED, "P too large");
@@ -466,7 +659,7 @@ std::vector<std::unique_ptr<bfast_plan>> g_cache;
 
 int env_mode() {
   const char *m = std::getenv("BFAST_KERNEL");
-  return !m ? 0 : (std::strcmp(m, "simt") == 0 ? 1 : std::strcmp(m, "tc") == 0 ? 2 : 0);
+  return !m ? 0 : (std::strcmp(m, "simt") == 0 ? 1 : std::strcmp(m, "tc1") == 0 ? 2 : 0);
 }
 
 bool same_plan(const bfast_plan &pl, int dev, int64_t N, const double *dates, int32_t n, int32_t k,
@@ -497,16 +690,33 @@ int ensure_list(bfast_plan &pl, int64_t P) {
   cudaFree(pl.dlist);
   pl.dlist = nullptr;
   pl.list_cap = 0;
-  CUDA_TRY(cudaMalloc(&pl.dlist, sizeof(int32_t) * (size_t)std::max<int64_t>(P, 1)));
+  CUDA_TRY(cudaMalloc(&pl.dlist, sizeof(int64_t) * (size_t)std::max<int64_t>(P, 1)));
   pl.list_cap = P;
   return BFAST_OK;
 }
+
+// Pixel ranges of at most 2^30 pixels per launch set: TMA box coordinates
+// and the kernels' tile arithmetic are 32-bit.
+constexpr int64_t kMaxLaunchPixels = (int64_t)1 << 30;
+
+int execute_one(bfast_plan &pl, const bfast_args *a, int64_t p0, int64_t P);
 
 int execute_range(bfast_plan &pl, const bfast_args *a, int64_t p0, int64_t P) {
   if (P == 0) {
     g_launches = 0;
     return BFAST_OK;
   }
+  int total = 0;
+  for (int64_t b = 0; b < P; b += kMaxLaunchPixels) {
+    const int rc = execute_one(pl, a, p0 + b, std::min(kMaxLaunchPixels, P - b));
+    if (rc) return rc;
+    total += g_launches;
+  }
+  g_launches = total;
+  return BFAST_OK;
+}
+
+int execute_one(bfast_plan &pl, const bfast_args *a, int64_t p0, int64_t P) {
   int rc = ensure_list(pl, P);
   if (rc) return rc;
   bfast::MonitorParams prm{};
@@ -550,6 +760,18 @@ int validate_args(const bfast_args *a) {
 }  // namespace
 
 extern "C" {
+
+#ifdef BFAST_FZ_TIMING
+// diagnostics build only: the fused kernel's cycle accounting (copied, then reset)
+int bfast_debug_fz_timing(unsigned long long *out, int n) {
+  unsigned long long h[16] = {0};
+  CUDA_TRY(cudaMemcpyFromSymbol(h, bfast::fz_timing, sizeof h));
+  const unsigned long long z[16] = {0};
+  CUDA_TRY(cudaMemcpyToSymbol(bfast::fz_timing, z, sizeof z));
+  for (int i = 0; i < n && i < 16; ++i) out[i] = h[i];
+  return BFAST_OK;
+}
+#endif
 
 int bfast_abi_version(void) { return BFAST_ABI_VERSION; }
 
@@ -635,7 +857,7 @@ int bfast_plan_create(bfast_plan **out, int device, int64_t N, const double *dat
     return fail(BFAST_EUNSUPPORTED, "N=%lld too large for the refit kernel", (long long)N);
   {
     const char *mode = std::getenv("BFAST_KERNEL");
-    pl->mode = !mode ? 0 : (std::strcmp(mode, "simt") == 0 ? 1 : std::strcmp(mode, "tc") == 0 ? 2 : 0);
+    pl->mode = !mode ? 0 : (std::strcmp(mode, "simt") == 0 ? 1 : std::strcmp(mode, "tc1") == 0 ? 2 : 0);
   }
   std::vector<float> X;
   std::vector<double> X64;
@@ -652,7 +874,10 @@ int bfast_plan_create(bfast_plan **out, int device, int64_t N, const double *dat
   if (e == cudaSuccess) e = cudaMemset(pl->dcount, 0, sizeof(int32_t));
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&pl->scratch_free, cudaEventDisableTiming);
   int trc = BFAST_OK;
-  if (e == cudaSuccess && pl->mode != 1 && N <= 32767) trc = build_tc(*pl);
+  if (e == cudaSuccess && pl->mode == 2 && N <= 32767) trc = build_tc(*pl);
+  if (e == cudaSuccess && trc == BFAST_OK && pl->mode == 0) trc = build_fz(*pl);
+  pl->nch = (n_hist + 15) / 16;
+  pl->ncm = ((int)N - n_hist + 15) / 16;
   cudaSetDevice(prev);
   if (trc != BFAST_OK) return trc;
   if (e != cudaSuccess)

@@ -48,7 +48,7 @@ struct MonitorParams {
   float *out_mag, *out_beta, *out_sigma;
   int32_t *out_nbar;
   uint8_t *out_flags;
-  int32_t *refit_list;
+  int64_t *refit_list;   // absolute pixel indices (int64: P may exceed 2^31 across launches)
   int32_t *refit_count;
 };
 
@@ -440,7 +440,7 @@ __global__ void __launch_bounds__(128, 4) monitor_simt_kernel(MonitorParams p) {
     int base = 0;
     if (lane == leader) base = atomicAdd(p.refit_count, __popc(mask));
     base = __shfl_sync(mask, base, leader);
-    p.refit_list[base + __popc(mask & ((1u << lane) - 1))] = (int32_t)pix;
+    p.refit_list[base + __popc(mask & ((1u << lane) - 1))] = pix;
   }
 }
 

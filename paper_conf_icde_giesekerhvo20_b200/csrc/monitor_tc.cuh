@@ -1427,7 +1427,7 @@ __global__ void __launch_bounds__(kTcThreads, TcShape<K>::CTAS)
           int base = 0;
           if (lane == leader) base = atomicAdd(p.refit_count, __popc(mask));
           base = __shfl_sync(mask, base, leader);
-          p.refit_list[base + __popc(mask & ((1u << lane) - 1))] = (int32_t)(pix0 + q);
+          p.refit_list[base + __popc(mask & ((1u << lane) - 1))] = pix0 + q;
         }
       }
     }
