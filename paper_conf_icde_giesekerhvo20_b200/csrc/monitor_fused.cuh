@@ -87,10 +87,12 @@ struct FzCfg {
   // operand buffers [mask 8 | y' hi 8 | y' lo 8].  Passes B/C: NYS yhat slots |
   // beta operand | db | one operand buffer [r0 hi 8 | mid 8 | lo 8].  The pass-B
   // layout overwrites pass A's only after the solve has read it.
+  static constexpr int NOPA = 3;  // pass-A operand buffers (the consumers run NOPA - 1 chunks ahead of the MMA)
   static constexpr int cG = 0, cB = NGn, cOPA = NGn + KBn;
-  static constexpr int PA_COLS = cOPA + 48;
+  static constexpr int PA_COLS = cOPA + 24 * NOPA;
   static constexpr int NYS = 3;  // yhat slots: yhat(c + 3) is issued when chunk c is published
   static_assert(NYS <= 3, "the publish barriers (pub[g % 4]) allow NYS outstanding groups");
+  static_assert(NOPA <= 3, "the publish barriers (pub[g % 4]) allow NOPA outstanding groups");
   static constexpr int cY = 0, cA3 = 16 * NYS, cDB = cA3 + KY / 2, cOPB = cDB + KBn;
   static constexpr int PB_COLS = cOPB + 24;  // one r0 operand buffer
   static constexpr int USED = PA_COLS > PB_COLS ? PA_COLS : PB_COLS;
@@ -115,7 +117,7 @@ struct FzCfg {
 #ifdef BFAST_FZ_ST
   static constexpr int ST = BFAST_FZ_ST;
 #else
-  static constexpr int ST = 5;                   // table stages (lookahead ST - 1 chunks)
+  static constexpr int ST = 6;                   // table stages (a stage is reloaded two chunks after its use)
 #endif
   static constexpr int PFB = 64;                 // dates per L2-prefetch box
   static constexpr int SCMAX = 3;                // stack chunk stages per tile (2 or 3, by shared memory)
@@ -433,7 +435,9 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
   // the tile's 4 warps published group g (on [g%4]: in pass C the consumers
   // may run NYS groups ahead of the control warp, so a parity pair would alias)
   __shared__ __align__(8) uint64_t pub[C::TMAX][4];
-  __shared__ __align__(8) uint64_t mdone[C::TMAX][2];       // tile's group g completes phase g/2 of mdone[g%2]
+  // tile's group g completes phase g/4 of mdone[g%4] (waiters look up to 3
+  // groups back: NOPA = 3 operand buffers)
+  __shared__ __align__(8) uint64_t mdone[C::TMAX][4];
   __shared__ __align__(8) uint64_t ybar[C::TMAX][C::NYS];  // tile's yhat slot s written (one phase per yhat)
   __shared__ __align__(8) uint64_t tfull[C::ST];            // table stages
   __shared__ uint32_t tfree[C::ST];                         // tiles done with a table stage (mod T)
@@ -483,7 +487,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
         sm100::mbar_init(&srel[i][j], 4);
       }
       for (int j = 0; j < 4; ++j) sm100::mbar_init(&pub[i][j], 4);
-      for (int j = 0; j < 2; ++j) sm100::mbar_init(&mdone[i][j], 1);
+      for (int j = 0; j < 4; ++j) sm100::mbar_init(&mdone[i][j], 1);
       for (int j = 0; j < C::NYS; ++j) sm100::mbar_init(&ybar[i][j], 1);
     }
     for (int i = 0; i < C::ST; ++i) {
@@ -636,6 +640,8 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
       const uint32_t idY = sm100::idesc_bf16_f32(128, C::DC);
       uint32_t g = 0;
       int cslot = 0;  // yhat slot of the current B / C chunk
+      int abuf = 0;   // pass-A operand buffer of the current A chunk
+      uint32_t gch1 = 0, gch2 = 0;  // group indices of the previous two chunk groups
       auto tstage = [&](const ChunkPos &cp) -> uint32_t { return a_tabs + (uint32_t)cp.st * C::TSTAGE; };
       auto wait_table = [&](const ChunkPos &cp) {
         FZT_T0(tt)
@@ -660,10 +666,14 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
         FZT_ADD(5, tp)
         FZT_T0(ti)
         sm100::tc_fence_after();
+        // group g commits to the barrier of group g - 4: observe that phase
+        // first (it completed long ago; every phase gets a waiter)
+        if (g >= 4) wait_sleep(a_mdone + 8 * ((g - 4) & 3), ((g - 4) >> 2) & 1u);
         if (kind == 0) {
           wait_table(cpos);
           sm100::tc_fence_after();
-          const uint32_t bf = tstage(cpos), bx = bf + 3 * C::BF_BYTES, at = tc + C::cOPA + 24 * (c & 1);
+          const uint32_t bf = tstage(cpos), bx = bf + 3 * C::BF_BYTES, at = tc + C::cOPA + 24 * abuf;
+          if (++abuf == C::NOPA) abuf = 0;
 #pragma unroll
           for (int e = 0; e < 3; ++e)
             sm100::umma_bf16_ts_e(tc + C::cG, at, sm100::smem_desc(bf + e * C::BF_BYTES, C::NGn * 16, 128), idG,
@@ -691,28 +701,33 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
               sm100::umma_bf16_ts_e(tc + C::cDB, at + 8 * e,
                                     sm100::smem_desc(bx + xx * C::BX_BYTES, C::KBn * 16, 128), idB,
                                     (c > 0 || e > 0 || xx > 0) ? 1u : 0u);
-          sm100::umma_commit_e(a_mdone + 8 * (g & 1));
+          sm100::umma_commit_e(a_mdone + 8 * (g & 3));
           if (c + C::NYS < nch) issue_yhat(advance_pos(cpos, C::NYS), cslot);
         } else {
           if (c + C::NYS < ncm) issue_yhat(advance_pos(cpos, C::NYS), cslot);
         }
         if (kind == 2 || kind == 4)
           if (++cslot == C::NYS) cslot = 0;
-        if (kind != 2) sm100::umma_commit_e(a_mdone + 8 * (g & 1));
+        if (kind != 2) sm100::umma_commit_e(a_mdone + 8 * (g & 3));
         if (kind == 0 || kind == 2 || kind == 4) {
-          if (cpos.s > 0) {
-            // this tile is done with the table stage of chunk s - 1 once its
-            // group g - 1 has completed; the last of the T tiles reloads it
+          if (cpos.s > 1) {
+            // this tile is done with the table stage of chunk s - 2 (its
+            // group completed two events ago: the wait is a formality); the
+            // last of the T tiles reloads it with chunk s - 2 + ST
             FZT_T0(tm)
-            wait_sleep(a_mdone + 8 * ((g - 1) & 1), ((g - 1) >> 1) & 1u);
+            wait_sleep(a_mdone + 8 * (gch2 & 3), (gch2 >> 2) & 1u);
             FZT_ADD(13, tm)
-            const ChunkPos nxt = advance_pos(cpos, C::ST - 1);  // chunk s - 1 + ST, the stage of s - 1
+            const ChunkPos nxt = advance_pos(cpos, C::ST - 2);
             if (lane == 0) {
               const uint32_t old = atom_add_acqrel(a_tfree + 4 * nxt.st, 1u);
-              if (old % (uint32_t)T == (uint32_t)T - 1) load_table(nxt);
+              const bool last = T == 4 ? (old & 3u) == 3u : T == 2 ? (old & 1u) == 1u : T == 1 ? true
+                                                                                           : old % 3u == 2u;
+              if (last) load_table(nxt);
             }
             __syncwarp();
           }
+          gch2 = gch1;
+          gch1 = g;
           cpos = advance_pos(cpos, 1);
         }
         ++g;
@@ -735,7 +750,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
         }
       }
       // the MMAs of the last groups complete before the CTA releases TMEM
-      if (g > 0) wait_sleep(a_mdone + 8 * ((g - 1) & 1), ((g - 1) >> 1) & 1u);
+      if (g > 0) wait_sleep(a_mdone + 8 * ((g - 1) & 3), ((g - 1) >> 2) & 1u);
     }
     FZT_ADD(8, t_kernel)
     FZT_FLUSH
@@ -775,7 +790,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
   };
   uint32_t g = 0;  // group sequence
   auto wait_group = [&](uint32_t gg) {  // group gg's MMAs have completed
-    mbar_wait_spin(a_mdone + 8 * (gg & 1), (gg >> 1) & 1);
+    mbar_wait_spin(a_mdone + 8 * (gg & 3), (gg >> 2) & 1);
     sm100::tc_fence_after();
   };
   // this warp's part of group g is done (its TMEM stores waited / loads
@@ -798,6 +813,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
   const float qnan = __int_as_float(0x7fc00000);
   const uint32_t rbase = sm100::opaque(sm100::smem_u32(ring) + (uint32_t)tile * hcap * 512 + 4 * (tid & 127));
 
+  int abuf = 0;  // pass-A operand buffer of the current chunk
   for (int64_t tg = blockIdx.x; tg < tb.ntg; tg += gridDim.x) {
     const int64_t pix = p.p0 + tg * (int64_t)T * 128 + ctid;
     // ================= pass A: masked Gram and moment on the tensor cores
@@ -838,7 +854,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
         }
       }
       FZT_T0(tw)
-      if (g >= 2) wait_group(g - 2);  // operand buffer c & 1 free
+      if (g >= C::NOPA) wait_group(g - C::NOPA);  // operand buffer abuf free
       FZT_ADD(0, tw)
       {
         uint32_t w16[16], w8[8];
@@ -846,8 +862,9 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
         for (int i = 0; i < 16; ++i) w16[i] = w[i];
 #pragma unroll
         for (int i = 0; i < 8; ++i) w8[i] = w[16 + i];
-        tmem_st16(lanebase + C::cOPA + 24 * (c & 1), w16);
-        sm100::tmem_st8(lanebase + C::cOPA + 24 * (c & 1) + 16, w8);
+        tmem_st16(lanebase + C::cOPA + 24 * abuf, w16);
+        sm100::tmem_st8(lanebase + C::cOPA + 24 * abuf + 16, w8);
+        if (++abuf == C::NOPA) abuf = 0;
       }
       sm100::tmem_st_wait();
       publish();
@@ -1144,57 +1161,65 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
     ys = 0;
     for (int c = 0; c < ncm; ++c) {
       wait_yhat(ys);  // yhat of this chunk
+      float yh[16];
+      sm100::tmem_ld16(lanebase + C::cY + 16 * ys, yh);
       const int crm = __reduce_max_sync(0xffffffffu, deg ? 0 : cr - nbar);
       const bool fast = crm + C::DC <= rank_flat_min;
       const uint32_t ya = acquire_chunk();
-#pragma unroll 1
-      for (int hf = 0; hf < 2; ++hf) {
-        float yh[8];
-        sm100::tmem_ld8(lanebase + C::cY + 16 * ys + 8 * hf, yh);
-        sm100::tmem_ld_wait();
-        if (hf == 1) publish();  // the slot is read: yhat of chunk c + 2 may overwrite it
-        float yv[8];
-        load8(ya, hf, yv);
-        float wv[8];
-        if (fast && ring8) {
-          // B_j == lambda here: the first |m| > lambda (1 - tol) decides; the
-          // dates track max |W| and W at each valid date, a half whose max
-          // crossed is scanned for its first crossing
+      sm100::tmem_ld_wait();
+      publish();  // the slot is read: yhat of chunk c + NYS may overwrite it
+      if (++ys == C::NYS) ys = 0;
+      if (fast && ring8) {
+        // B_j == lambda here: the first |m| > lambda (1 - tol) decides; the
+        // dates track max |W| and W at each valid date, a chunk whose max
+        // crossed is scanned for its first crossing
+        float wv[16];
+#pragma unroll
+        for (int hf = 0; hf < 2; ++hf) {
+          float yv[8];
+          load8(ya, hf, yv);
           uint32_t kk = 0;
           const uint32_t jw = (rend - wa) >> 9;
 #pragma unroll
-          for (int d = 0; d < 8; ++d) fc_date_k(yv[d], c0, yh[d], W, msum, mx, kk, wa, jw, hbytes, wv[d]);
-          if (hf == 1) release_chunk();
+          for (int d = 0; d < 8; ++d)
+            fc_date_k(yv[d], c0, yh[8 * hf + d], W, msum, mx, kk, wa, jw, hbytes, wv[8 * hf + d]);
           cr += (int)kk;
           const uint32_t a = wa + kk * 512;
           wa = a >= rend ? a - hbytes : a;
-          if (mx > thr_lo) {  // first < 0 while thr_lo is finite
-            int fd = 7;
-            float fw = wv[7];
+        }
+        release_chunk();
+        if (mx > thr_lo) {  // first < 0 while thr_lo is finite
+          int fd = 15;
+          float fw = wv[15];
 #pragma unroll
-            for (int d = 6; d >= 0; --d)
-              if (fabsf(wv[d]) > thr_lo) {
-                fd = d;
-                fw = wv[d];
-              }
-            first = c * C::DC + 8 * hf + fd;
-            mfirst = fw;
-            thr_lo = __int_as_float(0x7f800000);
-          }
-        } else {
+          for (int d = 14; d >= 0; --d)
+            if (fabsf(wv[d]) > thr_lo) {
+              fd = d;
+              fw = wv[d];
+            }
+          first = c * C::DC + fd;
+          mfirst = fw;
+          thr_lo = __int_as_float(0x7f800000);
+        }
+      } else {
+#pragma unroll 1
+        for (int hf = 0; hf < 2; ++hf) {
+          float yv[8], yq[8], wv[8];
+          load8(ya, hf, yv);
+#pragma unroll
+          for (int d = 0; d < 8; ++d) yq[d] = hf ? yh[8 + d] : yh[d];
 #pragma unroll
           for (int d = 0; d < 8; ++d) {
-            fc_date_1(yv[d], c0, yh[d], W, msum, mx, cr, wa, rend, hbytes, wv[d]);
+            fc_date_1(yv[d], c0, yq[d], W, msum, mx, cr, wa, rend, hbytes, wv[d]);
             if (wv[d] == wv[d] && brk < 0 && !tie && first < 0 && fabsf(W) > thr_lo) {
               const int code = fz_boundary_rare(W * inv_scale, cr, nbar, lam);
               tie = tie || (code >> 1);
               brk = (code & 1) ? c * C::DC + 8 * hf + d : brk;
             }
           }
-          if (hf == 1) release_chunk();
         }
+        release_chunk();
       }
-      if (++ys == C::NYS) ys = 0;
       if (first >= 0 && brk < 0 && !tie) {  // resolve a fast-path candidate
         if (fabsf(mfirst * inv_scale) > lam * (1.0f + kTieTol)) brk = first;
         else tie = true;
