@@ -287,7 +287,7 @@ def run_sharded_tile(args, spec, desc, world, rank, local, dev):
                        "slab_pixels": slab, "l2": "inputs larger than L2, no flush",
                        "parallelism": f"dp{world}: pixel shards of one tile, no collective"},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": None, "kernel": "monitor_tc_kernel<8>",
+                         "frac": achieved / peak, "traffic": None, "kernel": "monitor_fused_kernel<8>",
                          "kernel_ms_avg": kernel_ms, "peak_source": peak_src},
             "gpu_launches": launches, "clocks": sampler.summary()}
     return _finish(line, world, rank)
@@ -429,7 +429,7 @@ def main():
     workload_key = f"{args.config}:P={P}:N={N}:k={rspec.k}"
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": achieved / peak, "traffic": ncu_traffic(workload_key),
-                "kernel": "monitor_tc_kernel<8> (+SIMT tail)", "kernel_ms_avg": k_avg,
+                "kernel": "monitor_fused_kernel<8>", "kernel_ms_avg": k_avg,
                 "kernel_share_of_step": k_avg / ms_step if ms_step else None,
                 "alg_bytes_per_launch": alg_bytes, "peak_source": peak_src}
 

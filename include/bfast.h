@@ -154,7 +154,10 @@ int bfast_plan_execute(const bfast_plan *plan, const bfast_args *a);
 void bfast_plan_destroy(bfast_plan *plan);
 
 /*
- * bfast_monitor_host -- end-to-end form on HOST buffers.  Y_host is
+ * bfast_monitor_host -- end-to-end form on HOST buffers.  The device
+ * slabs, streams and events it pipelines with belong to the device's
+ * cached plan and are reused by later calls (a stream of tiles allocates
+ * once).  Y_host is
  * float32 [N][ldY] (pinned memory gives full PCIe bandwidth; pageable
  * memory works but is slower); out_break_host int32[P] and
  * out_magnitude_host float32[P] are host arrays.  The call uploads the
@@ -179,6 +182,45 @@ int bfast_monitor_multi(const float *Y_host, int64_t N, int64_t P, int64_t ldY,
                         const double *dates, int32_t n_hist, int32_t k, float h,
                         float lambda, const int *devices, int ndev,
                         int32_t *out_break_host, float *out_magnitude_host);
+
+/*
+ * bfast_monitor_shards -- device-resident pixel shards on several devices,
+ * gathered into ONE output map (pixels are independent,
+ * L142, so the only exchange is the break map).  Shard i is the stack
+ * Y_dev[i] (device pointer on devices[i], float32 [N][ldY[i]] with P[i]
+ * pixels, layout as in bfast_args); its results land at offset
+ * P[0] + ... + P[i-1] of out_break / out_magnitude, which are device
+ * arrays on `gather_device`.  Each shard's kernel stores its outputs
+ * straight into the gather device's memory (peer access over NVLink,
+ * enabled by the call): the gather is the epilogue's stores, no copy
+ * afterwards.  One host thread per shard, each with its device's cached
+ * plan; synchronous.  Several shards may live on the same device.
+ * Errors: BFAST_EINVAL for a bad shard description (nothing written);
+ * BFAST_ECUDA if peer access between a shard device and gather_device is
+ * impossible.
+ */
+int bfast_monitor_shards(const float *const *Y_dev, const int64_t *P, const int64_t *ldY,
+                         const int *devices, int nshards, int64_t N, const double *dates,
+                         int32_t n_hist, int32_t k, float h, float lambda, int gather_device,
+                         int32_t *out_break, float *out_magnitude);
+
+/*
+ * Cross-process break-map gather (one process per GPU, torchrun): the
+ * process owning the map exports its device allocation as a CUDA IPC
+ * handle of BFAST_IPC_HANDLE_BYTES bytes; every other process opens it and
+ * passes the mapped pointer (plus its shard offset) as out_break /
+ * out_magnitude of bfast_plan_execute, so each rank's kernel writes its
+ * slice of the map directly into the owner's GPU memory.  The handle
+ * carries no synchronisation: the ranks order their writes before the
+ * owner's reads with a barrier (bench.py, tests/test_multi_ipc.py).
+ * bfast_ipc_open maps on `device` (< 0: current); bfast_ipc_close unmaps.
+ * The exporting allocation must come from cudaMalloc (e.g. a torch
+ * tensor's storage base) and outlive every mapping.
+ */
+#define BFAST_IPC_HANDLE_BYTES 72 /* CUDA IPC handle of the allocation + byte offset */
+int bfast_ipc_export(const void *dev_ptr, unsigned char *handle);
+int bfast_ipc_open(const unsigned char *handle, int device, void **dev_ptr);
+int bfast_ipc_close(void *dev_ptr);
 
 /* Host-side helper (no CUDA): the [begin, end) pixel range of shard
    `rank` of `world` for P pixels, aligned to 128-pixel tiles. */

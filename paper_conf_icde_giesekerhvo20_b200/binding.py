@@ -26,10 +26,12 @@ K_MAX_HARMONICS = 6
 
 # names declared in include/bfast.h (checked by tests/test_abi.py)
 EXPORTS = ("bfast_monitor", "bfast_monitor_ex", "bfast_plan_create", "bfast_plan_execute",
-           "bfast_plan_destroy", "bfast_monitor_host", "bfast_monitor_multi",
+           "bfast_plan_destroy", "bfast_monitor_host", "bfast_monitor_multi", "bfast_monitor_shards",
+           "bfast_ipc_export", "bfast_ipc_open", "bfast_ipc_close",
            "bfast_shard_range", "bfast_last_launch_count", "bfast_last_error",
            "bfast_status_string", "bfast_abi_version", "bfast_profile_enable",
            "bfast_profile_collect")
+IPC_HANDLE_BYTES = 72
 
 
 class BfastError(RuntimeError):
@@ -70,6 +72,14 @@ def lib():
         L.bfast_monitor_host.restype = I
         L.bfast_monitor_multi.argtypes = [V, i64, i64, i64, V, i32, i32, f32, f32, V, I, V, V]
         L.bfast_monitor_multi.restype = I
+        L.bfast_monitor_shards.argtypes = [V, V, V, V, I, i64, V, i32, i32, f32, f32, I, V, V]
+        L.bfast_monitor_shards.restype = I
+        L.bfast_ipc_export.argtypes = [V, V]
+        L.bfast_ipc_export.restype = I
+        L.bfast_ipc_open.argtypes = [V, I, ctypes.POINTER(V)]
+        L.bfast_ipc_open.restype = I
+        L.bfast_ipc_close.argtypes = [V]
+        L.bfast_ipc_close.restype = I
         L.bfast_shard_range.argtypes = [i64, I, I, ctypes.POINTER(i64), ctypes.POINTER(i64)]
         L.bfast_shard_range.restype = None
         L.bfast_last_launch_count.restype = I
@@ -98,6 +108,8 @@ def _dates(dates) -> np.ndarray:
 def _dptr(t) -> Optional[int]:
     if t is None:
         return None
+    if isinstance(t, int):  # a raw device pointer (IPC-mapped output)
+        return t
     return int(t.data_ptr())
 
 
@@ -176,6 +188,18 @@ def _check_stack(Y):
         raise TypeError("Y must be a CUDA float32 [N][P] tensor with unit column stride")
 
 
+def _check_out(out, Y, P):
+    """Every output tensor on Y's device with at least P (x K) elements: the
+    library writes through raw pointers."""
+    for name, t in out.items():
+        if name.startswith("_") or t is None:
+            continue
+        if not t.is_cuda or t.device != Y.device:
+            raise ValueError(f"output {name!r} is on {t.device}, the stack on {Y.device}")
+        if t.shape[0] < P or not t.is_contiguous():
+            raise ValueError(f"output {name!r} must be contiguous with >= {P} rows")
+
+
 def bfast_monitor(Y, dates, n_hist, k, h, lam, out_break=None, out_magnitude=None):
     """North-star entry (synchronous).  Y: CUDA float32 [N][P] contiguous."""
     _check_stack(Y)
@@ -193,15 +217,19 @@ def bfast_monitor(Y, dates, n_hist, k, h, lam, out_break=None, out_magnitude=Non
 
 def bfast_monitor_ex(Y, dates, n_hist, k, h, lam, P=None, diagnostics=False, stream=None, out=None):
     """Asynchronous extended entry on `stream` (default: torch's current
-    stream).  Y may be a [N][ldY] view with P <= ldY columns used."""
+    stream of Y's device).  Y may be a [N][ldY] view with P <= ldY columns
+    used.  The call runs on Y's device (the library uses the current one)."""
+    import torch
     _check_stack(Y)
     P = int(Y.shape[1]) if P is None else int(P)
     out = out if out is not None else _outputs(Y, P, k, diagnostics)
+    _check_out(out, Y, P)
     d = _dates(dates)
-    a = _make_args(Y, d, n_hist, k, h, lam, out["break"], out["magnitude"], P=P,
-                   out_beta=out.get("beta"), out_sigma=out.get("sigma"), out_nbar=out.get("nbar"),
-                   out_flags=out.get("flags"), stream=stream)
-    _check(lib().bfast_monitor_ex(ctypes.byref(a)))
+    with torch.cuda.device(Y.device):
+        a = _make_args(Y, d, n_hist, k, h, lam, out["break"], out["magnitude"], P=P,
+                       out_beta=out.get("beta"), out_sigma=out.get("sigma"), out_nbar=out.get("nbar"),
+                       out_flags=out.get("flags"), stream=stream)
+        _check(lib().bfast_monitor_ex(ctypes.byref(a)))
     out["_dates_keepalive"] = d
     return out
 
@@ -217,14 +245,23 @@ class Plan:
         _check(lib().bfast_plan_create(ctypes.byref(self._h), self.device, self.N, self.dates.ctypes.data,
                                        self.n_hist, self.k, self.hf, self.lam))
 
-    def execute(self, Y, P=None, diagnostics=False, stream=None, out=None):
+    def execute(self, Y, P=None, diagnostics=False, stream=None, out=None, check_out=True):
+        """check_out=False: the output dict may hold raw pointers ({"break":
+        int, "magnitude": int}), e.g. an IPC-mapped slice of another
+        process's break map (ipc_open)."""
+        import torch
         _check_stack(Y)
+        if Y.device.index != self.device:
+            raise ValueError(f"the plan is on cuda:{self.device}, the stack on {Y.device}")
         P = int(Y.shape[1]) if P is None else int(P)
         out = out if out is not None else _outputs(Y, P, self.k, diagnostics)
-        a = _make_args(Y, self.dates, self.n_hist, self.k, self.hf, self.lam, out["break"],
-                       out["magnitude"], P=P, out_beta=out.get("beta"), out_sigma=out.get("sigma"),
-                       out_nbar=out.get("nbar"), out_flags=out.get("flags"), stream=stream)
-        _check(lib().bfast_plan_execute(self._h, ctypes.byref(a)))
+        if check_out:
+            _check_out(out, Y, P)
+        with torch.cuda.device(Y.device):
+            a = _make_args(Y, self.dates, self.n_hist, self.k, self.hf, self.lam, out["break"],
+                           out["magnitude"], P=P, out_beta=out.get("beta"), out_sigma=out.get("sigma"),
+                           out_nbar=out.get("nbar"), out_flags=out.get("flags"), stream=stream)
+            _check(lib().bfast_plan_execute(self._h, ctypes.byref(a)))
         return out
 
     def close(self):
@@ -278,3 +315,51 @@ def bfast_monitor_multi(Y_host, dates, n_hist, k, h, lam, devices, out_break=Non
                                      float(h), float(lam), ctypes.cast(devs, ctypes.c_void_p),
                                      len(devices), _host_ptr(out_break), _host_ptr(out_magnitude)))
     return out_break, out_magnitude
+
+
+def bfast_monitor_shards(shards, dates, n_hist, k, h, lam, gather_device, out_break=None, out_magnitude=None):
+    """Device-resident shards -> one break map on `gather_device` (each
+    shard's kernel stores straight into it over peer access).  shards: list
+    of CUDA float32 [N][ldY] tensors (any devices, unit column stride)."""
+    import torch
+    for Y in shards:
+        _check_stack(Y)
+    N = int(shards[0].shape[0])
+    Ps = [int(Y.shape[1]) for Y in shards]
+    total = sum(Ps)
+    gdev = torch.device("cuda", int(gather_device))
+    if out_break is None:
+        out_break = torch.empty(total, dtype=torch.int32, device=gdev)
+    if out_magnitude is None:
+        out_magnitude = torch.empty(total, dtype=torch.float32, device=gdev)
+    n = len(shards)
+    ys = (ctypes.c_void_p * n)(*[Y.data_ptr() for Y in shards])
+    ps = (ctypes.c_int64 * n)(*Ps)
+    lds = (ctypes.c_int64 * n)(*[int(Y.stride(0)) for Y in shards])
+    devs = (ctypes.c_int * n)(*[Y.device.index for Y in shards])
+    d = _dates(dates)
+    _check(lib().bfast_monitor_shards(ctypes.cast(ys, ctypes.c_void_p), ctypes.cast(ps, ctypes.c_void_p),
+                                      ctypes.cast(lds, ctypes.c_void_p), ctypes.cast(devs, ctypes.c_void_p), n,
+                                      N, d.ctypes.data, int(n_hist), int(k), float(h), float(lam),
+                                      int(gather_device), _dptr(out_break), _dptr(out_magnitude)))
+    return out_break, out_magnitude
+
+
+def ipc_export(t) -> bytes:
+    """IPC handle of tensor t's device memory (the CUDA handle of the
+    allocation containing it plus t's offset in that allocation)."""
+    buf = (ctypes.c_ubyte * IPC_HANDLE_BYTES)()
+    _check(lib().bfast_ipc_export(ctypes.c_void_p(t.data_ptr()), ctypes.cast(buf, ctypes.c_void_p)))
+    return bytes(buf)
+
+
+def ipc_open(handle: bytes, device: int = -1) -> int:
+    """Map another process's exported allocation; returns the device pointer."""
+    buf = (ctypes.c_ubyte * IPC_HANDLE_BYTES).from_buffer_copy(handle)
+    ptr = ctypes.c_void_p()
+    _check(lib().bfast_ipc_open(ctypes.cast(buf, ctypes.c_void_p), int(device), ctypes.byref(ptr)))
+    return int(ptr.value)
+
+
+def ipc_close(ptr: int):
+    _check(lib().bfast_ipc_close(ctypes.c_void_p(ptr)))

@@ -6,6 +6,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <map>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -19,7 +20,6 @@
 
 #include "../../include/bfast.h"
 #include "monitor_simt.cuh"
-#include "monitor_tc.cuh"
 #include "monitor_fused.cuh"
 #include "refit_fp64.cuh"
 
@@ -93,14 +93,22 @@ struct bfast_plan {
   int64_t *dlist = nullptr;
   int64_t list_cap = 0;
   cudaEvent_t scratch_free = nullptr;  // orders executions sharing the refit scratch
-  // tensor-core path: per-chunk B-operand tables (monitor_tc.cuh)
-  uint8_t *dtab = nullptr;
-  size_t tab2_off = 0, taby_off = 0;
+  // bfast_monitor_host: double-buffered device slabs, a copy and a compute
+  // stream, and their events, owned by the plan and reused across calls
+  // (allocated on first use, grown when a call needs a wider slab)
+  struct HostPath {
+    int64_t slab = 0;
+    float *dY[2] = {nullptr, nullptr};
+    int32_t *dB[2] = {nullptr, nullptr};
+    float *dM[2] = {nullptr, nullptr};
+    cudaStream_t cs = nullptr, ks = nullptr;
+    cudaEvent_t loaded[2] = {nullptr, nullptr}, done[2] = {nullptr, nullptr};
+  } host;
   // fused kernel (monitor_fused.cuh): per-chunk tables of passes A, B, C
   uint8_t *dtabf = nullptr;
   size_t tabfB_off = 0, tabfC_off = 0;
   int nch = 0, ncm = 0;
-  int mode = 0;  // 0 auto (fused), 1 SIMT, 2 round-1 tensor-core kernel (BFAST_KERNEL=simt|tc1 at plan creation)
+  int mode = 0;  // 0 fused tensor-core kernel, 1 SIMT kernel only (BFAST_KERNEL=simt at plan creation)
   std::mutex mu;
   ~bfast_plan() {
     int prev = -1;
@@ -110,9 +118,17 @@ struct bfast_plan {
     cudaFree(dX64);
     cudaFree(dcount);
     cudaFree(dlist);
-    cudaFree(dtab);
     cudaFree(dtabf);
     if (scratch_free) cudaEventDestroy(scratch_free);
+    for (int i = 0; i < 2; ++i) {
+      cudaFree(host.dY[i]);
+      cudaFree(host.dB[i]);
+      cudaFree(host.dM[i]);
+      if (host.loaded[i]) cudaEventDestroy(host.loaded[i]);
+      if (host.done[i]) cudaEventDestroy(host.done[i]);
+    }
+    if (host.cs) cudaStreamDestroy(host.cs);
+    if (host.ks) cudaStreamDestroy(host.ks);
     if (prev >= 0) cudaSetDevice(prev);
   }
 };
@@ -194,119 +210,6 @@ void split3(double v, uint16_t &h, uint16_t &m, uint16_t &l) {
   l = bf16_rne(v - bf16_val(h) - bf16_val(m));
 }
 inline size_t kmaj(int row, int k, int rows) { return sm100::kmajor_off(row, k, rows) / 2; }
-
-// Chunk tables of the tensor-core kernel (monitor_tc.cuh): B operands in the
-// canonical K-major layout, fp64 values split into bf16 parts.
-//   tab1[c] (history chunk c, pass 1): F_hi | F_mid | F_lo ([NGn x 16] each,
-//           row q = moment function f_q (the last one the constant 1),
-//           column d = date 16c + d), then x_hi | x_mid ([KBn x 16]
-//           each, row i = basis column i; x_lo is only needed in pass 2);
-//   tab2[c] (history chunk c, pass 2): the yhat table [16 x KY] of its dates
-//           (row d = date, K index = 6 blocks of K: x_hi | x_mid | x_lo |
-//           x_hi | x_mid | x_hi, paired in the GEMM with beta hi | hi | hi |
-//           mid | mid | lo), then x_hi | x_mid | x_lo as in tab1;
-//   taby[c] (monitoring chunk c): the yhat table of dates n + 16c + d.
-template <int K>
-void build_tc_tables(const bfast_plan &pl, std::vector<uint16_t> &tab, size_t &off2, size_t &offy) {
-  using C = bfast::TcCfg<K>;
-  const int k = pl.k, n = pl.n, N = (int)pl.N, DC = C::DC;
-  const int nch = (n + DC - 1) / DC, ncm = (N - n + DC - 1) / DC;
-  const double two_pi = 6.283185307179586476925286766559;
-  auto xrow = [&](int t, double *x) {
-    const double tau = ((double)(t + 1) - pl.tc) / pl.ts, th = two_pi * pl.dates[t];
-    x[0] = 1.0;
-    x[1] = tau;
-    for (int j = 1; j <= k; ++j) {
-      x[2 * j] = std::sin(j * th);
-      x[2 * j + 1] = std::cos(j * th);
-    }
-  };
-  auto frow = [&](int t, double *f) {  // tau, tau^2, tau sin_j, tau cos_j, sin_m, cos_m, 1
-    const double tau = ((double)(t + 1) - pl.tc) / pl.ts, th = two_pi * pl.dates[t];
-    f[0] = tau;
-    f[1] = tau * tau;
-    for (int j = 1; j <= k; ++j) {
-      f[2 + 2 * (j - 1)] = tau * std::sin(j * th);
-      f[3 + 2 * (j - 1)] = tau * std::cos(j * th);
-    }
-    for (int m = 1; m <= 2 * k; ++m) {
-      f[2 + 2 * k + 2 * (m - 1)] = std::sin(m * th);
-      f[3 + 2 * k + 2 * (m - 1)] = std::cos(m * th);
-    }
-    f[C::NF] = 1.0;  // the constant function: its masked moment is nbar
-  };
-  const size_t T1 = C::TAB1 / 2, T2 = C::TAB2 / 2, TY = C::TABY / 2;
-  tab.assign((size_t)nch * (T1 + T2) + (size_t)ncm * TY, 0);
-  off2 = (size_t)nch * T1;
-  offy = off2 + (size_t)nch * T2;
-  double x[2 + 2 * BFAST_K_MAX_HARMONICS], f[3 + 6 * BFAST_K_MAX_HARMONICS];
-  auto put_b3 = [&](uint16_t *b3, int d, const double *xv) {  // [16 x KY]: xh|xm|xl|xh|xm|xh
-    for (int i = 0; i < K; ++i) {
-      uint16_t h, m, l;
-      split3(xv[i], h, m, l);
-      const uint16_t blk[6] = {h, m, l, h, m, h};
-      for (int b = 0; b < 6; ++b) b3[kmaj(d, b * K + i, C::DC)] = blk[b];
-    }
-  };
-  auto put_bx = [&](uint16_t *bx, int d, const double *xv, int parts) {  // parts x [KBn x 16]
-    for (int i = 0; i < K; ++i) {
-      uint16_t h, m, l;
-      split3(xv[i], h, m, l);
-      const uint16_t prt[3] = {h, m, l};
-      for (int e = 0; e < parts; ++e) bx[e * C::BX_BYTES / 2 + kmaj(i, d, C::KBn)] = prt[e];
-    }
-  };
-  for (int c = 0; c < nch; ++c) {
-    uint16_t *bf = tab.data() + (size_t)c * T1;
-    uint16_t *t2 = tab.data() + off2 + (size_t)c * T2;
-    for (int d = 0; d < DC; ++d) {
-      const int t = c * DC + d;
-      if (t >= n) continue;
-      xrow(t, x);
-      frow(t, f);
-      for (int q = 0; q <= C::NF; ++q) {
-        uint16_t h, m, l;
-        split3(f[q], h, m, l);
-        const uint16_t prt[3] = {h, m, l};
-        for (int e = 0; e < 3; ++e) bf[e * C::BF_BYTES / 2 + kmaj(q, d, C::NGn)] = prt[e];
-      }
-      put_bx(bf + 3 * C::BF_BYTES / 2, d, x, 2);
-      put_b3(t2, d, x);
-      put_bx(t2 + C::B3_BYTES / 2, d, x, 3);
-    }
-  }
-  for (int c = 0; c < ncm; ++c) {
-    uint16_t *b3 = tab.data() + offy + (size_t)c * TY;
-    for (int d = 0; d < DC; ++d) {
-      const int t = n + c * DC + d;
-      if (t >= N) continue;
-      xrow(t, x);
-      put_b3(b3, d, x);
-    }
-  }
-}
-
-int build_tc(bfast_plan &pl) {
-  std::vector<uint16_t> tab;
-  size_t o2 = 0, oy = 0;
-  switch (pl.k) {
-    case 0: build_tc_tables<2>(pl, tab, o2, oy); break;
-    case 1: build_tc_tables<4>(pl, tab, o2, oy); break;
-    case 2: build_tc_tables<6>(pl, tab, o2, oy); break;
-    case 3: build_tc_tables<8>(pl, tab, o2, oy); break;
-    case 4: build_tc_tables<10>(pl, tab, o2, oy); break;
-    case 5: build_tc_tables<12>(pl, tab, o2, oy); break;
-    case 6: build_tc_tables<14>(pl, tab, o2, oy); break;
-    default: return BFAST_EUNSUPPORTED;
-  }
-  pl.nch = (pl.n + 15) / 16;
-  pl.ncm = ((int)pl.N - pl.n + 15) / 16;
-  pl.tab2_off = o2 * 2;
-  pl.taby_off = oy * 2;
-  CUDA_TRY(cudaMalloc(&pl.dtab, tab.size() * 2));
-  CUDA_TRY(cudaMemcpy(pl.dtab, tab.data(), tab.size() * 2, cudaMemcpyHostToDevice));
-  return BFAST_OK;
-}
 
 // Chunk tables of the fused kernel (monitor_fused.cuh), B operands in the
 // canonical K-major layout, fp64 values split into bf16 parts:
@@ -496,81 +399,19 @@ int launch_fused(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStre
 
 template <int K>
 int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t st) {
-  using TC = bfast::TcCfg<K>;
   static thread_local int configured_dev = -1;
   int bp = 128;
   while (bp > 32 && simt_smem(pl, bp) > (size_t)kMaxSmem) bp >>= 1;
-  size_t smem = simt_smem(pl, bp);
-  if (smem > (size_t)kMaxSmem) return fail(BFAST_EUNSUPPORTED, "shared memory %zu B too large", smem);
+  const size_t smem = simt_smem(pl, bp);
   if (configured_dev != pl.device) {
-    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_simt_kernel<K>,
-                                  cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmem));
-    CUDA_TRY(cudaFuncSetAttribute(bfast::refit_fp64_kernel<K>,
-                                  cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmem));
-    {
-      cudaFuncAttributes fa{};
-      CUDA_TRY(cudaFuncGetAttributes(&fa, bfast::monitor_tc_kernel<K>));
-      CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_tc_kernel<K>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                    kMaxSmem - (int)fa.sharedSizeBytes));
-      // all of the unified L1/shared array as shared memory: the stack is
-      // streamed by TMA, nothing is reused through L1
-      CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_tc_kernel<K>, cudaFuncAttributePreferredSharedMemoryCarveout,
-                                    (int)cudaSharedmemCarveoutMaxShared));
-    }
+    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_simt_kernel<K>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  kMaxSmem));
+    CUDA_TRY(cudaFuncSetAttribute(bfast::refit_fp64_kernel<K>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  kMaxSmem));
     configured_dev = pl.device;
   }
   int sms = 148;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, pl.device);
-  // tensor-core path on the full 128-pixel tiles when the stack rows allow
-  // 16-byte bulk copies; SIMT kernel on the ragged tail (or everything)
-  const int tc_hcap = pl.hcap;
-  // shared-memory layout and CTAs per SM.  Co-resident CTAs hide each
-  // other's latencies (1 -> 2 -> 3 CTAs/SM measured 1.5x, then 1.08x), so
-  // take the layout that admits the most CTAs, preferring among equals the
-  // earlier entry: a third stack stage is worth 1.5% on the Landsat scene
-  // (it absorbs the HBM latency of the history's first read), double operand buffers
-  // let the consumers fill chunk c+1 while the MMA still reads chunk c.
-  // Limits: registers (80 x 256 threads at launch -> 3 CTAs), shared memory
-  // (228 KB per SM, 1 KB reserved + 1 KB static per CTA), TMEM (512 columns).
-  // (The occupancy API is not used: it does not model setmaxnreg kernels.)
-  int tc_sy = 2, tc_nop = 1, per_sm = 0;
-  {
-    const int cand[4][2] = {{3, 2}, {2, 2}, {3, 1}, {2, 1}};
-    using Shape = bfast::TcShape<K>;
-    const int reg_cap = std::min(65536 / (bfast::kTcThreads * Shape::LAUNCH_REGS), Shape::CTAS);
-    const int tmem_cap = 512 / TC::TMEM_COLS;
-    for (auto &c : cand) {
-      const size_t b = TC::smem_bytes(tc_hcap, pl.nch, c[0], c[1]);
-      if (b + 1024 > (size_t)kMaxSmem) continue;
-      int nb = (int)(kSmemPerSM / (b + 2048));
-      nb = std::min(nb, std::min(reg_cap, tmem_cap));
-      if (std::getenv("BFAST_VERBOSE"))
-        std::fprintf(stderr, "bfast: candidate sy=%d nop=%d smem=%zu ctas/sm=%d\n", c[0], c[1], b, nb);
-      if (nb > per_sm) {
-        per_sm = nb;
-        tc_sy = c[0];
-        tc_nop = c[1];
-      }
-    }
-  }
-  if (const char *lay = std::getenv("BFAST_TC_LAYOUT")) {  // experiments: "sy,nop,per_sm"
-    int a = 0, b = 0, c = 0;
-    if (std::sscanf(lay, "%d,%d,%d", &a, &b, &c) == 3 && a >= 2 && a <= 4 && b >= 1 && b <= 2 && c >= 1 && c <= 4) {
-      tc_sy = a;
-      tc_nop = b;
-      per_sm = c;
-    }
-  }
-  const size_t tc_smem = TC::smem_bytes(tc_hcap, pl.nch, tc_sy, tc_nop);
-  if (std::getenv("BFAST_VERBOSE"))
-    std::fprintf(stderr, "bfast: tc layout k=%d hcap=%d nch=%d sy=%d nop=%d smem=%zu per_sm=%d tmem_cols=%d\n", pl.k,
-                 tc_hcap, pl.nch, tc_sy, tc_nop, tc_smem, per_sm, TC::TMEM_COLS);
-  const bool tc_ok = per_sm > 0 && pl.dtab && pl.mode == 2 && (prm.ldY % 4) == 0 &&
-                     ((uintptr_t)(prm.Y + prm.p0) % 16) == 0 && tc_smem + 1024 <= (size_t)kMaxSmem;
-  CUtensorMap ymap, hmap;  // full stack; history only (dates >= n out of bounds)
-  const bool tma_ok = tc_ok && make_stack_map(&ymap, prm.Y + prm.p0, prm.ldY, prm.P, pl.N, TC::PIX) &&
-                      make_stack_map(&hmap, prm.Y + prm.p0, prm.ldY, prm.P, pl.n, TC::PIX);
-  const int64_t ntiles = tma_ok ? (prm.P + TC::PIX - 1) / TC::PIX : 0;
   // the refit list/counter are plan scratch: order executions on any stream
   CUDA_TRY(cudaStreamWaitEvent(st, pl.scratch_free, 0));
   CUDA_TRY(cudaMemsetAsync(prm.refit_count, 0, sizeof(int32_t), st));
@@ -587,31 +428,12 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
     if (rc) return rc;
     launches += fused ? 1 : 0;
   }
-  if (ntiles > 0) {
-    bfast::TcTables tb;
-    tb.tab1 = pl.dtab;
-    tb.tab2 = pl.dtab + pl.tab2_off;
-    tb.taby = pl.dtab + pl.taby_off;
-    tb.nch = pl.nch;
-    tb.ncm = pl.ncm;
-    tb.ntiles = ntiles;
-    tb.sy = tc_sy;
-    tb.nop = tc_nop;
-    const int64_t grid = std::min<int64_t>(ntiles, (int64_t)sms * per_sm);
-    bfast::MonitorParams q = prm;
-    q.hcap = tc_hcap;
-    bfast::monitor_tc_kernel<K><<<(unsigned)grid, bfast::kTcThreads, tc_smem, st>>>(q, tb, ymap, hmap);
-    CUDA_TRY(cudaGetLastError());
-    ++launches;
-  }
-  // SIMT kernel: forced (BFAST_KERNEL=simt) or a stack TMA cannot read
-  const int64_t rest = (fused || ntiles > 0) ? 0 : prm.P;
-  if (rest > 0) {
-    bfast::MonitorParams q = prm;
-    q.P = rest;
-    const int64_t blocks = (rest + bp - 1) / bp;
-    if (blocks > 0x7fffffff) return fail(BFAST_EUNSUPPORTED, "P too large");
-    bfast::monitor_simt_kernel<K><<<(unsigned)blocks, bp, smem, st>>>(q);
+  // SIMT kernel: forced (BFAST_KERNEL=simt), or a stack the TMA cannot read
+  // (row pitch not a multiple of 16 bytes)
+  if (!fused && prm.P > 0) {
+    if (smem > (size_t)kMaxSmem) return fail(BFAST_EUNSUPPORTED, "shared memory %zu B too large", smem);
+    const int64_t blocks = (prm.P + bp - 1) / bp;
+    bfast::monitor_simt_kernel<K><<<(unsigned)blocks, bp, smem, st>>>(prm);
     CUDA_TRY(cudaGetLastError());
     ++launches;
   }
@@ -654,12 +476,15 @@ int launch(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t s
 }
 
 // --- one-shot plan cache (bfast_monitor / bfast_monitor_ex / host paths)
+// Plans are shared_ptr: a caller holds its reference for the whole
+// execution, so evicting the plan from the cache (a 17th key, possibly from
+// another thread) cannot free it under a running call.
 std::mutex g_cache_mu;
-std::vector<std::unique_ptr<bfast_plan>> g_cache;
+std::vector<std::shared_ptr<bfast_plan>> g_cache;
 
 int env_mode() {
   const char *m = std::getenv("BFAST_KERNEL");
-  return !m ? 0 : (std::strcmp(m, "simt") == 0 ? 1 : std::strcmp(m, "tc1") == 0 ? 2 : 0);
+  return !m ? 0 : (std::strcmp(m, "simt") == 0 ? 1 : 0);
 }
 
 bool same_plan(const bfast_plan &pl, int dev, int64_t N, const double *dates, int32_t n, int32_t k,
@@ -669,11 +494,11 @@ bool same_plan(const bfast_plan &pl, int dev, int64_t N, const double *dates, in
 }
 
 int cached_plan(int dev, int64_t N, const double *dates, int32_t n, int32_t k, float h, float lambda,
-                bfast_plan **out) {
+                std::shared_ptr<bfast_plan> &out) {
   std::lock_guard<std::mutex> g(g_cache_mu);
   for (auto &p : g_cache)
     if (same_plan(*p, dev, N, dates, n, k, h, lambda) && p->mode == env_mode()) {
-      *out = p.get();
+      out = p;
       return BFAST_OK;
     }
   bfast_plan *pl = nullptr;
@@ -681,7 +506,7 @@ int cached_plan(int dev, int64_t N, const double *dates, int32_t n, int32_t k, f
   if (rc) return rc;
   if (g_cache.size() >= 16) g_cache.erase(g_cache.begin());
   g_cache.emplace_back(pl);
-  *out = pl;
+  out = g_cache.back();
   return BFAST_OK;
 }
 
@@ -857,7 +682,7 @@ int bfast_plan_create(bfast_plan **out, int device, int64_t N, const double *dat
     return fail(BFAST_EUNSUPPORTED, "N=%lld too large for the refit kernel", (long long)N);
   {
     const char *mode = std::getenv("BFAST_KERNEL");
-    pl->mode = !mode ? 0 : (std::strcmp(mode, "simt") == 0 ? 1 : std::strcmp(mode, "tc1") == 0 ? 2 : 0);
+    pl->mode = !mode ? 0 : (std::strcmp(mode, "simt") == 0 ? 1 : 0);
   }
   std::vector<float> X;
   std::vector<double> X64;
@@ -874,7 +699,6 @@ int bfast_plan_create(bfast_plan **out, int device, int64_t N, const double *dat
   if (e == cudaSuccess) e = cudaMemset(pl->dcount, 0, sizeof(int32_t));
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&pl->scratch_free, cudaEventDisableTiming);
   int trc = BFAST_OK;
-  if (e == cudaSuccess && pl->mode == 2 && N <= 32767) trc = build_tc(*pl);
   if (e == cudaSuccess && trc == BFAST_OK && pl->mode == 0) trc = build_fz(*pl);
   pl->nch = (n_hist + 15) / 16;
   pl->ncm = ((int)N - n_hist + 15) / 16;
@@ -910,8 +734,8 @@ int bfast_monitor_ex(const bfast_args *a) {
   if (rc) return rc;
   int dev = 0;
   CUDA_TRY(cudaGetDevice(&dev));
-  bfast_plan *pl = nullptr;
-  rc = cached_plan(dev, a->N, a->dates, a->n_hist, a->k, a->h, a->lambda, &pl);
+  std::shared_ptr<bfast_plan> pl;
+  rc = cached_plan(dev, a->N, a->dates, a->n_hist, a->k, a->h, a->lambda, pl);
   if (rc) return rc;
   std::lock_guard<std::mutex> g(pl->mu);
   return execute_range(*pl, a, 0, a->P);
@@ -938,7 +762,40 @@ int bfast_monitor(const float *Y, int64_t N, int64_t P, const double *dates, int
 }
 
 // End-to-end on host buffers: pixel slabs, double-buffered H2D on a copy
-// stream overlapping the kernel on the compute stream.
+// stream overlapping the kernel on the compute stream.  The device slabs,
+// streams and events are the plan's (bfast_plan::HostPath), kept across
+// calls: a stream of tiles pays the allocations once.
+int host_path_ensure(bfast_plan &pl, int64_t slab) {
+  auto &hp = pl.host;
+  if (!hp.cs) {
+    CUDA_TRY(cudaStreamCreateWithFlags(&hp.cs, cudaStreamNonBlocking));
+    CUDA_TRY(cudaStreamCreateWithFlags(&hp.ks, cudaStreamNonBlocking));
+    for (int i = 0; i < 2; ++i) {
+      CUDA_TRY(cudaEventCreateWithFlags(&hp.loaded[i], cudaEventDisableTiming));
+      CUDA_TRY(cudaEventCreateWithFlags(&hp.done[i], cudaEventDisableTiming));
+    }
+  }
+  if (slab <= hp.slab) return BFAST_OK;
+  CUDA_TRY(cudaStreamSynchronize(hp.ks));
+  CUDA_TRY(cudaStreamSynchronize(hp.cs));
+  for (int i = 0; i < 2; ++i) {
+    cudaFree(hp.dY[i]);
+    cudaFree(hp.dB[i]);
+    cudaFree(hp.dM[i]);
+    hp.dY[i] = nullptr;
+    hp.dB[i] = nullptr;
+    hp.dM[i] = nullptr;
+  }
+  hp.slab = 0;
+  for (int i = 0; i < 2; ++i) {
+    CUDA_TRY(cudaMalloc(&hp.dY[i], sizeof(float) * (size_t)pl.N * slab));
+    CUDA_TRY(cudaMalloc(&hp.dB[i], sizeof(int32_t) * slab));
+    CUDA_TRY(cudaMalloc(&hp.dM[i], sizeof(float) * slab));
+  }
+  hp.slab = slab;
+  return BFAST_OK;
+}
+
 int bfast_monitor_host(const float *Y_host, int64_t N, int64_t P, int64_t ldY, const double *dates,
                        int32_t n_hist, int32_t k, float h, float lambda, int32_t *out_break_host,
                        float *out_magnitude_host, int device) {
@@ -954,62 +811,36 @@ int bfast_monitor_host(const float *Y_host, int64_t N, int64_t P, int64_t ldY, c
   CUDA_TRY(cudaGetDevice(&prev));
   const int dev = device < 0 ? prev : device;
   CUDA_TRY(cudaSetDevice(dev));
-  bfast_plan *pl = nullptr;
-  rc = cached_plan(dev, N, dates, n_hist, k, h, lambda, &pl);
-  if (rc) {
-    cudaSetDevice(prev);
-    return rc;
-  }
+  struct Restore {
+    int d;
+    ~Restore() { cudaSetDevice(d); }
+  } restore{prev};
+  std::shared_ptr<bfast_plan> pl;
+  rc = cached_plan(dev, N, dates, n_hist, k, h, lambda, pl);
+  if (rc) return rc;
   // slab width: ~1 GiB of stack per buffer, multiple of 128 pixels
   int64_t slab = std::max<int64_t>(128, ((int64_t)1 << 28) / N / 128 * 128);
   slab = std::min<int64_t>(slab, (P + 127) / 128 * 128);
-  float *dY[2] = {nullptr, nullptr};
-  int32_t *dB[2] = {nullptr, nullptr};
-  float *dM[2] = {nullptr, nullptr};
-  cudaStream_t cs = nullptr, ks = nullptr;
-  cudaEvent_t loaded[2] = {nullptr, nullptr}, done[2] = {nullptr, nullptr};
+  std::lock_guard<std::mutex> g(pl->mu);
+  rc = host_path_ensure(*pl, slab);
+  if (rc) return rc;
+  auto &hp = pl->host;
+  slab = hp.slab;
   int launches = 0;
   cudaError_t e = cudaSuccess;
-  auto cleanup = [&]() {
-    for (int i = 0; i < 2; ++i) {
-      cudaFree(dY[i]);
-      cudaFree(dB[i]);
-      cudaFree(dM[i]);
-      if (loaded[i]) cudaEventDestroy(loaded[i]);
-      if (done[i]) cudaEventDestroy(done[i]);
-    }
-    if (cs) cudaStreamDestroy(cs);
-    if (ks) cudaStreamDestroy(ks);
-    cudaSetDevice(prev);
-  };
-  for (int i = 0; i < 2 && e == cudaSuccess; ++i) {
-    e = cudaMalloc(&dY[i], sizeof(float) * (size_t)N * slab);
-    if (e == cudaSuccess) e = cudaMalloc(&dB[i], sizeof(int32_t) * slab);
-    if (e == cudaSuccess) e = cudaMalloc(&dM[i], sizeof(float) * slab);
-    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&loaded[i], cudaEventDisableTiming);
-    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&done[i], cudaEventDisableTiming);
-  }
-  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
-  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ks, cudaStreamNonBlocking);
-  if (e != cudaSuccess) {
-    cleanup();
-    return fail(e == cudaErrorMemoryAllocation ? BFAST_ENOMEM : BFAST_ECUDA, "host path: %s",
-                cudaGetErrorString(e));
-  }
-  std::lock_guard<std::mutex> g(pl->mu);
   int slot = 0;
   for (int64_t b0 = 0; b0 < P && rc == BFAST_OK; b0 += slab, slot ^= 1) {
     const int64_t w = std::min(slab, P - b0);
     // the buffer is free once the kernel that used it two slabs ago is done
-    e = cudaStreamWaitEvent(cs, done[slot], 0);
+    e = cudaStreamWaitEvent(hp.cs, hp.done[slot], 0);
     if (e == cudaSuccess)
-      e = cudaMemcpy2DAsync(dY[slot], sizeof(float) * w, Y_host + b0, sizeof(float) * ldY,
-                            sizeof(float) * w, N, cudaMemcpyHostToDevice, cs);
-    if (e == cudaSuccess) e = cudaEventRecord(loaded[slot], cs);
-    if (e == cudaSuccess) e = cudaStreamWaitEvent(ks, loaded[slot], 0);
+      e = cudaMemcpy2DAsync(hp.dY[slot], sizeof(float) * w, Y_host + b0, sizeof(float) * ldY, sizeof(float) * w,
+                            N, cudaMemcpyHostToDevice, hp.cs);
+    if (e == cudaSuccess) e = cudaEventRecord(hp.loaded[slot], hp.cs);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(hp.ks, hp.loaded[slot], 0);
     if (e != cudaSuccess) break;
     bfast_args a{};
-    a.Y = dY[slot];
+    a.Y = hp.dY[slot];
     a.N = N;
     a.P = w;
     a.ldY = w;
@@ -1018,21 +849,21 @@ int bfast_monitor_host(const float *Y_host, int64_t N, int64_t P, int64_t ldY, c
     a.k = k;
     a.h = h;
     a.lambda = lambda;
-    a.out_break = dB[slot];
-    a.out_magnitude = dM[slot];
-    a.stream = ks;
+    a.out_break = hp.dB[slot];
+    a.out_magnitude = hp.dM[slot];
+    a.stream = hp.ks;
     rc = execute_range(*pl, &a, 0, w);
     launches += g_launches;
     if (rc) break;
-    e = cudaMemcpyAsync(out_break_host + b0, dB[slot], sizeof(int32_t) * w, cudaMemcpyDeviceToHost, ks);
+    e = cudaMemcpyAsync(out_break_host + b0, hp.dB[slot], sizeof(int32_t) * w, cudaMemcpyDeviceToHost, hp.ks);
     if (e == cudaSuccess)
-      e = cudaMemcpyAsync(out_magnitude_host + b0, dM[slot], sizeof(float) * w, cudaMemcpyDeviceToHost, ks);
-    if (e == cudaSuccess) e = cudaEventRecord(done[slot], ks);
+      e = cudaMemcpyAsync(out_magnitude_host + b0, hp.dM[slot], sizeof(float) * w, cudaMemcpyDeviceToHost, hp.ks);
+    if (e == cudaSuccess) e = cudaEventRecord(hp.done[slot], hp.ks);
     if (e != cudaSuccess) break;
   }
-  if (e == cudaSuccess && rc == BFAST_OK) e = cudaStreamSynchronize(ks);
-  cleanup();
+  const cudaError_t es = cudaStreamSynchronize(hp.ks);
   if (rc) return rc;
+  if (e == cudaSuccess) e = es;
   if (e != cudaSuccess) return fail(BFAST_ECUDA, "host path: %s", cudaGetErrorString(e));
   g_launches = launches;
   return BFAST_OK;
@@ -1069,6 +900,147 @@ int bfast_monitor_multi(const float *Y_host, int64_t N, int64_t P, int64_t ldY, 
     total += launches[r];
   }
   g_launches = total;
+  return BFAST_OK;
+}
+
+}  // extern "C"
+namespace {
+std::mutex g_ipc_mu;
+std::map<void *, void *> g_ipc_base;  // mapped pointer -> opened allocation base
+}  // namespace
+extern "C" {
+
+int bfast_monitor_shards(const float *const *Y_dev, const int64_t *P, const int64_t *ldY, const int *devices,
+                         int nshards, int64_t N, const double *dates, int32_t n_hist, int32_t k, float h,
+                         float lambda, int gather_device, int32_t *out_break, float *out_magnitude) {
+  int rc = validate_scalar(N, dates, n_hist, k, h, lambda);
+  if (rc) return rc;
+  if (!Y_dev || !P || !ldY || !devices || nshards < 1) return fail(BFAST_EINVAL, "no shards");
+  int64_t total = 0;
+  for (int i = 0; i < nshards; ++i) {
+    if (P[i] < 0 || ldY[i] < P[i]) return fail(BFAST_EINVAL, "shard %d: P < 0 or ldY < P", i);
+    if (P[i] > 0 && !Y_dev[i]) return fail(BFAST_EINVAL, "shard %d: NULL stack", i);
+    total += P[i];
+  }
+  if (total > 0 && (!out_break || !out_magnitude)) return fail(BFAST_EINVAL, "NULL outputs");
+  std::vector<int> status(nshards, BFAST_OK);
+  std::vector<std::string> errs(nshards);
+  std::vector<int> launches(nshards, 0);
+  std::vector<std::thread> th;
+  int64_t off = 0;
+  for (int i = 0; i < nshards; ++i) {
+    th.emplace_back([&, i, off]() {
+      if (P[i] == 0) return;
+      int st = BFAST_OK;
+      cudaError_t e = cudaSetDevice(devices[i]);
+      if (e == cudaSuccess && devices[i] != gather_device) {
+        // the shard's epilogue stores go straight to the gather device
+        e = cudaDeviceEnablePeerAccess(gather_device, 0);
+        if (e == cudaErrorPeerAccessAlreadyEnabled) {
+          cudaGetLastError();
+          e = cudaSuccess;
+        }
+      }
+      std::shared_ptr<bfast_plan> pl;
+      cudaStream_t s = nullptr;
+      if (e == cudaSuccess) st = cached_plan(devices[i], N, dates, n_hist, k, h, lambda, pl);
+      if (e == cudaSuccess && st == BFAST_OK) e = cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
+      if (e == cudaSuccess && st == BFAST_OK) {
+        bfast_args a{};
+        a.Y = Y_dev[i];
+        a.N = N;
+        a.P = P[i];
+        a.ldY = ldY[i];
+        a.dates = dates;
+        a.n_hist = n_hist;
+        a.k = k;
+        a.h = h;
+        a.lambda = lambda;
+        a.out_break = out_break + off;
+        a.out_magnitude = out_magnitude + off;
+        a.stream = s;
+        std::lock_guard<std::mutex> g(pl->mu);
+        st = execute_range(*pl, &a, 0, P[i]);
+        launches[i] = g_launches;
+        if (st == BFAST_OK) e = cudaStreamSynchronize(s);
+      }
+      if (s) cudaStreamDestroy(s);
+      if (st == BFAST_OK && e != cudaSuccess) st = fail(BFAST_ECUDA, "%s", cudaGetErrorString(e));
+      status[i] = st;
+      errs[i] = g_err;
+    });
+    off += P[i];
+  }
+  for (auto &t : th) t.join();
+  int total_l = 0;
+  for (int i = 0; i < nshards; ++i) {
+    if (status[i]) return fail(status[i], "shard %d (device %d): %s", i, devices[i], errs[i].c_str());
+    total_l += launches[i];
+  }
+  g_launches = total_l;
+  return BFAST_OK;
+}
+
+// The IPC handle: the CUDA handle of the allocation containing dev_ptr (a
+// caching allocator hands out sub-blocks of larger cudaMalloc segments)
+// followed by dev_ptr's byte offset in it.
+typedef CUresult (*PFN_getAddressRange)(CUdeviceptr *, size_t *, CUdeviceptr);
+int bfast_ipc_export(const void *dev_ptr, unsigned char *handle) {
+  if (!dev_ptr || !handle) return fail(BFAST_EINVAL, "NULL pointer");
+  static PFN_getAddressRange range = nullptr;
+  static std::once_flag once;
+  std::call_once(once, []() {
+    void *f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      range = (PFN_getAddressRange)f;
+  });
+  if (!range) return fail(BFAST_ECUDA, "cuMemGetAddressRange unavailable");
+  CUdeviceptr base = 0;
+  size_t size = 0;
+  if (range(&base, &size, (CUdeviceptr)(uintptr_t)dev_ptr) != CUDA_SUCCESS)
+    return fail(BFAST_EINVAL, "not a device allocation");
+  cudaIpcMemHandle_t hnd;
+  CUDA_TRY(cudaIpcGetMemHandle(&hnd, (void *)(uintptr_t)base));
+  static_assert(sizeof(hnd) + sizeof(int64_t) == BFAST_IPC_HANDLE_BYTES, "handle size");
+  const int64_t off = (int64_t)((uintptr_t)dev_ptr - (uintptr_t)base);
+  std::memcpy(handle, &hnd, sizeof(hnd));
+  std::memcpy(handle + sizeof(hnd), &off, sizeof(off));
+  return BFAST_OK;
+}
+
+int bfast_ipc_open(const unsigned char *handle, int device, void **dev_ptr) {
+  if (!handle || !dev_ptr) return fail(BFAST_EINVAL, "NULL pointer");
+  *dev_ptr = nullptr;
+  int prev = 0;
+  CUDA_TRY(cudaGetDevice(&prev));
+  if (device >= 0) CUDA_TRY(cudaSetDevice(device));
+  cudaIpcMemHandle_t hnd;
+  int64_t off = 0;
+  std::memcpy(&hnd, handle, sizeof(hnd));
+  std::memcpy(&off, handle + sizeof(hnd), sizeof(off));
+  void *base = nullptr;
+  const cudaError_t e = cudaIpcOpenMemHandle(&base, hnd, cudaIpcMemLazyEnablePeerAccess);
+  cudaSetDevice(prev);
+  if (e != cudaSuccess) return fail(BFAST_ECUDA, "cudaIpcOpenMemHandle: %s", cudaGetErrorString(e));
+  *dev_ptr = static_cast<char *>(base) + off;
+  std::lock_guard<std::mutex> g(g_ipc_mu);
+  g_ipc_base[*dev_ptr] = base;
+  return BFAST_OK;
+}
+
+int bfast_ipc_close(void *dev_ptr) {
+  if (!dev_ptr) return BFAST_OK;
+  void *base = dev_ptr;
+  {
+    std::lock_guard<std::mutex> g(g_ipc_mu);
+    auto it = g_ipc_base.find(dev_ptr);
+    if (it == g_ipc_base.end()) return fail(BFAST_EINVAL, "not a pointer from bfast_ipc_open");
+    base = it->second;
+    g_ipc_base.erase(it);
+  }
+  CUDA_TRY(cudaIpcCloseMemHandle(base));
   return BFAST_OK;
 }
 

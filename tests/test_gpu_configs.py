@@ -1,0 +1,176 @@
+"""GPU parity on the configurations round 1 left untested (VERDICT r1
+"What's weak" 3), and the multi-GPU gather paths.
+
+Every case compares the CUDA path (through the C ABI) with the fp64 oracle
+on the same device bytes (oracle/parity.py tolerances), or with another
+CUDA-path result that must be bit-identical.
+"""
+import json
+import math
+import os
+import subprocess
+import sys
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+import oracle
+from oracle import parity
+from paper_conf_icde_giesekerhvo20_b200 import binding, synth
+
+pytestmark = pytest.mark.gpu
+DEV = "cuda:0"
+HERE = os.path.dirname(os.path.abspath(__file__))
+
+
+def _parity(out, Y, idx, dates, n, k, hf, lam):
+    it = torch.tensor(idx, device=Y.device)
+    Ys = np.ascontiguousarray(Y.index_select(1, it).cpu().numpy())
+    orc = oracle.monitor(Ys, dates, n, k, hf, lam)
+    gpu = {key: v.index_select(0, it).cpu().numpy() for key, v in out.items() if torch.is_tensor(v)}
+    rep = parity.compare(gpu, orc, dates, n, k)
+    assert rep["ok"], json.dumps(rep)
+    np.testing.assert_array_equal(gpu["nbar"], orc["nbar"])
+    return rep, gpu, orc
+
+
+def test_sentinel2_shape_parity():
+    """configs[3] shape: N = 700, n = 350, 5-day cadence (f = 73), i.i.d. 50%
+    missing -- a 2^20-pixel shard of the 10980^2 tile generated exactly as
+    bench.py's strong-scaling run does (columns of the full scene), every
+    pixel against the oracle."""
+    spec = synth.CONFIGS["sentinel2"]
+    Y, dates = synth.generate(spec, DEV, columns=(5_000_000, 5_000_000 + (1 << 20)))
+    out = binding.bfast_monitor_ex(Y, dates, spec.n_hist, spec.k, spec.hf, spec.lam, diagnostics=True)
+    torch.cuda.synchronize()
+    rep, _, _ = _parity(out, Y, np.arange(Y.shape[1]), dates, spec.n_hist, spec.k, spec.hf, spec.lam)
+    assert rep["breaks_oracle"] > 0.05 * Y.shape[1]
+
+
+def test_irregular_dates():
+    """Acquisition dates jittered by up to +-1 day (reading R11: harmonics of
+    2 pi j dates[t], trend the 1-based index): the product-to-sum Gram
+    tables and the yhat tables are built from the actual dates."""
+    spec = synth.StackSpec(P=200_000, N=400, n_hist=200, miss=0.6, mask="cloud", seed=81)
+    Y, _ = synth.generate(spec, DEV)
+    rng = np.random.default_rng(5)
+    dates = synth.make_dates(spec.N) + rng.uniform(-1.0, 1.0, spec.N) / 365.25
+    assert np.all(np.diff(dates) > 0)
+    out = binding.bfast_monitor_ex(Y, dates, spec.n_hist, spec.k, spec.hf, spec.lam, diagnostics=True)
+    torch.cuda.synchronize()
+    idx = synth.sample_columns(Y, spec.P, 1 << 16, seed=1)
+    _parity(out, Y, idx, dates, spec.n_hist, spec.k, spec.hf, spec.lam)
+
+
+@pytest.mark.parametrize("mode", ["fused", "simt"])
+def test_nan_payloads_on_device(mode, monkeypatch):
+    """Any NaN payload is missing (L164, reading R9): quiet, signalling,
+    negative and payload-carrying NaNs give bit-identical outputs to the
+    canonical NaN, on both kernels, and match the oracle."""
+    monkeypatch.setenv("BFAST_KERNEL", mode)
+    spec = synth.StackSpec(P=65_536, N=230, n_hist=115, miss=0.5, seed=91)
+    Y, dates = synth.generate(spec, DEV)
+    ref = binding.bfast_monitor_ex(Y, dates, spec.n_hist, spec.k, spec.hf, spec.lam, diagnostics=True)
+    torch.cuda.synchronize()
+    bits = Y.view(torch.int32).clone()
+    nan = torch.isnan(Y)
+    payloads = torch.tensor([0x7FC00001, -0x00400000, 0x7F800001, -0x007EDCBB, 0x7FFFFFFF],
+                            dtype=torch.int32, device=DEV)  # -0x00400000 = 0xFFC00000
+    pick = torch.randint(0, len(payloads), Y.shape, device=DEV, generator=torch.Generator(DEV).manual_seed(3))
+    bits = torch.where(nan, payloads[pick], bits)
+    Y2 = bits.view(torch.float32)
+    assert torch.isnan(Y2).equal(nan)
+    out = binding.bfast_monitor_ex(Y2, dates, spec.n_hist, spec.k, spec.hf, spec.lam, diagnostics=True)
+    torch.cuda.synchronize()
+    for key in ("break", "magnitude", "sigma", "nbar", "beta"):
+        assert torch.equal(out[key].nan_to_num(), ref[key].nan_to_num()), key
+    _parity(out, Y2, np.arange(0, spec.P, 4), dates, spec.n_hist, spec.k, spec.hf, spec.lam)
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("N,miss,k", [(250, 0.9, 5), (100, 0.9, 1), (1000, 0.1, 5)])
+def test_full_size_sweep_corners_sampled(N, miss, k):
+    """configs[2] corners at the full 4096^2 pixels in bench.py's launch
+    configuration (Plan.execute), 2^16 sampled pixels against the oracle:
+    the ill-conditioned / mostly-degenerate corners (90% missing) and the
+    long, dense one (ring of 125 slots: 2 tiles per CTA)."""
+    idx = [100, 250, 500, 1000].index(N) * 9 + [0.1, 0.5, 0.9].index(miss) * 3 + [1, 3, 5].index(k)
+    spec = synth.sweep_spec(N, miss, k, index=idx)
+    Y, dates = synth.generate(spec, DEV)
+    plan = binding.Plan(0, spec.N, dates, spec.n_hist, spec.k, spec.hf, spec.lam)
+    out = plan.execute(Y, diagnostics=True)
+    torch.cuda.synchronize()
+    idx = synth.sample_columns(Y, spec.P, 1 << 16, seed=2)
+    _parity(out, Y, idx, dates, spec.n_hist, spec.k, spec.hf, spec.lam)
+    plan.close()
+    del Y, out
+    torch.cuda.empty_cache()
+
+
+def test_low_sigma_pixels():
+    """sigma-hat / |y| from ~1e-7 (the fp32 quantisation of the data) to
+    1e-4: valid pixels under reading R4 (only an exact fit, sigma-hat <=
+    1e-10 max|y|, is invalid).  The fused kernel sends them to the fp64
+    refit (sigma-hat < 2e-3 max|y|), which must match the oracle; the
+    exactly-fitted constant pixels are -2 on both sides."""
+    N, n, k, P = 230, 115, 2, 8192
+    dates = synth.make_dates(N)
+    rng = np.random.default_rng(11)
+    t = np.arange(1, N + 1)
+    level = rng.uniform(0.3, 0.8, P)
+    rel = 10.0 ** rng.uniform(-7, -4, P)
+    Yh = (level[None, :] + 0.1 * np.sin(2 * math.pi * dates)[:, None] * rng.uniform(-1, 1, P)[None, :]
+          + 0.001 * (t[:, None] / N) + rng.normal(size=(N, P)) * (rel * level)[None, :])
+    Yh[rng.random((N, P)) < 0.5] = np.nan
+    Yh[:, :64] = 0.5                                        # exact fits: sigma-hat = 0
+    Y = torch.tensor(Yh.astype(np.float32), device=DEV)
+    out = binding.bfast_monitor_ex(Y, dates, n, k, 0.25, 1.65, diagnostics=True)
+    torch.cuda.synchronize()
+    rep, gpu, orc = _parity(out, Y, np.arange(P), dates, n, k, 0.25, 1.65)
+    assert (orc["break"][:64] == -2).all() and (orc["deg_reason"][:64] == 5).all()
+    ok = orc["break"][64:] != -2
+    assert ok.mean() > 0.95                                 # the low-noise pixels are valid
+    assert ((gpu["flags"][64:][ok] & binding.FLAG_REFIT_FP64) != 0).all()
+
+
+def test_shards_gather_into_one_map():
+    """bfast_monitor_shards: device-resident shards (ragged sizes; one with a
+    row pitch TMA cannot read -> the SIMT kernel) written straight into one
+    break map; identical to per-shard runs of the same kernels."""
+    spec = synth.StackSpec(P=150_001, N=200, n_hist=100, miss=0.6, mask="cloud", seed=23)
+    Yfull, dates = synth.generate(spec, DEV)
+    cuts = [0, 40_000, 40_000 + 70_001, spec.P]
+    shards = [Yfull[:, cuts[i]:cuts[i + 1]].contiguous() for i in range(3)]
+    odd = torch.empty((spec.N, shards[1].shape[1] + 1), device=DEV)   # ldY % 4 != 0
+    odd[:, : shards[1].shape[1]] = shards[1]
+    shards[1] = odd[:, : shards[1].shape[1]]
+    b, m = binding.bfast_monitor_shards(shards, dates, spec.n_hist, spec.k, spec.hf, spec.lam, gather_device=0)
+    torch.cuda.synchronize()
+    for i, Y in enumerate(shards):
+        o = binding.bfast_monitor_ex(Y, dates, spec.n_hist, spec.k, spec.hf, spec.lam)
+        torch.cuda.synchronize()
+        assert torch.equal(b[cuts[i]:cuts[i + 1]], o["break"]), i
+        assert torch.equal(m[cuts[i]:cuts[i + 1]].nan_to_num(), o["magnitude"].nan_to_num()), i
+    assert binding.last_launch_count() > 0
+
+
+def test_two_process_ipc_gather(tmp_path):
+    """One process per GPU in miniature: two processes on cuda:0, rank 0 owns
+    the break map, rank 1 maps it by CUDA IPC and its kernel stores its
+    shard straight into it; the gathered map equals a one-process run."""
+    init = tmp_path / "rdzv"
+    out = tmp_path / "map.npz"
+    procs = [subprocess.Popen([sys.executable, os.path.join(HERE, "_ipc_worker.py"), str(r), "2", str(init),
+                               str(out)], stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True)
+             for r in range(2)]
+    logs = [p.communicate(timeout=300)[0] for p in procs]
+    assert all(p.returncode == 0 for p in procs), "\n".join(logs)
+    got = np.load(out)
+    spec = synth.StackSpec(P=300_000, N=230, n_hist=115, miss=0.6, mask="cloud", seed=17)
+    Y, dates = synth.generate(spec, DEV)
+    ref = binding.bfast_monitor_ex(Y, dates, spec.n_hist, spec.k, spec.hf, spec.lam)
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(got["brk"], ref["break"].cpu().numpy())
+    np.testing.assert_array_equal(np.nan_to_num(got["mag"]), np.nan_to_num(ref["magnitude"].cpu().numpy()))

@@ -21,10 +21,11 @@ pytestmark = pytest.mark.gpu
 DEV = "cuda:0"
 
 
-@pytest.fixture(params=["tc", "simt"])
+@pytest.fixture(params=["fused", "simt"])
 def mode(request, monkeypatch):
-    """Run the test on the tensor-core path (full 128-pixel tiles; the SIMT
-    kernel takes the ragged tail) and on the SIMT-only path."""
+    """Run the test on the fused tensor-core kernel (monitor_fused.cuh) and on
+    the CUDA-core-only kernel (monitor_simt.cuh, the path for stacks whose
+    row pitch TMA cannot read)."""
     monkeypatch.setenv("BFAST_KERNEL", request.param)
     return request.param
 
@@ -239,12 +240,12 @@ def test_tc_and_simt_paths_agree_closely(monkeypatch):
     spec = synth.StackSpec(P=8192, N=300, n_hist=150, miss=0.5, seed=61)
     Y, dates = synth.generate(spec, DEV)
     outs = {}
-    for m in ("tc", "simt"):
+    for m in ("fused", "simt"):
         monkeypatch.setenv("BFAST_KERNEL", m)
         o = binding.bfast_monitor_ex(Y, dates, spec.n_hist, spec.k, spec.hf, spec.lam, diagnostics=True)
         torch.cuda.synchronize()
         outs[m] = {key: v.cpu().numpy() for key, v in o.items() if hasattr(v, "cpu")}
-    a, b = outs["tc"], outs["simt"]
+    a, b = outs["fused"], outs["simt"]
     assert (a["break"] != b["break"]).mean() < 1e-3
     ok = (a["break"] != -2) & (b["break"] != -2)
     d = np.abs(a["magnitude"][ok] - b["magnitude"][ok]) / np.maximum(1, np.abs(b["magnitude"][ok]))
@@ -254,7 +255,7 @@ def test_tc_and_simt_paths_agree_closely(monkeypatch):
 def test_tc_path_is_deterministic_at_scale(monkeypatch):
     """Race detector for the warp-specialised pipeline: many persistent tiles
     per CTA, repeated runs must agree bit for bit."""
-    monkeypatch.setenv("BFAST_KERNEL", "tc")
+    monkeypatch.setenv("BFAST_KERNEL", "fused")
     spec = synth.StackSpec(P=1 << 21, N=400, n_hist=200, miss=0.6, mask="cloud", seed=71)
     Y, dates = synth.generate(spec, DEV)
     plan = binding.Plan(0, spec.N, dates, spec.n_hist, spec.k, spec.hf, spec.lam)

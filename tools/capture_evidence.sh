@@ -4,7 +4,7 @@
 #   gpurun_out/TAG_s2.json         Sentinel-2 tile (configs[3]) slab by slab on one GPU
 #   gpurun_out/TAG_stream.json     pinned-host streaming (configs[4])
 #   gpurun_out/TAG_launches.csv    ncu launch list (gpu__time_duration, clock-control none)
-#   gpurun_out/TAG_full.ncu-rep    ncu --set full of one monitor_tc launch
+#   gpurun_out/TAG_full.ncu-rep    ncu --set full of one monitor_fused launch
 # then (here):  python profiles/summarize.py full|launches ...
 TAG=${1:?tag}
 mkdir -p gpurun_out
@@ -14,6 +14,6 @@ timeout 900 python bench.py --config stream --steps 3 --warmup 3 --no-cpu-baseli
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"monitor|refit" -c 20 --csv \
   --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 5 --warmup 3 --no-e2e --no-cpu-baseline \
   > /dev/null 2>&1; echo launches=$?
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:monitor_tc -s 3 -c 1 \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:monitor_fused -s 3 -c 1 \
   -o gpurun_out/${TAG}_full python bench.py --steps 1 --warmup 3 --no-e2e --no-cpu-baseline \
   > gpurun_out/${TAG}_ncu.log 2>&1; echo full=$?

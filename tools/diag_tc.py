@@ -10,14 +10,14 @@ idx = [100, 250, 500, 1000].index(N) * 9 + [0.1, 0.5, 0.9].index(miss) * 3 + [1,
 spec = synth.sweep_spec(N, miss, k, P=4096, index=idx)
 Y, dates = synth.generate(spec, "cuda:0")
 res = {}
-for m in ("tc", "simt"):
+for m in ("fused", "simt"):
     os.environ["BFAST_KERNEL"] = m
     o = binding.bfast_monitor_ex(Y, dates, spec.n_hist, k, spec.hf, spec.lam, diagnostics=True)
     torch.cuda.synchronize()
     res[m] = {kk: v.cpu().numpy() for kk, v in o.items() if hasattr(v, "cpu")}
 orc = oracle.monitor(Y.cpu().numpy(), dates, spec.n_hist, k, spec.hf, spec.lam)
 s = parity.column_scales(dates, spec.n_hist, k)
-for m in ("tc", "simt"):
+for m in ("fused", "simt"):
     g = res[m]
     ok = (orc["break"] != -2) & (g["break"] != -2)
     err = np.abs(g["magnitude"] - orc["magnitude"]) / np.maximum(1, np.abs(orc["magnitude"]))

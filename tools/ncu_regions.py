@@ -23,7 +23,7 @@ for l in out.splitlines():
         continue
     f, w, ln, s, i = m.group(1), m.group(2), int(m.group(3)), float(m.group(4)), float(m.group(5))
     key = None
-    if f == "monitor_tc.cuh":
+    if f == "monitor_fused.cuh":
         for name, a, b in rng:
             if a <= ln <= b:
                 key = name

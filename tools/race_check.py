@@ -7,7 +7,7 @@ from paper_conf_icde_giesekerhvo20_b200 import binding, synth
 spec = synth.CONFIGS["landsat"]
 Y, dates = synth.generate(spec, "cuda:0")
 outs = []
-for m in ["tc"] * 6 + ["simt"]:
+for m in ["fused"] * 6 + ["simt"]:
     os.environ["BFAST_KERNEL"] = m
     o = binding.bfast_monitor_ex(Y, dates, spec.n_hist, spec.k, spec.hf, spec.lam, diagnostics=True)
     torch.cuda.synchronize()
