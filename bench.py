@@ -165,6 +165,55 @@ def ncu_traffic(workload_key: str):
         return None
 
 
+def host_cpu():
+    """lscpu sockets x cores x threads of the box (SURVEY 8(d) baseline protocol)."""
+    info = {}
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for ln in out.splitlines():
+            if ":" in ln:
+                k, v = ln.split(":", 1)
+                info[k.strip()] = v.strip()
+    except Exception:
+        pass
+    return {"model": info.get("Model name"), "sockets": info.get("Socket(s)"),
+            "cores_per_socket": info.get("Core(s) per socket"), "threads_per_core": info.get("Thread(s) per core"),
+            "cpus": info.get("CPU(s)")}
+
+
+_ONE_THREAD = {}
+
+
+def cpu_baseline_entry(value, threads, sample):
+    """cpu_baseline object: the all-cores oracle figure plus a 1-thread figure
+    measured on the same workload recipe (bounded sample)."""
+    return {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample,
+            "host": host_cpu(), "one_thread": _ONE_THREAD.get("value")}
+
+
+def measure_one_thread(Y, dates, spec, seconds=3.0):
+    """The oracle on ONE host thread over a bounded sample (pixels/s)."""
+    import numpy as np
+    import torch
+    import oracle
+    from paper_conf_icde_giesekerhvo20_b200 import synth
+    nmax = oracle.max_threads()
+    idx = synth.sample_columns(Y, spec.P, 1024, seed=5)
+    Ys = np.ascontiguousarray(Y.index_select(1, torch.tensor(idx, device=Y.device)).cpu().numpy())
+    t0 = time.perf_counter()
+    oracle.monitor(Ys, dates, spec.n_hist, spec.k, spec.hf, spec.lam, threads=1)
+    dt = time.perf_counter() - t0
+    count = int(min(1 << 16, max(1024, 1024 * seconds / max(dt, 1e-3))))
+    idx = synth.sample_columns(Y, spec.P, count, seed=6)
+    Ys = np.ascontiguousarray(Y.index_select(1, torch.tensor(idx, device=Y.device)).cpu().numpy())
+    t0 = time.perf_counter()
+    oracle.monitor(Ys, dates, spec.n_hist, spec.k, spec.hf, spec.lam, threads=1)
+    dt = time.perf_counter() - t0
+    _ONE_THREAD["value"] = {"value": count / dt, "unit": UNIT, "threads": 1, "sample": f"{count} pixels, {dt:.1f} s"}
+    oracle.monitor(Ys[:, :1], dates, spec.n_hist, spec.k, spec.hf, spec.lam, threads=nmax)  # restore the thread count
+    return _ONE_THREAD["value"]
+
+
 def oracle_sample(Y, dates, spec, count, seed=0):
     """Run the oracle on `count` sampled pixel columns of the device stack Y;
     returns (oracle outputs, seconds, threads, idx)."""
@@ -211,7 +260,7 @@ def run_reference(args):
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": desc, "sample": f"{sub.P} pixels per step (same recipe, CPU sub-scene)"},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
-                             "sample": f"{sub.P} pixels of the workload per step"},
+                             "sample": f"{sub.P} pixels of the workload per step", "host": host_cpu()},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
@@ -229,8 +278,13 @@ def _finish(line, world, rank):
 def run_sharded_tile(args, spec, desc, world, rank, local, dev):
     """configs[3]: one tile too large for a GPU, sharded over the ranks (strong
     scaling).  Each rank generates exactly its pixel range of the scene and
-    processes it in device-sized slabs; the step time is the sum of the slab
-    kernel times, max over ranks."""
+    processes it in device-sized slabs; the break map and magnitudes of the
+    WHOLE tile live on rank 0's GPU and every rank's kernel stores its slice
+    straight into them (CUDA IPC mapping of rank 0's allocation, NVLink peer
+    stores from the epilogue: the gather of SURVEY 8(e) happens inside the
+    timed kernels).  The step time is the sum of the slab times, max over
+    ranks."""
+    import numpy as np
     import torch
     import torch.distributed as dist
     from paper_conf_icde_giesekerhvo20_b200 import binding, synth
@@ -241,27 +295,39 @@ def run_sharded_tile(args, spec, desc, world, rank, local, dev):
     stream = torch.cuda.Stream(device=dev)
     slab = max(128, min(args.slab, e - b))
     Ybuf = torch.empty((N, slab), dtype=torch.float32, device=dev)
-    out = {"break": torch.empty(slab, dtype=torch.int32, device=dev),
-           "magnitude": torch.empty(slab, dtype=torch.float32, device=dev)}
+    # the tile's map on rank 0's GPU, mapped by every rank
+    if rank == 0:
+        gmap = {"break": torch.full((P,), -7, dtype=torch.int32, device=dev),
+                "magnitude": torch.empty(P, dtype=torch.float32, device=dev)}
+        handles = [binding.ipc_export(gmap["break"]), binding.ipc_export(gmap["magnitude"])] if world > 1 else None
+        ptrs = [gmap["break"].data_ptr(), gmap["magnitude"].data_ptr()]
+    else:
+        handles = None
+    if world > 1:
+        box = [handles]
+        dist.broadcast_object_list(box, src=0)
+        if rank != 0:
+            ptrs = [binding.ipc_open(box[0][0], local), binding.ipc_open(box[0][1], local)]
     sampler = ClockSampler(local)
     sampler.start()
     time.sleep(0.6)
     total_ms, kernel_ms, launches = 0.0, 0.0, 0
+    last = None
     for s0 in range(b, e, slab):
         s1 = min(e, s0 + slab)
         synth.generate(spec, dev, columns=(s0, s1), out=Ybuf, ldY=slab)
         Y = Ybuf[:, : s1 - s0]  # [N][ldY = slab] view
-        o = {k: v[: s1 - s0] for k, v in out.items()}
+        o = {"break": ptrs[0] + 4 * s0, "magnitude": ptrs[1] + 4 * s0}
         with torch.cuda.stream(stream):
             for _ in range(args.warmup):
-                plan.execute(Y, P=s1 - s0, stream=stream, out=o)
+                plan.execute(Y, P=s1 - s0, stream=stream, out=o, check_out=False)
         torch.cuda.synchronize()
         binding.profile_enable(True)
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         sampler.mark(True) if sampler.t0 is None else None
         ev0.record(stream)
         for _ in range(args.steps):
-            plan.execute(Y, P=s1 - s0, stream=stream, out=o)
+            plan.execute(Y, P=s1 - s0, stream=stream, out=o, check_out=False)
             launches += binding.last_launch_count()
         ev1.record(stream)
         torch.cuda.synchronize()
@@ -269,6 +335,7 @@ def run_sharded_tile(args, spec, desc, world, rank, local, dev):
         binding.profile_enable(False)
         total_ms += ev0.elapsed_time(ev1) / args.steps
         kernel_ms += sum(kms) / max(len(kms), 1)
+        last = (s0, s1)
     sampler.mark(False)
     sampler.stop()
     if world > 1:
@@ -285,11 +352,43 @@ def run_sharded_tile(args, spec, desc, world, rank, local, dev):
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
             "config": {"workload": desc, "pixels_total": P, "pixels_per_gpu": e - b, "N": N,
                        "slab_pixels": slab, "l2": "inputs larger than L2, no flush",
-                       "parallelism": f"dp{world}: pixel shards of one tile, no collective"},
+                       "parallelism": f"dp{world}: pixel shards of one tile; the break map is gathered on "
+                                      f"rank 0's GPU by the kernels' own stores (CUDA IPC peer mapping)"},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": None, "kernel": "monitor_fused_kernel<8>",
+                         "frac": achieved / peak, "traffic": None, "kernel": f"monitor_fused_kernel<{2 + 2 * spec.k}>",
                          "kernel_ms_avg": kernel_ms, "peak_source": peak_src},
             "gpu_launches": launches, "clocks": sampler.summary()}
+    if world > 1:
+        dist.barrier()  # every rank's stores into rank 0's map are done
+    if rank == 0:
+        # the whole tile was written: no sentinel left in the map
+        line["gather_check"] = {"unwritten_pixels": int((gmap["break"] == -7).sum())}
+        if not args.no_cpu_baseline and last is not None:
+            # parity + oracle baseline on a sample of rank 0's last slab (its
+            # stack is still in the buffer), read back from the gathered map
+            from oracle import parity
+            s0, s1 = last
+            Y = Ybuf[:, : s1 - s0]
+            sub = synth.StackSpec(**{**spec.asdict(), "P": s1 - s0})
+            probe = 1 << 12
+            _, dt, threads, _ = oracle_sample(Y, dates, sub, probe, seed=7)
+            count = int(min(1 << 18, max(probe, probe * args.cpu_seconds / max(dt, 1e-3))))
+            orc, dt, threads, idx = oracle_sample(Y, dates, sub, count, seed=11)
+            it = torch.tensor(idx, device=dev) + s0
+            gpu = {"break": gmap["break"].index_select(0, it).cpu().numpy(),
+                   "magnitude": gmap["magnitude"].index_select(0, it).cpu().numpy()}
+            rep = parity.compare(gpu, orc)
+            line["cpu_baseline"] = cpu_baseline_entry(count / dt, threads,
+                                                      f"{count} uniformly sampled pixel columns of the tile's "
+                                                      f"last slab on rank 0, {dt:.1f} s")
+            line["parity_sample"] = {k: rep[k] for k in ("pixels", "ok", "break_mismatch",
+                                                         "break_mismatch_unexcused", "invalid_mismatch",
+                                                         "mag_fail", "mag_max_scaled_err")}
+    elif world > 1:
+        binding.ipc_close(ptrs[0])
+        binding.ipc_close(ptrs[1])
+    if world > 1:
+        dist.barrier()
     return _finish(line, world, rank)
 
 
@@ -429,7 +528,7 @@ def main():
     workload_key = f"{args.config}:P={P}:N={N}:k={rspec.k}"
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": achieved / peak, "traffic": ncu_traffic(workload_key),
-                "kernel": "monitor_fused_kernel<8>", "kernel_ms_avg": k_avg,
+                "kernel": f"monitor_fused_kernel<{2 + 2 * rspec.k}>", "kernel_ms_avg": k_avg,
                 "kernel_share_of_step": k_avg / ms_step if ms_step else None,
                 "alg_bytes_per_launch": alg_bytes, "peak_source": peak_src}
 
@@ -454,9 +553,10 @@ def main():
         gpu = {"break": out["break"].index_select(0, it).cpu().numpy(),
                "magnitude": out["magnitude"].index_select(0, it).cpu().numpy()}
         rep = parity.compare(gpu, orc)
-        line["cpu_baseline"] = {"value": count / dt, "unit": UNIT, "cores": threads, "kind": "oracle",
-                                "sample": f"{count} uniformly sampled pixel columns of the same scene, "
-                                          f"{dt:.1f} s"}
+        measure_one_thread(Y, dates, rspec)
+        line["cpu_baseline"] = cpu_baseline_entry(count / dt, threads,
+                                                  f"{count} uniformly sampled pixel columns of the same scene, "
+                                                  f"{dt:.1f} s")
         line["parity_sample"] = {k: rep[k] for k in ("pixels", "ok", "break_mismatch",
                                                      "break_mismatch_unexcused", "invalid_mismatch",
                                                      "mag_fail", "mag_max_scaled_err")}
