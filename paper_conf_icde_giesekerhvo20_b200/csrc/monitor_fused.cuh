@@ -28,20 +28,21 @@
 //   pass C  monitoring yhat = X beta, r = y - yhat, MOSUM recurrence over the
 //                      ring, boundary, first break, mean       L518-L537
 //
-// Roles.  A CTA owns T tiles (4 warps each, T*128 pixels) and loops over
-// tile groups.  There is no producer or MMA-issuer warp:
-//  - each warp streams its own [8 dates x 32 px] boxes of the stack by 2-D
-//    TMA into a private ring of half-chunk stages, refilling a stage as soon
-//    as its values have been consumed, and prefetches the first-touch
-//    boxes (passes A and C) into L2 a few chunks ahead;
-//  - every chunk is one "group": each warp publishes its part (operands
-//    written to TMEM, or the yhat slot read) with one shared-memory atomic,
-//    and the LAST warp to publish issues the group's tcgen05.mma for all T
-//    tiles (after checking the previous group completed: the accumulate
-//    chains and the table stages are ordered by completion, not by issue)
-//    and the bulk copy of the table the chunk ST-1 ahead needs;
+// Roles.  One persistent CTA per SM = a control warpgroup (warps 0-3) and T
+// consumer warpgroups (T = FzShape::TMAX tiles of 128 pixels, by registers);
+// the CTA loops over tile groups of T * 128 pixels.
+//  - control warp i drives tile i in the tile's fixed event order: when the
+//    tile's 4 consumer warps release a stack stage (mbarrier srel) it loads
+//    the chunk SC ahead -- one [16 dates x 128 px] 2-D TMA box (8 KB) into
+//    that stage, plus an L2 prefetch of first-touch dates pfd ahead; when
+//    they publish a chunk's operands (mbarrier pub) it issues the chunk's
+//    tcgen05.mma (one elected lane) and commits them to mdone / ybar.  Its
+//    waits sleep in hardware (try_wait + suspend hint);
+//  - the consumers only compute: per date registers, per chunk tcgen05.st /
+//    tcgen05.ld of TMEM operands and accumulators;
 //  - all B-operand tables (fixed functions of the dates, L2-resident) stream
-//    through one ST-stage ring shared by the T tiles.
+//    through one ST-stage ring shared by the T tiles; a stage is reloaded by
+//    the last tile to be done with it, two chunks after its use.
 // The stack is read through tensor maps whose out-of-bounds fill is NaN, so
 // ragged tiles and the partial last chunk of each period need no special case.
 #pragma once
