@@ -66,6 +66,11 @@ def spec_for(name: str):
                      "k=3, h=0.25, lambda=1.65, 50% NaN i.i.d.; pixel shards over the GPUs (strong scaling)",
         "stream": "continental streaming (BASELINE configs[4]): Landsat-shaped tiles (4096x4096 px x N=400, "
                   "60% cloud) from pinned host memory through the e2e path, H2D double-buffered",
+        "dense": "SURVEY 8(f) f3: Landsat-shaped scene (4096x4096 px x N=400, n_hist=200, k=3) with a complete "
+                 "history (the NaN-free case of L93), 60% cloud gaps in the monitoring period only",
+        "africa": "SURVEY 8(f) f2: 2^23 px x 2000 dates (n_hist=1000, k=3), 88% of the date slices empty "
+                  "(Africa: ~350 of 6873 dates hold data, L379), 50% NaN i.i.d. in the others; step = scan for "
+                  "empty slices + gather of the kept ones + the hot path on the compacted stack",
     }[name]
     return spec, desc
 
@@ -443,6 +448,112 @@ def run_stream(args, spec, desc, world, rank, local, dev):
     return _finish(line, world, rank)
 
 
+def run_africa(args, spec, desc, world, rank, local, dev):
+    """the preprocessing step of the paper's pipeline (drop
+    the date slices holding no value, L291/L379) followed by the hot path on
+    the compacted stack, per step; rank-local scenes (weak scaling)."""
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    from paper_conf_icde_giesekerhvo20_b200 import binding, synth
+    rspec = synth.StackSpec(**{**spec.asdict(), "seed": spec.seed + 1000 * rank})
+    Y, dates = synth.generate(rspec, dev)
+    P, N = rspec.P, rspec.N
+    stream = torch.cuda.Stream(device=dev)
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
+    res = {}
+
+    def step(timed=False):
+        if timed:
+            ev[0].record(stream)
+        keep = binding.bfast_valid_dates(Y, stream=stream)
+        if timed:
+            ev[1].record(stream)
+        stream.synchronize()
+        kh = keep.cpu().numpy()
+        keep_idx = np.flatnonzero(kh)
+        idx = torch.from_numpy(keep_idx.astype(np.int32)).to(dev, non_blocking=False)
+        Yc = binding.bfast_gather_dates(Y, idx, stream=stream)
+        if timed:
+            ev[2].record(stream)
+        nc = int(np.count_nonzero(keep_idx < rspec.n_hist))
+        out = binding.bfast_monitor_ex(Yc, dates[keep_idx], nc, rspec.k, rspec.hf, rspec.lam, stream=stream)
+        if timed:
+            ev[3].record(stream)
+        res.update(out=out, keep_idx=keep_idx, nc=nc, Yc=Yc)
+
+    with torch.cuda.stream(stream):
+        for _ in range(args.warmup):
+            step()
+    torch.cuda.synchronize()
+    sampler = ClockSampler(local)
+    sampler.start()
+    time.sleep(0.6)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    sampler.mark(True)
+    scan, gather, mon, tot = [], [], [], []
+    launches = 0
+    with torch.cuda.stream(stream):
+        for _ in range(args.steps):
+            step(timed=True)
+            launches += 3 + binding.last_launch_count() - 1
+            torch.cuda.synchronize()
+            scan.append(ev[0].elapsed_time(ev[1]))
+            gather.append(ev[1].elapsed_time(ev[2]))
+            mon.append(ev[2].elapsed_time(ev[3]))
+            tot.append(ev[0].elapsed_time(ev[3]))
+    sampler.mark(False)
+    sampler.stop()
+    t = torch.tensor([sum(tot)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.barrier()
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_step = float(t.item()) / args.steps
+    Nc = len(res["keep_idx"])
+    empty = N - Nc
+    peak, peak_src = load_peaks()
+    s_ms = sum(scan) / len(scan)
+    g_ms = sum(gather) / len(gather)
+    scan_bytes = empty * P * 4  # every empty slice is read in full (a slice with data stops at its first value)
+    gather_bytes = 2 * Nc * P * 4
+    roofline = {"bound": "hbm", "achieved": scan_bytes / (s_ms / 1e3) / 1e9, "peak": peak, "unit": "GB/s",
+                "frac": scan_bytes / (s_ms / 1e3) / 1e9 / peak, "traffic": None, "kernel": "slice_any_kernel",
+                "kernel_ms_avg": s_ms, "kernel_share_of_step": s_ms / ms_step, "alg_bytes_per_launch": scan_bytes,
+                "peak_source": peak_src,
+                "gather": {"kernel": "gather_dates_kernel", "ms": g_ms, "bytes": gather_bytes,
+                           "GB/s": gather_bytes / (g_ms / 1e3) / 1e9},
+                "monitor_ms": sum(mon) / len(mon)}
+    line = {"metric": METRIC, "value": P * world / (ms_step / 1e3), "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": desc, "pixels_per_gpu": P, "N_raw": N, "N_kept": Nc, "n_hist_kept": res["nc"],
+                       "k": rspec.k, "l2": "inputs larger than L2 (%.1f GB stack), no flush" % (4 * N * P / 1e9),
+                       "parallelism": f"dp{world}: pixel shards, no collective"},
+            "roofline": roofline, "gpu_launches": launches, "clocks": sampler.summary()}
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        from oracle import parity
+        Yc = res["Yc"]
+        orc, dt, threads, idx = oracle_sample(Yc, dates[res["keep_idx"]],
+                                              synth.StackSpec(**{**rspec.asdict(), "N": Nc, "n_hist": res["nc"]}),
+                                              1 << 16, seed=5)
+        it = torch.tensor(idx, device=dev)
+        gpu = {"break": res["out"]["break"].index_select(0, it).cpu().numpy(),
+               "magnitude": res["out"]["magnitude"].index_select(0, it).cpu().numpy()}
+        rep = parity.compare(gpu, orc)
+        line["parity_sample"] = {k: rep[k] for k in ("pixels", "ok", "break_mismatch", "invalid_mismatch",
+                                                     "mag_fail", "mag_max_scaled_err")}
+        # the kept-date list against its plain definition over the whole scene (a slice is kept iff it
+        # holds any value), evaluated row block by row block
+        ref = torch.cat([~torch.isnan(Y[r:r + 64]).all(dim=1) for r in range(0, N, 64)]).cpu().numpy()
+        line["parity_sample"]["keep_list_exact"] = bool(np.array_equal(np.flatnonzero(ref), res["keep_idx"]))
+        line["parity_sample"]["ok"] = bool(line["parity_sample"]["ok"] and line["parity_sample"]["keep_list_exact"])
+        line["cpu_baseline"] = cpu_baseline_entry(len(idx) / dt, threads,
+                                                  f"{len(idx)} sampled columns of the compacted stack, {dt:.1f} s")
+    return _finish(line, world, rank)
+
+
 def main():
     args = parse()
     if args.impl == "reference":
@@ -467,6 +578,8 @@ def main():
         return run_sharded_tile(args, spec, desc, world, rank, local, dev)
     if args.config == "stream":
         return run_stream(args, spec, desc, world, rank, local, dev)
+    if args.config == "africa":
+        return run_africa(args, spec, desc, world, rank, local, dev)
     # each rank: its own scene of the configured shape (weak scaling); seed per rank
     rspec = synth.StackSpec(**{**spec.asdict(), "seed": spec.seed + 1000 * rank})
     Y, dates = synth.generate(rspec, dev)
@@ -531,6 +644,23 @@ def main():
                 "kernel": f"monitor_fused_kernel<{2 + 2 * rspec.k}>", "kernel_ms_avg": k_avg,
                 "kernel_share_of_step": k_avg / ms_step if ms_step else None,
                 "alg_bytes_per_launch": alg_bytes, "peak_source": peak_src}
+
+    if args.config == "dense":
+        # f3 A/B on the same scene: the shared fp64 factor vs every pixel factoring its own Gram
+        ab = {}
+        for key, val in (("per_pixel_factor", "0"), ("shared_factor", "1")):
+            os.environ["BFAST_SHARED_FACTOR"] = val
+            with torch.cuda.stream(stream):
+                step()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            for _ in range(5):
+                step()
+            e1.record(stream)
+            torch.cuda.synchronize()
+            ab[key + "_ms_per_step"] = e0.elapsed_time(e1) / 5
+        os.environ.pop("BFAST_SHARED_FACTOR", None)
+        roofline["f3_ab"] = ab
 
     clocks = sampler.summary()
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,

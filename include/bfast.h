@@ -205,6 +205,57 @@ int bfast_monitor_shards(const float *const *Y_dev, const int64_t *P, const int6
                          int32_t *out_break, float *out_magnitude);
 
 /*
+ * ---- Preprocessing before the hot path --------------
+ * after a chunk is copied to the GPU, "removal of slices only
+ * containing NaN values"; L379: a Landsat image of Africa spans 6873 dates
+ * of which only about 350 slices contain any data, and they "are extracted
+ * efficiently before applying the core algorithm".  The monitoring entries
+ * never renumber dates (reading R13); these two calls do it explicitly.
+ * The caller then runs bfast_monitor* on the compacted stack with the kept
+ * dates and n_hist' = #kept dates < n_hist (the trend regressor is then
+ * the 1-based index in the compacted stack, as in the paper's pipeline); a
+ * break offset b >= 0 maps back to the original date keep_idx[n_hist' + b].
+ *
+ * bfast_valid_dates -- keep[t] = 1 iff some pixel p < P of date slice t of
+ * the DEVICE stack Y (float32 [N][ldY], NaN = missing, any payload) holds
+ * a value, else 0.  keep: device int32[N].  Asynchronous on `stream`
+ * (NULL = legacy default stream).  A slice stops being read once a value
+ * is found, so the cost is about one 32 KB segment per slice with data and
+ * the whole slice (4 P bytes) per empty one.  Errors: BFAST_EINVAL (N < 0,
+ * P < 0, ldY < P, NULL pointer); BFAST_EUNSUPPORTED (N > 2^31 - 1 or P >
+ * 2^29); nothing is written on error.
+ */
+int bfast_valid_dates(const float *Y, int64_t N, int64_t P, int64_t ldY, int32_t *keep, void *stream);
+
+/*
+ * bfast_gather_dates -- Yc[i][p] = Y[idx[i]][p] for i < Nc, p < P: the
+ * kept slices (idx: device int32[Nc], values in [0, N), normally
+ * increasing) as a compact DEVICE stack Yc float32 [Nc][ldYc].  Y and Yc
+ * must not overlap.  Asynchronous on `stream`.  Errors: BFAST_EINVAL (P <
+ * 0, Nc < 0, ldY < P, ldYc < P, NULL pointer); BFAST_EUNSUPPORTED (Nc >
+ * 65535).
+ */
+int bfast_gather_dates(const float *Y, int64_t ldY, int64_t P, const int32_t *idx, int64_t Nc, float *Yc,
+                       int64_t ldYc, void *stream);
+
+/*
+ * bfast_monitor_host_resume -- a scene streamed tile by tile with
+ * tile-level resume (the paper splits scenes that do
+ * not fit in memory into chunks on the host, L291).  Processes the pixels
+ * [*done, P) of the HOST stack (arguments as bfast_monitor_host) in tiles
+ * of `tile` pixels, at most `max_tiles` of them (< 0: all), and advances
+ * *done past each tile whose results are in the host arrays.  A call that
+ * returns early (error, interruption, max_tiles) is resumed by calling it
+ * again with the same *done; the results are identical to one
+ * uninterrupted call.  Errors: as bfast_monitor_host, plus BFAST_EINVAL for
+ * done == NULL, *done outside [0, P] or tile < 1.
+ */
+int bfast_monitor_host_resume(const float *Y_host, int64_t N, int64_t P, int64_t ldY,
+                              const double *dates, int32_t n_hist, int32_t k, float h,
+                              float lambda, int32_t *out_break_host, float *out_magnitude_host,
+                              int device, int64_t tile, int64_t max_tiles, int64_t *done);
+
+/*
  * Cross-process break-map gather (one process per GPU, torchrun): the
  * process owning the map exports its device allocation as a CUDA IPC
  * handle of BFAST_IPC_HANDLE_BYTES bytes; every other process opens it and

@@ -166,3 +166,19 @@ def mosum(rbar, nbar, Nbar, h, sigma):
     m = np.empty(max(Nbar - nbar, 0), np.float64)
     _load().oracle_mosum(_ptr(rbar), int(nbar), int(Nbar), int(h), float(sigma), _ptr(m))
     return m
+
+
+def drop_empty_dates(Y, dates, n_hist, P: int | None = None):
+    """PAPER.md L291 ("removal of slices only containing
+    NaN values", a preprocessing step after each chunk reaches the GPU) and
+    L379 (about 350 of 6873 Africa dates hold any data).  Plain definition:
+    slice t is kept iff some pixel p < P has y[t, p] == y[t, p] (not NaN, any
+    payload, reading R9); the kept slices in their original order, their
+    dates, and n_hist' = the number of kept dates before n_hist (the history
+    of the compacted stack).  Returns (Yc, dates_c, n_hist_c, keep_idx)."""
+    Y = np.asarray(Y)
+    P = Y.shape[1] if P is None else int(P)
+    keep_idx = np.flatnonzero(~np.all(np.isnan(Y[:, :P]), axis=1))
+    d = np.asarray(dates, dtype=np.float64)
+    return (np.ascontiguousarray(Y[keep_idx, :P]), d[keep_idx],
+            int(np.count_nonzero(keep_idx < int(n_hist))), keep_idx)

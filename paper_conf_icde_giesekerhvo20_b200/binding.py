@@ -30,7 +30,8 @@ EXPORTS = ("bfast_monitor", "bfast_monitor_ex", "bfast_plan_create", "bfast_plan
            "bfast_ipc_export", "bfast_ipc_open", "bfast_ipc_close",
            "bfast_shard_range", "bfast_last_launch_count", "bfast_last_error",
            "bfast_status_string", "bfast_abi_version", "bfast_profile_enable",
-           "bfast_profile_collect")
+           "bfast_profile_collect", "bfast_valid_dates", "bfast_gather_dates",
+           "bfast_monitor_host_resume")
 IPC_HANDLE_BYTES = 72
 
 
@@ -89,6 +90,13 @@ def lib():
         L.bfast_abi_version.restype = I
         L.bfast_profile_enable.argtypes = [I]
         L.bfast_profile_enable.restype = I
+        L.bfast_valid_dates.argtypes = [V, i64, i64, i64, V, V]
+        L.bfast_valid_dates.restype = I
+        L.bfast_gather_dates.argtypes = [V, i64, i64, V, i64, V, i64, V]
+        L.bfast_gather_dates.restype = I
+        L.bfast_monitor_host_resume.argtypes = [V, i64, i64, i64, V, i32, i32, f32, f32, V, V, I, i64, i64,
+                                                ctypes.POINTER(i64)]
+        L.bfast_monitor_host_resume.restype = I
         L.bfast_profile_collect.argtypes = [V, I]
         L.bfast_profile_collect.restype = I
         _lib = L
@@ -299,6 +307,74 @@ def bfast_monitor_host(Y_host, dates, n_hist, k, h, lam, out_break=None, out_mag
                                     float(h), float(lam), _host_ptr(out_break), _host_ptr(out_magnitude),
                                     int(device)))
     return out_break, out_magnitude
+
+
+def bfast_monitor_host_resume(Y_host, dates, n_hist, k, h, lam, out_break, out_magnitude, done=0,
+                              tile=1 << 22, max_tiles=-1, P=None, device=-1) -> int:
+    """Tile-by-tile host streaming with resume (f2): processes pixels
+    [done, P) in tiles, at most max_tiles of them; returns the new `done`
+    (pass it back to resume).  out_break / out_magnitude: host arrays [P]."""
+    N, ldY = int(Y_host.shape[0]), int(Y_host.shape[1])
+    P = ldY if P is None else int(P)
+    d = _dates(dates)
+    dn = ctypes.c_int64(int(done))
+    _check(lib().bfast_monitor_host_resume(_host_ptr(Y_host), N, P, ldY, d.ctypes.data, int(n_hist), int(k),
+                                           float(h), float(lam), _host_ptr(out_break), _host_ptr(out_magnitude),
+                                           int(device), int(tile), int(max_tiles), ctypes.byref(dn)))
+    return int(dn.value)
+
+
+def bfast_valid_dates(Y, P=None, stream=None):
+    """f2 scan (L291, L379): int32 device tensor keep[N], 1 where the date
+    slice holds any value among pixels [0, P)."""
+    import torch
+    _check_stack(Y)
+    N, ldY = int(Y.shape[0]), int(Y.shape[1])
+    P = ldY if P is None else int(P)
+    keep = torch.empty(N, dtype=torch.int32, device=Y.device)
+    with torch.cuda.device(Y.device):
+        _check(lib().bfast_valid_dates(_dptr(Y), N, P, ldY, _dptr(keep), _stream_ptr(stream)))
+    return keep
+
+
+def bfast_gather_dates(Y, idx, P=None, stream=None):
+    """f2 gather: the slices idx (int32 device tensor) of Y as a compact
+    [len(idx)][P] device stack."""
+    import torch
+    _check_stack(Y)
+    ldY = int(Y.shape[1])
+    P = ldY if P is None else int(P)
+    assert idx.dtype == torch.int32 and idx.device == Y.device
+    Yc = torch.empty((int(idx.numel()), P), dtype=torch.float32, device=Y.device)
+    with torch.cuda.device(Y.device):
+        _check(lib().bfast_gather_dates(_dptr(Y), ldY, P, _dptr(idx), int(idx.numel()), _dptr(Yc), P,
+                                        _stream_ptr(stream)))
+    return Yc
+
+
+def drop_empty_dates(Y, dates, n_hist, P=None):
+    """f2 as the paper's pipeline runs it (L291): scan, then gather the
+    slices holding any value.  Returns (Yc, dates_c, n_hist_c, keep_idx):
+    the compact stack, its dates, the number of kept history dates and the
+    original index of every kept date (host int64)."""
+    import torch
+    keep = bfast_valid_dates(Y, P).cpu().numpy()
+    keep_idx = np.flatnonzero(keep).astype(np.int64)
+    idx = torch.from_numpy(keep_idx.astype(np.int32)).to(Y.device)
+    Yc = bfast_gather_dates(Y, idx, P)
+    d = _dates(dates)
+    return Yc, d[keep_idx], int(np.count_nonzero(keep_idx < int(n_hist))), keep_idx
+
+
+def original_break_offsets(brk, keep_idx, n_hist_c, n_hist):
+    """Break offsets on a compacted stack (relative to its monitoring start)
+    as offsets from the original monitoring start: keep_idx[n_c + b] - n;
+    -1 / -2 unchanged (index mapping only)."""
+    b = np.asarray(brk)
+    out = b.copy()
+    hit = b >= 0
+    out[hit] = np.asarray(keep_idx)[int(n_hist_c) + b[hit]] - int(n_hist)
+    return out
 
 
 def bfast_monitor_multi(Y_host, dates, n_hist, k, h, lam, devices, out_break=None, out_magnitude=None,

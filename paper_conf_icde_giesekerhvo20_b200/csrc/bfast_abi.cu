@@ -22,6 +22,7 @@
 #include "monitor_simt.cuh"
 #include "monitor_fused.cuh"
 #include "refit_fp64.cuh"
+#include "preprocess.cuh"
 
 namespace {
 
@@ -107,6 +108,11 @@ struct bfast_plan {
   // fused kernel (monitor_fused.cuh): per-chunk tables of passes A, B, C
   uint8_t *dtabf = nullptr;
   size_t tabfB_off = 0, tabfC_off = 0;
+  // NaN-free history: the Cholesky factor of the
+  // common Gram sum_{t<n} x_t x_t^T, fp64 on the host, in the kernel's
+  // register layout (FzTables::shared); nullptr when the history Gram is
+  // singular
+  float *dshared = nullptr;
   int nch = 0, ncm = 0;
   int mode = 0;  // 0 fused tensor-core kernel, 1 SIMT kernel only (BFAST_KERNEL=simt at plan creation)
   std::mutex mu;
@@ -119,6 +125,7 @@ struct bfast_plan {
     cudaFree(dcount);
     cudaFree(dlist);
     cudaFree(dtabf);
+    cudaFree(dshared);
     if (scratch_free) cudaEventDestroy(scratch_free);
     for (int i = 0; i < 2; ++i) {
       cudaFree(host.dY[i]);
@@ -301,7 +308,71 @@ void build_fz_tables(const bfast_plan &pl, std::vector<uint16_t> &tab, size_t &o
   }
 }
 
+// f3 (the [27] special case): every pixel whose
+// history has no missing value shares the Gram A = sum_{t<n} x_t x_t^T, so
+// its factor is computed once: Cholesky in fp64, rounded to fp32 in the
+// layout fz_chol leaves (Tri<K>: idx(j, j) = A_jj, idx(q, i) = L_iq for q <
+// i), then the K reciprocal pivots, the smallest pivot ratio d_j / A_jj and
+// the largest variance inflation factor A_jj (A^-1)_jj (the fused kernel's
+// fp64-refit triggers, here exact).  Returns false if A is not positive
+// definite (the kernel then factors every pixel itself).
+bool shared_factor(const bfast_plan &pl, std::vector<float> &out) {
+  const int K = pl.K;
+  std::vector<float> Xf;
+  std::vector<double> X64;
+  build_design(pl, Xf, X64);
+  std::vector<double> A((size_t)K * K, 0.0), L((size_t)K * K, 0.0);
+  for (int t = 0; t < pl.n; ++t)
+    for (int i = 0; i < K; ++i)
+      for (int j = 0; j < K; ++j) A[i * K + j] += X64[(size_t)t * K + i] * X64[(size_t)t * K + j];
+  double minratio = 1.0;
+  for (int j = 0; j < K; ++j) {
+    double d = A[j * K + j];
+    for (int q = 0; q < j; ++q) d -= L[j * K + q] * L[j * K + q];
+    if (!(d > 0.0)) return false;
+    minratio = std::min(minratio, d / A[j * K + j]);
+    L[j * K + j] = std::sqrt(d);
+    for (int i = j + 1; i < K; ++i) {
+      double v = A[j * K + i];
+      for (int q = 0; q < j; ++q) v -= L[i * K + q] * L[j * K + q];
+      L[i * K + j] = v / L[j * K + j];
+    }
+  }
+  // (A^-1)_jj = sum_i (L^-1)_ij^2
+  double vif = 0.0;
+  for (int j = 0; j < K; ++j) {
+    std::vector<double> m(K, 0.0);
+    m[j] = 1.0 / L[j * K + j];
+    double ss = m[j] * m[j];
+    for (int i = j + 1; i < K; ++i) {
+      double v = 0.0;
+      for (int q = j; q < i; ++q) v += L[i * K + q] * m[q];
+      m[i] = -v / L[i * K + i];
+      ss += m[i] * m[i];
+    }
+    vif = std::max(vif, ss * A[j * K + j]);
+  }
+  const int kN = K * (K + 1) / 2;
+  out.assign((size_t)kN + K + 2, 0.f);
+  auto tri = [&](int i, int j) { return i * K - i * (i - 1) / 2 + (j - i); };  // Tri<K>::idx, i <= j
+  for (int j = 0; j < K; ++j) {
+    out[tri(j, j)] = (float)A[j * K + j];
+    for (int i = j + 1; i < K; ++i) out[tri(j, i)] = (float)L[i * K + j];
+    out[kN + j] = (float)(1.0 / L[j * K + j]);
+  }
+  out[kN + K] = (float)minratio;
+  out[kN + K + 1] = (float)vif;
+  return true;
+}
+
 int build_fz(bfast_plan &pl) {
+  {
+    std::vector<float> sf;
+    if (shared_factor(pl, sf)) {
+      CUDA_TRY(cudaMalloc(&pl.dshared, sf.size() * sizeof(float)));
+      CUDA_TRY(cudaMemcpy(pl.dshared, sf.data(), sf.size() * sizeof(float), cudaMemcpyHostToDevice));
+    }
+  }
   std::vector<uint16_t> tab;
   size_t ob = 0, oc = 0;
   switch (pl.k) {
@@ -380,6 +451,9 @@ int launch_fused(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStre
   tb.tabA = pl.dtabf;
   tb.tabB = pl.dtabf + pl.tabfB_off;
   tb.tabC = pl.dtabf + pl.tabfC_off;
+  // BFAST_SHARED_FACTOR=0: every pixel factors its own Gram (A/B of f3)
+  const char *sfe = std::getenv("BFAST_SHARED_FACTOR");
+  tb.shared = (sfe && sfe[0] == '0') ? nullptr : pl.dshared;
   tb.nch = pl.nch;
   tb.ncm = pl.ncm;
   tb.T = T;
@@ -900,6 +974,67 @@ int bfast_monitor_multi(const float *Y_host, int64_t N, int64_t P, int64_t ldY, 
     total += launches[r];
   }
   g_launches = total;
+  return BFAST_OK;
+}
+
+// ---- f2: host-pipeline preprocessing -----------------
+int bfast_valid_dates(const float *Y, int64_t N, int64_t P, int64_t ldY, int32_t *keep, void *stream) {
+  if (N < 0 || P < 0 || ldY < P) return fail(BFAST_EINVAL, "N < 0, P < 0 or ldY < P");
+  if (N == 0) {
+    g_launches = 0;
+    return BFAST_OK;
+  }
+  if (!keep || (P > 0 && !Y)) return fail(BFAST_EINVAL, "NULL pointer");
+  const int64_t nseg = (P + bfast::kScanSeg - 1) / bfast::kScanSeg;
+  if (N > 0x7fffffff || nseg > 65535) return fail(BFAST_EUNSUPPORTED, "stack too large for one scan");
+  cudaStream_t st = (cudaStream_t)stream;
+  CUDA_TRY(cudaMemsetAsync(keep, 0, sizeof(int32_t) * N, st));
+  g_launches = 0;
+  if (P == 0) return BFAST_OK;
+  const int vec4 = (ldY % 4 == 0) && ((uintptr_t)Y % 16 == 0);
+  bfast::slice_any_kernel<<<dim3((unsigned)N, (unsigned)nseg), bfast::kScanThreads, 0, st>>>(Y, P, ldY, keep, vec4);
+  CUDA_TRY(cudaGetLastError());
+  g_launches = 1;
+  return BFAST_OK;
+}
+
+int bfast_gather_dates(const float *Y, int64_t ldY, int64_t P, const int32_t *idx, int64_t Nc, float *Yc,
+                       int64_t ldYc, void *stream) {
+  if (P < 0 || Nc < 0 || ldY < P || ldYc < P) return fail(BFAST_EINVAL, "P < 0, Nc < 0, ldY < P or ldYc < P");
+  g_launches = 0;
+  if (P == 0 || Nc == 0) return BFAST_OK;
+  if (!Y || !idx || !Yc) return fail(BFAST_EINVAL, "NULL pointer");
+  if (Nc > 65535) return fail(BFAST_EUNSUPPORTED, "Nc=%lld > 65535", (long long)Nc);
+  const int vec4 = (ldY % 4 == 0) && (ldYc % 4 == 0) && ((uintptr_t)Y % 16 == 0) && ((uintptr_t)Yc % 16 == 0);
+  int dev = 0, sms = 148;
+  CUDA_TRY(cudaGetDevice(&dev));
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  // about 8 resident blocks per SM over all rows
+  const int64_t per_row = std::max<int64_t>(1, std::min<int64_t>((P / (vec4 ? 4 : 1) + 255) / 256,
+                                                               std::max<int64_t>(1, 8 * sms / Nc)));
+  bfast::gather_dates_kernel<<<dim3((unsigned)per_row, (unsigned)Nc), 256, 0, (cudaStream_t)stream>>>(
+      Y, ldY, P, idx, Yc, ldYc, vec4);
+  CUDA_TRY(cudaGetLastError());
+  g_launches = 1;
+  return BFAST_OK;
+}
+
+int bfast_monitor_host_resume(const float *Y_host, int64_t N, int64_t P, int64_t ldY, const double *dates,
+                              int32_t n_hist, int32_t k, float h, float lambda, int32_t *out_break_host,
+                              float *out_magnitude_host, int device, int64_t tile, int64_t max_tiles,
+                              int64_t *done) {
+  if (!done || *done < 0 || *done > P || tile < 1)
+    return fail(BFAST_EINVAL, "done NULL or outside [0, P], or tile < 1");
+  int launches = 0;
+  for (int64_t t = 0; *done < P && (max_tiles < 0 || t < max_tiles); ++t) {
+    const int64_t b = *done, w = std::min(tile, P - b);
+    const int rc = bfast_monitor_host(Y_host + b, N, w, ldY, dates, n_hist, k, h, lambda, out_break_host + b,
+                                      out_magnitude_host + b, device);
+    if (rc) return rc;
+    launches += g_launches;
+    *done = b + w;  // the tile's results are in the host arrays
+  }
+  g_launches = launches;
   return BFAST_OK;
 }
 

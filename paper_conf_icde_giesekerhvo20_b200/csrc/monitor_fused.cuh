@@ -136,6 +136,9 @@ struct FzTables {
   int pfd;                            // L2 prefetch distance in dates (multiple of FzCfg::PFB; 0: off)
   int sc;                             // stack chunk stages per tile (2..FzCfg::SCMAX)
   int64_t ntg;                        // tile groups of T * 128 pixels
+  // NaN-free history (f3): the common Cholesky factor, [Tri<K>::kN | dinv K |
+  // min pivot ratio | max VIF] (bfast_abi.cu shared_factor); nullptr = off
+  const float *shared;
 };
 
 #ifndef BFAST_FZ_CTLWAIT
@@ -924,10 +927,24 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
       float diagA[K];
 #pragma unroll
       for (int i = 0; i < K; ++i) diagA[i] = A[Tri<K>::idx(i, i)];
-      const float minratio = fz_chol<K>(A, dinv);
+      // f3 (L93): a warp whose 32 histories have no missing value shares
+      // one Gram, factored once on the host in fp64: beta0 = A^-1 (X_hist^T
+      // y'), the moment b being the tensor-core GEMM of pass A
+      const bool dense = tb.shared != nullptr && __all_sync(0xffffffffu, nbar == n);
+      float minratio, vif = 0.f;
+      if (dense) {
+#pragma unroll
+        for (int i = 0; i < Tri<K>::kN; ++i) A[i] = __ldg(tb.shared + i);
+#pragma unroll
+        for (int i = 0; i < K; ++i) dinv[i] = __ldg(tb.shared + Tri<K>::kN + i);
+        minratio = __ldg(tb.shared + Tri<K>::kN + K);
+        vif = __ldg(tb.shared + Tri<K>::kN + K + 1);
+      } else {
+        minratio = fz_chol<K>(A, dinv);
+      }
       fz_solve<K>(A, dinv, b, beta);
       if (!deg && !(minratio >= (float)kRefitRatio)) refit = true;
-      if (!deg && !refit && !(fz_vif_max<K>(A, dinv, diagA) <= kRefitVif)) refit = true;
+      if (!deg && !refit && !((dense ? vif : fz_vif_max<K>(A, dinv, diagA)) <= kRefitVif)) refit = true;
       if (deg || !have) {
 #pragma unroll
         for (int i = 0; i < K; ++i) beta[i] = 0.f;

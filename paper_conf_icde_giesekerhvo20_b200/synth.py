@@ -46,6 +46,8 @@ class StackSpec:
     seed: int = 1
     noise_lo: float = 0.01
     noise_hi: float = 0.05
+    dense_hist: bool = False   # no missing value before n_hist (the NaN-free case of L93)
+    empty_frac: float = 0.0    # share of date slices with no value at all (L379; drawn per date)
 
     def asdict(self):
         return asdict(self)
@@ -59,6 +61,15 @@ CONFIGS = {
                          break_frac=0.1, seed=2),
     "sentinel2": StackSpec(P=10980 * 10980, N=700, n_hist=350, miss=0.5, mask="iid",
                            f=73.0, year0=2016.0, break_frac=0.1, seed=4),
+    # the Landsat scene with a complete history (the [27]
+    # special case, L93); gaps (60% cloud) only in the monitoring period
+    "dense": StackSpec(P=4096 * 4096, N=400, n_hist=200, miss=0.6, mask="cloud",
+                       break_frac=0.1, seed=6, dense_hist=True),
+    # a dated cube in which most slices hold no value at all
+    # (Africa: ~350 of 6873 dates per image, L379): 2000 dates at 16 days
+    # (f = 23), 88% of them empty, 50% i.i.d. gaps in the others
+    "africa": StackSpec(P=1 << 23, N=2000, n_hist=1000, miss=0.5, mask="iid",
+                        break_frac=0.1, seed=7, empty_frac=0.88),
 }
 
 
@@ -158,13 +169,19 @@ def generate(spec: StackSpec, device="cpu", ldY: int | None = None, out: torch.T
             blkv -= delta[None, :] * (tidx[c0:c1, None] >= t0[None, :])
             if spec.mask == "iid":
                 miss = torch.rand(c1 - c0, nb, generator=gcn, device=dev) < spec.miss
+                if spec.dense_hist:
+                    miss[: max(0, min(c1, spec.n_hist) - c0)] = False
                 blkv.masked_fill_(miss, float("nan"))
             elif spec.mask == "cloud":
-                for t in range(c0, c1):
+                for t in range(max(c0, spec.n_hist) if spec.dense_hist else c0, c1):
                     field, thr = _cloud_rows(H, Wd, P, spec.seed, t, float(cover[t]), pb, pe, dev)
                     blkv[t - c0].masked_fill_(field < thr, float("nan"))
             elif spec.mask != "none":
                 raise ValueError(spec.mask)
+            if spec.empty_frac > 0:
+                ge = _gen(dev, spec.seed, 4)
+                empty = torch.rand(N, generator=ge, device=dev) < spec.empty_frac
+                blkv[empty[c0:c1]] = float("nan")
             Y[c0:c1, sb - b0:se - b0] = blkv[:, sl]
             del blkv
     if ldY > W_:

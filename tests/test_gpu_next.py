@@ -1,0 +1,149 @@
+"""GPU parity of the SURVEY.md 8(f) NEXT rows built in round 2.
+
+f3  NaN-free histories share one Gram (the [27] special case):
+    its factor is computed once on the host in fp64; every warp whose 32
+    histories are complete skips its own factorisation.
+f2  all-NaN date slices dropped before the hot path (L291, L379): the scan
+    and gather kernels, bit-exact against numpy, and the monitoring result on
+    the compacted stack against the oracle on the same compacted stack.
+
+Every case compares the CUDA path (through the C ABI) with the fp64 oracle on
+the same device bytes (oracle/parity.py tolerances).
+"""
+import json
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+import oracle
+from oracle import parity
+from paper_conf_icde_giesekerhvo20_b200 import binding, synth
+
+pytestmark = pytest.mark.gpu
+DEV = "cuda:0"
+
+
+def _compare(out, Y, dates, n, k, hf, lam):
+    orc = oracle.monitor(np.ascontiguousarray(Y.cpu().numpy()), dates, n, k, hf, lam)
+    gpu = {key: v.cpu().numpy() for key, v in out.items() if torch.is_tensor(v)}
+    rep = parity.compare(gpu, orc, dates, n, k)
+    assert rep["ok"], json.dumps(rep)
+    np.testing.assert_array_equal(gpu["nbar"], orc["nbar"])
+    return rep, gpu, orc
+
+
+def _dense_history(spec, dense_cols=None):
+    """i.i.d. gaps in the monitoring period only (or, with dense_cols, a
+    complete history only for those columns): the mask-free draw of the same
+    seed supplies the history values (synth draws the mask after the values)."""
+    Y, dates = synth.generate(spec, DEV)
+    Y0, _ = synth.generate(synth.StackSpec(**{**spec.asdict(), "mask": "none"}), DEV)
+    ok = ~torch.isnan(Y)
+    assert torch.equal(Y[ok], Y0[ok])
+    cols = slice(None) if dense_cols is None else dense_cols
+    Y[: spec.n_hist, cols] = Y0[: spec.n_hist, cols]
+    return Y, dates
+
+
+@pytest.mark.parametrize("shared", ["1", "0"])
+@pytest.mark.parametrize("N,k", [(228, 3), (400, 3), (250, 5), (100, 1), (1000, 2)])
+def test_f3_nan_free_history(N, k, shared, monkeypatch):
+    monkeypatch.setenv("BFAST_SHARED_FACTOR", shared)
+    spec = synth.StackSpec(P=20_000 + 37, N=N, n_hist=N // 2, k=k, miss=0.3, mask="iid", seed=700 + N + k)
+    Y, dates = _dense_history(spec)
+    out = binding.bfast_monitor_ex(Y, dates, spec.n_hist, spec.k, spec.hf, spec.lam, diagnostics=True)
+    torch.cuda.synchronize()
+    rep, gpu, _ = _compare(out, Y, dates, spec.n_hist, spec.k, spec.hf, spec.lam)
+    assert np.all(gpu["nbar"] == spec.n_hist)
+    assert rep["breaks_oracle"] > 0
+
+
+def test_f3_mixed_warps_and_paths_agree(monkeypatch):
+    """Half the columns with a complete history, half with gaps: warps of
+    either kind (and the boundary warp) in one launch; the shared-factor and
+    per-pixel-factor runs agree to fp32 rounding and both match the oracle."""
+    spec = synth.StackSpec(P=40_000, N=400, n_hist=200, miss=0.5, mask="iid", seed=733)
+    Y, dates = _dense_history(spec, dense_cols=slice(0, 20_011))
+    res = {}
+    for shared in ("1", "0"):
+        monkeypatch.setenv("BFAST_SHARED_FACTOR", shared)
+        out = binding.bfast_monitor_ex(Y, dates, spec.n_hist, spec.k, spec.hf, spec.lam, diagnostics=True)
+        torch.cuda.synchronize()
+        _compare(out, Y, dates, spec.n_hist, spec.k, spec.hf, spec.lam)
+        res[shared] = {key: v.cpu().numpy() for key, v in out.items() if torch.is_tensor(v)}
+    a, b = res["1"], res["0"]
+    np.testing.assert_array_equal(a["nbar"], b["nbar"])
+    same = a["break"] == b["break"]
+    assert same.mean() > 0.9999
+    fin = np.isfinite(a["magnitude"])
+    assert np.max(np.abs(a["magnitude"][fin] - b["magnitude"][fin]) / np.maximum(1, np.abs(b["magnitude"][fin]))) < 1e-4
+
+
+def _stack_with_empty_slices(P, ldY, N, n, seed, frac_empty=0.4):
+    """A stack with a share of all-NaN date slices (the Africa case, L379),
+    padding columns holding values, and a slice whose only value is the last
+    pixel."""
+    spec = synth.StackSpec(P=P, N=N, n_hist=n, miss=0.4, mask="iid", seed=seed)
+    Y, dates = synth.generate(spec, DEV, ldY=ldY)
+    rng = np.random.default_rng(seed)
+    empty = np.sort(rng.choice(np.arange(1, N - 1), size=int(frac_empty * N), replace=False))
+    Y[torch.from_numpy(empty).to(DEV), :P] = float("nan")
+    if ldY > P:
+        Y[torch.from_numpy(empty).to(DEV), P:] = 3.0  # values outside the P pixels do not count
+    Y[N - 1, :P] = float("nan")
+    Y[N - 1, P - 1] = 0.5
+    return spec, Y, dates
+
+
+@pytest.mark.parametrize("P,ldY", [(50_000, 50_000), (40_001, 40_007), (3, 8), (300_000, 300_004)])
+def test_f2_valid_dates_and_gather_bit_exact(P, ldY):
+    spec, Y, dates = _stack_with_empty_slices(P, ldY, 160, 80, seed=900 + P % 97)
+    keep = binding.bfast_valid_dates(Y, P=P).cpu().numpy()
+    assert binding.last_launch_count() == 1
+    _, _, _, keep_idx = oracle.drop_empty_dates(Y.cpu().numpy(), dates, spec.n_hist, P=P)
+    assert np.flatnonzero(keep).tolist() == keep_idx.tolist()
+    idx = torch.from_numpy(keep_idx.astype(np.int32)).to(DEV)
+    Yc = binding.bfast_gather_dates(Y, idx, P=P)
+    torch.cuda.synchronize()
+    ref = Y[idx.long(), :P]
+    assert torch.equal(Yc.view(torch.int32), ref.contiguous().view(torch.int32))
+
+
+def test_f2_monitoring_on_the_compacted_stack():
+    """drop_empty_dates + the hot path = the oracle run on the oracle's own
+    compacted stack; break offsets map back to a valid original date."""
+    spec, Y, dates = _stack_with_empty_slices(30_000, 30_000, 400, 200, seed=931, frac_empty=0.5)
+    Yc, dc, nc, keep_idx = binding.drop_empty_dates(Y, dates, spec.n_hist)
+    Yo, do, nco, ko = oracle.drop_empty_dates(Y.cpu().numpy(), dates, spec.n_hist)
+    assert nc == nco and np.array_equal(keep_idx, ko) and np.array_equal(dc, do)
+    out = binding.bfast_monitor_ex(Yc, dc, nc, spec.k, spec.hf, spec.lam, diagnostics=True)
+    torch.cuda.synchronize()
+    assert np.array_equal(Yc.cpu().numpy().view(np.uint32), Yo.view(np.uint32))
+    rep, gpu, orc = _compare(out, Yc, dc, nc, spec.k, spec.hf, spec.lam)
+    ob = binding.original_break_offsets(gpu["break"], keep_idx, nc, spec.n_hist)
+    hit = np.flatnonzero(ob >= 0)
+    assert len(hit) > 100
+    Yh = Y.cpu().numpy()
+    assert np.all(~np.isnan(Yh[spec.n_hist + ob[hit], hit]))  # the break date holds the pixel's value
+    assert np.all(ob[gpu["break"] < 0] == gpu["break"][gpu["break"] < 0])
+
+
+def test_f2_tile_level_resume_is_identical():
+    """A scene streamed from host memory in tiles, interrupted after two
+    tiles and resumed, gives the bytes of one uninterrupted call."""
+    spec = synth.StackSpec(P=300_000, N=228, n_hist=114, miss=0.5, mask="iid", seed=955)
+    Y, dates = synth.generate(spec, DEV)
+    Yh = Y.cpu().pin_memory()
+    b1, m1 = binding.bfast_monitor_host(Yh, dates, spec.n_hist, spec.k, spec.hf, spec.lam)
+    b2 = np.full(spec.P, 7, np.int32)
+    m2 = np.full(spec.P, 7.0, np.float32)
+    done = binding.bfast_monitor_host_resume(Yh, dates, spec.n_hist, spec.k, spec.hf, spec.lam, b2, m2,
+                                             done=0, tile=70_000, max_tiles=2)
+    assert done == 140_000 and np.all(b2[done:] == 7)
+    done = binding.bfast_monitor_host_resume(Yh, dates, spec.n_hist, spec.k, spec.hf, spec.lam, b2, m2,
+                                             done=done, tile=70_000)
+    assert done == spec.P
+    np.testing.assert_array_equal(b1, b2)
+    np.testing.assert_array_equal(m1.view(np.uint32), m2.view(np.uint32))

@@ -401,3 +401,40 @@ def test_design_row_order_sin_before_cos():
     x = oracle.design_row(d, 1, 2)
     np.testing.assert_allclose(x, [1, 2, math.sin(TWO_PI * 0.35), math.cos(TWO_PI * 0.35),
                                    math.sin(2 * TWO_PI * 0.35), math.cos(2 * TWO_PI * 0.35)])
+
+
+def test_p10_drop_empty_dates_brute_force():
+    """f2 (L291, L379): the kept slices of the oracle's date filter against a
+    loop over every element, on a stack built to trip the plausible mistakes:
+    values only in the padding columns (>= P) of an otherwise empty slice,
+    non-canonical NaN payloads, empty slices at n-1 and n (the history count
+    n_hist' of the compacted stack), a slice whose only value is the last
+    pixel."""
+    rng = np.random.default_rng(11)
+    N, P, ldY, n = 40, 37, 44, 20
+    Y = rng.normal(size=(N, ldY)).astype(np.float32)
+    Y[rng.random((N, ldY)) < 0.5] = np.nan
+    empty = [0, 3, n - 1, n, 31, N - 1]
+    Y[empty, :P] = np.nan
+    Y[3, P:] = 1.0                      # values only in the padding
+    bits = Y.view(np.uint32)
+    bits[31, :P] = np.uint32(0xFFC00001)  # negative, non-canonical NaNs
+    Y[7, :P] = np.nan
+    Y[7, P - 1] = 2.5                   # only the last pixel
+    dates = np.arange(1, N + 1) / 23.0 + 2000.0
+    Yc, dc, nc, keep = oracle.drop_empty_dates(Y, dates, n, P=P)
+    brute = []
+    for t in range(N):
+        has = False
+        for p in range(P):
+            v = float(Y[t, p])
+            if v == v:
+                has = True
+                break
+        if has:
+            brute.append(t)
+    assert keep.tolist() == brute
+    assert set(empty).isdisjoint(brute) and 7 in brute
+    assert nc == sum(1 for t in brute if t < n) == n - 3
+    assert np.array_equal(Yc.view(np.uint32), Y[brute, :P].view(np.uint32))
+    assert np.array_equal(dc, dates[brute])
