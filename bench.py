@@ -56,7 +56,7 @@ def spec_for(name: str):
     if name.startswith("sweep:"):
         _, N, miss, k = name.split(":")
         return synth.sweep_spec(int(N), float(miss), int(k)), f"sweep N={N} miss={miss} k={k}"
-    spec = synth.CONFIGS["landsat" if name == "stream" else name]
+    spec = synth.CONFIGS["landsat" if name in ("stream", "int16") else name]
     desc = {
         "landsat": "Landsat-like scene (BASELINE configs[1]): 4096x4096 px x N=400 dates "
                    "(n_hist=200), k=3, h=0.25, lambda=1.65, 60% missing (cloud masks)",
@@ -66,6 +66,8 @@ def spec_for(name: str):
                      "k=3, h=0.25, lambda=1.65, 50% NaN i.i.d.; pixel shards over the GPUs (strong scaling)",
         "stream": "continental streaming (BASELINE configs[4]): Landsat-shaped tiles (4096x4096 px x N=400, "
                   "60% cloud) from pinned host memory through the e2e path, H2D double-buffered",
+        "int16": "SURVEY 8(f) f4: the Landsat scene (BASELINE configs[1] shape) as scaled int16 codes "
+                 "(y = 1e-4 code, nodata -32768), read by the fused kernel as codes: 2 bytes per stack element",
         "dense": "SURVEY 8(f) f3: Landsat-shaped scene (4096x4096 px x N=400, n_hist=200, k=3) with a complete "
                  "history (the NaN-free case of L93), 60% cloud gaps in the monitoring period only",
         "africa": "SURVEY 8(f) f2: 2^23 px x 2000 dates (n_hist=1000, k=3), 88% of the date slices empty "
@@ -588,10 +590,22 @@ def main():
     stream = torch.cuda.Stream(device=dev)
     out = {"break": torch.empty(P, dtype=torch.int32, device=dev),
            "magnitude": torch.empty(P, dtype=torch.float32, device=dev)}
+    I16 = (1e-4, 0.0, -32768)  # codec of the int16 config (scale, offset, nodata)
+    codes = None
+    if args.config == "int16":
+        codes = synth.quantize_i16(Y, *I16)
+        del Y
+        Y = None
+        torch.cuda.empty_cache()
+        args.no_e2e = True
     torch.cuda.synchronize()
 
     def step():
-        plan.execute(Y, stream=stream, out=out)
+        if codes is not None:
+            binding.bfast_monitor_i16(codes, dates, rspec.n_hist, rspec.k, rspec.hf, rspec.lam, *I16,
+                                      stream=stream, out=out)
+        else:
+            plan.execute(Y, stream=stream, out=out)
 
     with torch.cuda.stream(stream):
         for _ in range(args.warmup):
@@ -633,7 +647,7 @@ def main():
     value = total_pixels / (ms_step / 1000.0)
 
     # roofline of the dominant (fused) kernel: algorithmic bytes per launch
-    alg_bytes = P * (4 * N + 8)
+    alg_bytes = P * ((2 if codes is not None else 4) * N + 8)
     kms = sorted(kernel_ms)
     k_avg = sum(kms) / len(kms) if kms else float("nan")
     peak, peak_src = load_peaks()
@@ -673,7 +687,26 @@ def main():
             "roofline": roofline, "gpu_launches": launches, "clocks": clocks}
 
     # cpu baseline + sampled parity (rank 0, N = 1 only)
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and codes is not None:
+        # int16: the oracle decodes the sampled code columns itself (oracle.decode_i16)
+        import oracle
+        from oracle import parity
+        idx = synth.sample_columns(codes, P, 1 << 17, seed=11)
+        it = torch.tensor(idx, device=dev)
+        Yd = oracle.decode_i16(codes.index_select(1, it).cpu().numpy(), np.float32(I16[0]), np.float32(I16[1]),
+                               I16[2])
+        t0 = time.perf_counter()
+        orc = oracle.monitor(np.ascontiguousarray(Yd), dates, rspec.n_hist, rspec.k, rspec.hf, rspec.lam)
+        dt = time.perf_counter() - t0
+        gpu = {"break": out["break"].index_select(0, it).cpu().numpy(),
+               "magnitude": out["magnitude"].index_select(0, it).cpu().numpy()}
+        rep = parity.compare(gpu, orc)
+        line["cpu_baseline"] = cpu_baseline_entry(len(idx) / dt, oracle.max_threads(),
+                                                  f"{len(idx)} sampled columns decoded by the oracle, {dt:.1f} s")
+        line["parity_sample"] = {k: rep[k] for k in ("pixels", "ok", "break_mismatch",
+                                                     "break_mismatch_unexcused", "invalid_mismatch",
+                                                     "mag_fail", "mag_max_scaled_err")}
+    elif rank == 0 and world == 1 and not args.no_cpu_baseline:
         from oracle import parity
         probe = 1 << 13
         _, dt, threads, _ = oracle_sample(Y, dates, rspec, probe, seed=7)

@@ -205,6 +205,33 @@ int bfast_monitor_shards(const float *const *Y_dev, const int64_t *P, const int6
                          int32_t *out_break, float *out_magnitude);
 
 /*
+ * ---- Compact input codec (not from the paper) --------
+ * Landsat NDMI products are delivered as scaled int16 with a nodata code;
+ * reading the codes halves the stack bytes per date.
+ *   y = fmaf(scale, (float)code, offset)  for code != nodata (one rounding)
+ *   code == nodata -> missing (the NaN of L164)
+ * bfast_monitor_i16 runs the hot path of bfast_monitor_ex on such a stack:
+ * codec->Y is the DEVICE stack int16 [N][ldY] (a->ldY counts int16
+ * elements; a->Y must be NULL), every other argument and output as in
+ * bfast_args, in the units of y.  The result is that of bfast_monitor_ex on
+ * the decoded float32 stack up to the parity tolerances: the
+ * path runs on the codes and applies the codec to beta, sigma-hat and the
+ * MOSUM's sign; flagged pixels are refitted in fp64 on the decoded values.
+ * Requirements: a 16-byte aligned codec->Y and ldY % 8 == 0 (TMA rows), the
+ * fused tensor-core kernel (not BFAST_KERNEL=simt).  Errors: BFAST_EINVAL
+ * (NULL codec/args, a->Y != NULL, scale zero or not finite, offset not
+ * finite, nodata outside [-32768, 32767], and every bfast_args rule);
+ * BFAST_EUNSUPPORTED (alignment, SIMT-only plan).  Asynchronous on a->stream.
+ */
+typedef struct {
+  const int16_t *Y; /* device [N][ldY] codes */
+  float scale;      /* y = fmaf(scale, code, offset) */
+  float offset;
+  int32_t nodata;   /* the missing-value code, in [-32768, 32767] */
+} bfast_codec_i16;
+int bfast_monitor_i16(const bfast_codec_i16 *codec, const bfast_args *a);
+
+/*
  * ---- Preprocessing before the hot path --------------
  * after a chunk is copied to the GPU, "removal of slices only
  * containing NaN values"; L379: a Landsat image of Africa spans 6873 dates

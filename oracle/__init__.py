@@ -56,6 +56,8 @@ def _load():
         lib.oracle_gauss_jordan_inverse.restype = ctypes.c_int
         lib.oracle_fit.argtypes = [P, P, i32, i32, P, P]
         lib.oracle_fit.restype = ctypes.c_int
+        lib.oracle_decode_i16.argtypes = [P, i64, f32, f32, ctypes.c_int32, P]
+        lib.oracle_decode_i16.restype = None
         lib.oracle_boundary.argtypes = [f64, i32, i64]
         lib.oracle_boundary.restype = f64
         lib.oracle_mosum.argtypes = [P, i32, i32, i32, f64, P]
@@ -182,3 +184,12 @@ def drop_empty_dates(Y, dates, n_hist, P: int | None = None):
     d = np.asarray(dates, dtype=np.float64)
     return (np.ascontiguousarray(Y[keep_idx, :P]), d[keep_idx],
             int(np.count_nonzero(keep_idx < int(n_hist))), keep_idx)
+
+
+def decode_i16(codes, scale: float, offset: float, nodata: int):
+    """f4 (reading R15): y = fmaf(scale, code, offset) in fp32, nodata -> NaN
+    (oracle_decode_i16, C99 fmaf).  Same shape as `codes`."""
+    c = np.ascontiguousarray(np.asarray(codes, dtype=np.int16))
+    y = np.empty(c.shape, dtype=np.float32)
+    _load().oracle_decode_i16(_ptr(c), int(c.size), float(scale), float(offset), int(nodata), _ptr(y))
+    return y

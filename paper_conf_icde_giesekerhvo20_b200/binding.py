@@ -31,7 +31,7 @@ EXPORTS = ("bfast_monitor", "bfast_monitor_ex", "bfast_plan_create", "bfast_plan
            "bfast_shard_range", "bfast_last_launch_count", "bfast_last_error",
            "bfast_status_string", "bfast_abi_version", "bfast_profile_enable",
            "bfast_profile_collect", "bfast_valid_dates", "bfast_gather_dates",
-           "bfast_monitor_host_resume")
+           "bfast_monitor_host_resume", "bfast_monitor_i16")
 IPC_HANDLE_BYTES = 72
 
 
@@ -39,6 +39,11 @@ class BfastError(RuntimeError):
     def __init__(self, status: int, msg: str):
         super().__init__(f"{msg} (status {status})")
         self.status = status
+
+
+class _CodecI16(ctypes.Structure):
+    _fields_ = [("Y", ctypes.c_void_p), ("scale", ctypes.c_float), ("offset", ctypes.c_float),
+                ("nodata", ctypes.c_int32)]
 
 
 class _Args(ctypes.Structure):
@@ -90,6 +95,8 @@ def lib():
         L.bfast_abi_version.restype = I
         L.bfast_profile_enable.argtypes = [I]
         L.bfast_profile_enable.restype = I
+        L.bfast_monitor_i16.argtypes = [ctypes.POINTER(_CodecI16), ctypes.POINTER(_Args)]
+        L.bfast_monitor_i16.restype = I
         L.bfast_valid_dates.argtypes = [V, i64, i64, i64, V, V]
         L.bfast_valid_dates.restype = I
         L.bfast_gather_dates.argtypes = [V, i64, i64, V, i64, V, i64, V]
@@ -238,6 +245,30 @@ def bfast_monitor_ex(Y, dates, n_hist, k, h, lam, P=None, diagnostics=False, str
                        out_beta=out.get("beta"), out_sigma=out.get("sigma"), out_nbar=out.get("nbar"),
                        out_flags=out.get("flags"), stream=stream)
         _check(lib().bfast_monitor_ex(ctypes.byref(a)))
+    out["_dates_keepalive"] = d
+    return out
+
+
+def bfast_monitor_i16(Y16, dates, n_hist, k, h, lam, scale, offset, nodata, P=None, diagnostics=False,
+                      stream=None, out=None):
+    """f4: the hot path on an int16-coded stack (CUDA int16 [N][ldY], ldY %
+    8 == 0): y = fmaf(scale, code, offset), code == nodata missing.  Outputs
+    as bfast_monitor_ex, in the units of y."""
+    import torch
+    if not (isinstance(Y16, torch.Tensor) and Y16.is_cuda and Y16.dtype == torch.int16 and Y16.dim() == 2
+            and Y16.stride(1) == 1):
+        raise TypeError("Y16 must be a CUDA int16 [N][P] tensor with unit column stride")
+    P = int(Y16.shape[1]) if P is None else int(P)
+    out = out if out is not None else _outputs(Y16, P, k, diagnostics)
+    _check_out(out, Y16, P)
+    d = _dates(dates)
+    with torch.cuda.device(Y16.device):
+        a = _make_args(Y16, d, n_hist, k, h, lam, out["break"], out["magnitude"], P=P,
+                       out_beta=out.get("beta"), out_sigma=out.get("sigma"), out_nbar=out.get("nbar"),
+                       out_flags=out.get("flags"), stream=stream)
+        a.Y = None
+        c = _CodecI16(_dptr(Y16), float(scale), float(offset), int(nodata))
+        _check(lib().bfast_monitor_i16(ctypes.byref(c), ctypes.byref(a)))
     out["_dates_keepalive"] = d
     return out
 

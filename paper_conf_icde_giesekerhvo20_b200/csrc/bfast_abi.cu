@@ -185,16 +185,20 @@ PFN_encodeTiled get_encode() {
 
 // Tensor map of the stack range [p0, p0+P) x [0, N): box `pix` px x 16 dates
 // (one tile), out-of-bounds elements read as NaN (= missing).
-bool make_stack_map(CUtensorMap *m, const float *Y, int64_t ldY, int64_t P, int64_t N, int pix, int dates = 16) {
+bool make_stack_map(CUtensorMap *m, const void *Y, int64_t ldY, int64_t P, int64_t N, int pix, int dates = 16,
+                    bool i16 = false) {
   PFN_encodeTiled enc = get_encode();
   if (!enc) return false;
   cuuint64_t dims[2] = {(cuuint64_t)P, (cuuint64_t)N};
-  cuuint64_t strides[1] = {(cuuint64_t)ldY * sizeof(float)};
+  cuuint64_t strides[1] = {(cuuint64_t)ldY * (i16 ? 2 : 4)};
   cuuint32_t box[2] = {(cuuint32_t)pix, (cuuint32_t)dates};
   cuuint32_t es[2] = {1, 1};
-  return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void *)Y, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-             CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-             CU_TENSOR_MAP_FLOAT_OOB_FILL_NAN_REQUEST_ZERO_FMA) == CUDA_SUCCESS;
+  // float32: out-of-bounds elements read as NaN (= missing); int16 codes:
+  // zero (the kernel marks a period's dates past its end itself)
+  return enc(m, i16 ? CU_TENSOR_MAP_DATA_TYPE_UINT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void *)Y, dims, strides,
+             box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+             i16 ? CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE : CU_TENSOR_MAP_FLOAT_OOB_FILL_NAN_REQUEST_ZERO_FMA) ==
+         CUDA_SUCCESS;
 }
 
 uint16_t bf16_rne(double v) {
@@ -402,31 +406,33 @@ size_t simt_smem(const bfast_plan &pl, int bp) {
 // registers admit, and a persistent grid over the tile groups.
 // Returns BFAST_OK with `done` = false when the stack cannot be read by TMA
 // (row pitch not a multiple of 16 bytes): the caller falls back to SIMT.
-template <int K>
+template <int K, bool I16>
 int launch_fused(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t st, bool &done) {
   using C = bfast::FzCfg<K>;
   done = false;
   static thread_local int configured_dev = -1;
   cudaFuncAttributes fa{};
-  CUDA_TRY(cudaFuncGetAttributes(&fa, bfast::monitor_fused_kernel<K>));
+  CUDA_TRY(cudaFuncGetAttributes(&fa, bfast::monitor_fused_kernel<K, I16>));
   const int static_smem = (int)fa.sharedSizeBytes;
   if (configured_dev != pl.device) {
-    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_fused_kernel<K>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                  kMaxSmem - static_smem));
-    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_fused_kernel<K>, cudaFuncAttributePreferredSharedMemoryCarveout,
-                                  (int)cudaSharedmemCarveoutMaxShared));
+    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_fused_kernel<K, I16>,
+                                  cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmem - static_smem));
+    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_fused_kernel<K, I16>,
+                                  cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared));
     configured_dev = pl.device;
   }
-  if (!pl.dtabf || (prm.ldY % 4) != 0 || ((uintptr_t)(prm.Y + prm.p0) % 16) != 0) return BFAST_OK;
+  constexpr int esz = I16 ? 2 : 4;
+  const void *Ybase = I16 ? (const void *)(prm.Y16 + prm.p0) : (const void *)(prm.Y + prm.p0);
+  if (!pl.dtabf || (prm.ldY * esz) % 16 != 0 || ((uintptr_t)Ybase % 16) != 0) return BFAST_OK;
   // tiles per CTA and stack stages: the most tiles that fit with 3 stack
   // stages, else with 2
   int T = C::TMAX, sc = C::SCMAX;
   if (const char *e = std::getenv("BFAST_FZ_T")) T = std::max(1, std::min(C::TMAX, std::atoi(e)));
   if (const char *e = std::getenv("BFAST_FZ_SC")) sc = std::max(2, std::min(C::SCMAX, std::atoi(e)));
-  auto fits = [&](int t, int c) { return C::smem_bytes(t, pl.hcap, c) + static_smem <= (size_t)kMaxSmem; };
+  auto fits = [&](int t, int c) { return C::smem_bytes(t, pl.hcap, c, esz) + static_smem <= (size_t)kMaxSmem; };
   while (T > 1 && !fits(T, 2)) --T;
   if (!fits(T, sc)) sc = 2;
-  const size_t smem = C::smem_bytes(T, pl.hcap, sc);
+  const size_t smem = C::smem_bytes(T, pl.hcap, sc, esz);
   if (smem + static_smem > (size_t)kMaxSmem)
     return fail(BFAST_EUNSUPPORTED, "fused kernel: shared memory %zu B for window %d", smem, pl.hcap);
   int sms = 148;
@@ -441,9 +447,9 @@ int launch_fused(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStre
   const int per_sm = std::max(1, std::min(std::min(by_smem, by_tmem), std::min(by_regs, by_thr)));
   // full stack; history only (dates >= n out of bounds -> NaN); L2 prefetch boxes
   CUtensorMap ymap, hmap, pmap;
-  if (!make_stack_map(&ymap, prm.Y + prm.p0, prm.ldY, prm.P, pl.N, 128, 16) ||
-      !make_stack_map(&hmap, prm.Y + prm.p0, prm.ldY, prm.P, pl.n, 128, 16) ||
-      !make_stack_map(&pmap, prm.Y + prm.p0, prm.ldY, prm.P, pl.N, 128, C::PFB))
+  if (!make_stack_map(&ymap, Ybase, prm.ldY, prm.P, pl.N, 128, 16, I16) ||
+      !make_stack_map(&hmap, Ybase, prm.ldY, prm.P, pl.n, 128, 16, I16) ||
+      !make_stack_map(&pmap, Ybase, prm.ldY, prm.P, pl.N, 128, C::PFB, I16))
     return BFAST_OK;
   int pfd = 128;
   if (const char *e = std::getenv("BFAST_FZ_PFD")) pfd = std::max(0, std::atoi(e)) / C::PFB * C::PFB;
@@ -451,6 +457,11 @@ int launch_fused(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStre
   tb.tabA = pl.dtabf;
   tb.tabB = pl.dtabf + pl.tabfB_off;
   tb.tabC = pl.dtabf + pl.tabfC_off;
+  // the float an int16 nodata code turns into (monitor_fused.cuh fz_code)
+  {
+    const uint32_t u = (((uint32_t)(uint16_t)prm.nodata) ^ 0x8000u) | 0x4B000000u;
+    std::memcpy(&tb.fnd, &u, 4);
+  }
   // BFAST_SHARED_FACTOR=0: every pixel factors its own Gram (A/B of f3)
   const char *sfe = std::getenv("BFAST_SHARED_FACTOR");
   tb.shared = (sfe && sfe[0] == '0') ? nullptr : pl.dshared;
@@ -465,7 +476,7 @@ int launch_fused(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStre
   if (std::getenv("BFAST_VERBOSE"))
     std::fprintf(stderr, "bfast: fused k=%d T=%d sc=%d smem=%zu+%d regs=%d per_sm=%d grid=%lld tile groups=%lld\n",
                  pl.k, T, sc, smem, static_smem, fa.numRegs, per_sm, (long long)grid, (long long)tb.ntg);
-  bfast::monitor_fused_kernel<K><<<(unsigned)grid, threads, smem, st>>>(prm, tb, ymap, hmap, pmap);
+  bfast::monitor_fused_kernel<K, I16><<<(unsigned)grid, threads, smem, st>>>(prm, tb, ymap, hmap, pmap);
   CUDA_TRY(cudaGetLastError());
   done = true;
   return BFAST_OK;
@@ -498,8 +509,15 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
   int launches = 0;
   bool fused = false;
   if (pl.mode == 0) {
-    const int rc = launch_fused<K>(pl, prm, st, fused);
+    const int rc = prm.Y16 ? launch_fused<K, true>(pl, prm, st, fused) : launch_fused<K, false>(pl, prm, st, fused);
     if (rc) return rc;
+  }
+  if (!fused && prm.Y16 && prm.P > 0) {
+    if (e0) cudaEventDestroy(e0);
+    if (e1) cudaEventDestroy(e1);
+    return fail(BFAST_EUNSUPPORTED, "int16 stacks run on the fused kernel only (ldY %% 8 == 0, 16-byte aligned Y)");
+  }
+  {
     launches += fused ? 1 : 0;
   }
   // SIMT kernel: forced (BFAST_KERNEL=simt), or a stack the TMA cannot read
@@ -598,16 +616,17 @@ int ensure_list(bfast_plan &pl, int64_t P) {
 // and the kernels' tile arithmetic are 32-bit.
 constexpr int64_t kMaxLaunchPixels = (int64_t)1 << 30;
 
-int execute_one(bfast_plan &pl, const bfast_args *a, int64_t p0, int64_t P);
+int execute_one(bfast_plan &pl, const bfast_args *a, int64_t p0, int64_t P, const bfast_codec_i16 *codec);
 
-int execute_range(bfast_plan &pl, const bfast_args *a, int64_t p0, int64_t P) {
+int execute_range(bfast_plan &pl, const bfast_args *a, int64_t p0, int64_t P,
+                  const bfast_codec_i16 *codec = nullptr) {
   if (P == 0) {
     g_launches = 0;
     return BFAST_OK;
   }
   int total = 0;
   for (int64_t b = 0; b < P; b += kMaxLaunchPixels) {
-    const int rc = execute_one(pl, a, p0 + b, std::min(kMaxLaunchPixels, P - b));
+    const int rc = execute_one(pl, a, p0 + b, std::min(kMaxLaunchPixels, P - b), codec);
     if (rc) return rc;
     total += g_launches;
   }
@@ -615,11 +634,17 @@ int execute_range(bfast_plan &pl, const bfast_args *a, int64_t p0, int64_t P) {
   return BFAST_OK;
 }
 
-int execute_one(bfast_plan &pl, const bfast_args *a, int64_t p0, int64_t P) {
+int execute_one(bfast_plan &pl, const bfast_args *a, int64_t p0, int64_t P, const bfast_codec_i16 *codec) {
   int rc = ensure_list(pl, P);
   if (rc) return rc;
   bfast::MonitorParams prm{};
-  prm.Y = a->Y;
+  prm.Y = codec ? nullptr : a->Y;
+  if (codec) {
+    prm.Y16 = codec->Y;
+    prm.dscale = codec->scale;
+    prm.doffset = codec->offset;
+    prm.nodata = codec->nodata;
+  }
   prm.ldY = a->ldY;
   prm.P = P;
   prm.p0 = p0;
@@ -813,6 +838,28 @@ int bfast_monitor_ex(const bfast_args *a) {
   if (rc) return rc;
   std::lock_guard<std::mutex> g(pl->mu);
   return execute_range(*pl, a, 0, a->P);
+}
+
+int bfast_monitor_i16(const bfast_codec_i16 *codec, const bfast_args *a) {
+  if (!codec || !a) return fail(BFAST_EINVAL, "codec or args NULL");
+  if (a->Y) return fail(BFAST_EINVAL, "args->Y must be NULL (the stack is codec->Y)");
+  if (!(codec->scale != 0.f) || !std::isfinite(codec->scale) || !std::isfinite(codec->offset))
+    return fail(BFAST_EINVAL, "codec scale must be finite and non-zero, offset finite");
+  if (codec->nodata < -32768 || codec->nodata > 32767) return fail(BFAST_EINVAL, "nodata outside int16");
+  bfast_args v = *a;
+  v.Y = reinterpret_cast<const float *>(codec->Y);  // validated as the stack pointer
+  int rc = validate_args(&v);
+  if (rc) return rc;
+  if (a->P > 0 && (((uintptr_t)codec->Y) % 16 != 0 || a->ldY % 8 != 0))
+    return fail(BFAST_EUNSUPPORTED, "int16 stack: Y must be 16-byte aligned and ldY %% 8 == 0 (TMA)");
+  int dev = 0;
+  CUDA_TRY(cudaGetDevice(&dev));
+  std::shared_ptr<bfast_plan> pl;
+  rc = cached_plan(dev, a->N, a->dates, a->n_hist, a->k, a->h, a->lambda, pl);
+  if (rc) return rc;
+  if (pl->mode != 0) return fail(BFAST_EUNSUPPORTED, "int16 stacks run on the fused kernel only");
+  std::lock_guard<std::mutex> g(pl->mu);
+  return execute_range(*pl, &v, 0, a->P, codec);
 }
 
 int bfast_monitor(const float *Y, int64_t N, int64_t P, const double *dates, int32_t n_hist,

@@ -122,9 +122,9 @@ struct FzCfg {
 #endif
   static constexpr int PFB = 64;                 // dates per L2-prefetch box
   static constexpr int SCMAX = 3;                // stack chunk stages per tile (2 or 3, by shared memory)
-  static constexpr int CBYTES = DC * 128 * 4;    // one [16 dates x 128 px] box (8 KB)
-  static constexpr size_t smem_bytes(int T, int hcap, int sc) {
-    return (size_t)T * sc * CBYTES + (size_t)ST * TSTAGE + (size_t)T * hcap * 512;
+  static constexpr int CBYTES = DC * 128 * 4;    // one [16 dates x 128 px] box (8 KB; 4 KB of int16 codes)
+  static constexpr size_t smem_bytes(int T, int hcap, int sc, int esz = 4) {
+    return (size_t)T * sc * (CBYTES / 4 * esz) + (size_t)ST * TSTAGE + (size_t)T * hcap * 512;
   }
 };
 
@@ -139,7 +139,27 @@ struct FzTables {
   // NaN-free history (f3): the common Cholesky factor, [Tri<K>::kN | dinv K |
   // min pivot ratio | max VIF] (bfast_abi.cu shared_factor); nullptr = off
   const float *shared;
+  // int16 codec (f4): the float every code equal to the nodata code turns
+  // into (fz_code: 2^23 + (code ^ 0x8000), exact), i.e. "missing"
+  float fnd;
 };
+
+// int16 codes (f4) enter the per-date arithmetic as the exact floats
+// 2^23 + (code + 32768): one LOP3 from the zero-extended 16-bit load.  The
+// path is invariant to an offset and, up to the sign of the MOSUM, to a
+// scale (y = scale code + offset: residuals and sigma-hat scale by scale,
+// W / (sigma-hat sqrt(nbar)) by sign(scale)); the epilogue applies the
+// codec to beta, sigma-hat and the magnitude.
+constexpr float kCodeBias = 8421376.0f;  // 2^23 + 32768: fz_code(code) - kCodeBias == code
+__device__ __forceinline__ float fz_code(uint32_t u16) { return __uint_as_float((u16 ^ 0x8000u) | 0x4B000000u); }
+__device__ __forceinline__ uint32_t lds_u16(uint32_t a) {
+  uint32_t v;
+  asm volatile("ld.shared.u16 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ void sts_u16(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u16 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
 
 #ifndef BFAST_FZ_CTLWAIT
 #define BFAST_FZ_CTLWAIT 1  // control-warp waits: 1 = hardware-suspended try_wait, 0 = spin
@@ -216,18 +236,40 @@ __device__ __forceinline__ uint32_t hi16x2(float lo_elem, float hi_elem) {
 
 // ---- per-date steps (inline PTX keeps the validity predicate in a register)
 // Pass A: vm = all-ones iff y is a value (set.num), yp = (y - c) & vm.
-__device__ __forceinline__ void fa_date(float y, float c0, uint32_t &vm, float &yp) {
+template <bool I16>
+__device__ __forceinline__ void fa_date(float y, float c0, uint32_t &vm, float &yp, float fnd) {
+  if constexpr (I16) {
+  asm("{\n\t.reg .f32 t;\n\t"
+      "set.ne.u32.f32 %0, %2, %4;\n\t"
+      "sub.f32 t, %2, %3;\n\t"
+      "and.b32 %1, t, %0;\n\t}"
+      : "=r"(vm), "=f"(yp)
+      : "f"(y), "f"(c0), "f"(fnd));
+  } else {
   asm("{\n\t.reg .f32 t;\n\t"
       "set.num.u32.f32 %0, %2, %2;\n\t"
       "sub.f32 t, %2, %3;\n\t"
       "and.b32 %1, t, %0;\n\t}"
       : "=r"(vm), "=f"(yp)
       : "f"(y), "f"(c0));
+  }
 }
 // Pass B: r = y - yhat0 (NaN iff missing); if valid: s2 += r^2 and bit BIT
 // of vb is set; rz = r or 0.
-template <int BIT>
-__device__ __forceinline__ void fb_date(float y, float c0, float yh, float &s2, uint32_t &vb, float &rz) {
+template <bool I16, int BIT>
+__device__ __forceinline__ void fb_date(float y, float c0, float yh, float &s2, uint32_t &vb, float &rz,
+                                        float fnd) {
+  if constexpr (I16) {
+  asm("{\n\t.reg .pred p;\n\t.reg .f32 r;\n\t"
+      "sub.f32 r, %3, %4;\n\t"
+      "sub.f32 r, r, %5;\n\t"
+      "setp.ne.f32 p, %3, %7;\n\t"
+      "@p fma.rn.f32 %0, r, r, %0;\n\t"
+      "@p or.b32 %1, %1, %6;\n\t"
+      "selp.f32 %2, r, 0f00000000, p;\n\t}"
+      : "+f"(s2), "+r"(vb), "=f"(rz)
+      : "f"(y), "f"(c0), "f"(yh), "n"(1u << BIT), "f"(fnd));
+  } else {
   asm("{\n\t.reg .pred p;\n\t.reg .f32 r;\n\t"
       "sub.f32 r, %3, %4;\n\t"
       "sub.f32 r, r, %5;\n\t"
@@ -237,13 +279,32 @@ __device__ __forceinline__ void fb_date(float y, float c0, float yh, float &s2, 
       "selp.f32 %2, r, 0f00000000, p;\n\t}"
       : "+f"(s2), "+r"(vb), "=f"(rz)
       : "f"(y), "f"(c0), "f"(yh), "n"(1u << BIT));
+  }
 }
 // the same with the ring write of mon ranks: slot a = wa + k*512 (wrapped
 // once by hbytes when k >= jw); the residual enters it and k advances when
 // the date is valid
-template <int BIT>
+template <bool I16, int BIT>
 __device__ __forceinline__ void fb_date_ring(float y, float c0, float yh, float &s2, uint32_t &vb, float &rz,
-                                             uint32_t &k, uint32_t wa, uint32_t jw, uint32_t hbytes) {
+                                             uint32_t &k, uint32_t wa, uint32_t jw, uint32_t hbytes, float fnd) {
+  if constexpr (I16) {
+  asm volatile(
+      "{\n\t.reg .pred p, q;\n\t.reg .f32 r;\n\t.reg .u32 a;\n\t"
+      "sub.f32 r, %4, %5;\n\t"
+      "sub.f32 r, r, %6;\n\t"
+      "setp.ne.f32 p, %4, %11;\n\t"
+      "@p fma.rn.f32 %0, r, r, %0;\n\t"
+      "@p or.b32 %1, %1, %10;\n\t"
+      "selp.f32 %2, r, 0f00000000, p;\n\t"
+      "mad.lo.u32 a, %3, 512, %7;\n\t"
+      "setp.ge.u32 q, %3, %8;\n\t"
+      "@q sub.u32 a, a, %9;\n\t"
+      "@p st.shared.f32 [a], r;\n\t"
+      "@p add.u32 %3, %3, 1;\n\t}"
+      : "+f"(s2), "+r"(vb), "=f"(rz), "+r"(k)
+      : "f"(y), "f"(c0), "f"(yh), "r"(wa), "r"(jw), "r"(hbytes), "n"(1u << BIT), "f"(fnd)
+      : "memory");
+  } else {
   asm volatile(
       "{\n\t.reg .pred p, q;\n\t.reg .f32 r;\n\t.reg .u32 a;\n\t"
       "sub.f32 r, %4, %5;\n\t"
@@ -260,12 +321,30 @@ __device__ __forceinline__ void fb_date_ring(float y, float c0, float yh, float 
       : "+f"(s2), "+r"(vb), "=f"(rz), "+r"(k)
       : "f"(y), "f"(c0), "f"(yh), "r"(wa), "r"(jw), "r"(hbytes), "n"(1u << BIT)
       : "memory");
+  }
 }
 // the same, ring slot advanced date by date (a pixel whose window h < 8 may
 // wrap more than once per 8-date half)
-template <int BIT>
+template <bool I16, int BIT>
 __device__ __forceinline__ void fb_date_ring1(float y, float c0, float yh, float &s2, uint32_t &vb, float &rz,
-                                              uint32_t &wa, uint32_t rend, uint32_t hbytes) {
+                                              uint32_t &wa, uint32_t rend, uint32_t hbytes, float fnd) {
+  if constexpr (I16) {
+  asm volatile(
+      "{\n\t.reg .pred p, q;\n\t.reg .f32 r;\n\t"
+      "sub.f32 r, %4, %5;\n\t"
+      "sub.f32 r, r, %6;\n\t"
+      "setp.ne.f32 p, %4, %10;\n\t"
+      "@p fma.rn.f32 %0, r, r, %0;\n\t"
+      "@p or.b32 %1, %1, %9;\n\t"
+      "selp.f32 %2, r, 0f00000000, p;\n\t"
+      "@p st.shared.f32 [%3], r;\n\t"
+      "@p add.u32 %3, %3, 512;\n\t"
+      "setp.ge.u32 q, %3, %7;\n\t"
+      "@q sub.u32 %3, %3, %8;\n\t}"
+      : "+f"(s2), "+r"(vb), "=f"(rz), "+r"(wa)
+      : "f"(y), "f"(c0), "f"(yh), "r"(rend), "r"(hbytes), "n"(1u << BIT), "f"(fnd)
+      : "memory");
+  } else {
   asm volatile(
       "{\n\t.reg .pred p, q;\n\t.reg .f32 r;\n\t"
       "sub.f32 r, %4, %5;\n\t"
@@ -281,13 +360,37 @@ __device__ __forceinline__ void fb_date_ring1(float y, float c0, float yh, float
       : "+f"(s2), "+r"(vb), "=f"(rz), "+r"(wa)
       : "f"(y), "f"(c0), "f"(yh), "r"(rend), "r"(hbytes), "n"(1u << BIT)
       : "memory");
+  }
 }
 // Monitoring date (Eq. (4) recurrence, L520-L525), k-indexed ring slot (h >=
 // 8): the slot holds rank cr - h; if r = y - yhat is a value it replaces
 // it, W += r - old, msum += W, mx = max(mx, |W|); wv = W after a valid date,
 // 0 after a missing one (the crossing scan of a half reads these).
+template <bool I16>
 __device__ __forceinline__ void fc_date_k(float y, float c0, float yh, float &W, float &msum, float &mx, uint32_t &k,
-                                          uint32_t wa, uint32_t jw, uint32_t hbytes, float &wv) {
+                                          uint32_t wa, uint32_t jw, uint32_t hbytes, float &wv, float fnd) {
+  if constexpr (I16) {
+  asm volatile(
+      "{\n\t.reg .pred p, q;\n\t.reg .f32 r, o, t;\n\t.reg .u32 a;\n\t"
+      "sub.f32 r, %5, %6;\n\t"
+      "sub.f32 r, r, %7;\n\t"
+      "setp.ne.f32 p, %5, %11;\n\t"
+      "mad.lo.u32 a, %3, 512, %8;\n\t"
+      "setp.ge.u32 q, %3, %9;\n\t"
+      "@q sub.u32 a, a, %10;\n\t"
+      "ld.shared.f32 o, [a];\n\t"
+      "@p st.shared.f32 [a], r;\n\t"
+      "@p add.u32 %3, %3, 1;\n\t"
+      "sub.f32 t, r, o;\n\t"
+      "@p add.f32 %0, %0, t;\n\t"
+      "@p add.f32 %1, %1, %0;\n\t"
+      "abs.f32 t, %0;\n\t"
+      "@p max.f32 %2, %2, t;\n\t"
+      "selp.f32 %4, %0, 0f00000000, p;\n\t}"
+      : "+f"(W), "+f"(msum), "+f"(mx), "+r"(k), "=f"(wv)
+      : "f"(y), "f"(c0), "f"(yh), "r"(wa), "r"(jw), "r"(hbytes), "f"(fnd)
+      : "memory");
+  } else {
   asm volatile(
       "{\n\t.reg .pred p, q;\n\t.reg .f32 r, o, t;\n\t.reg .u32 a;\n\t"
       "sub.f32 r, %5, %6;\n\t"
@@ -308,11 +411,35 @@ __device__ __forceinline__ void fc_date_k(float y, float c0, float yh, float &W,
       : "+f"(W), "+f"(msum), "+f"(mx), "+r"(k), "=f"(wv)
       : "f"(y), "f"(c0), "f"(yh), "r"(wa), "r"(jw), "r"(hbytes)
       : "memory");
+  }
 }
 // the same with the slot pointer advanced date by date (any h); returns r
 // and validity for the slow boundary path
+template <bool I16>
 __device__ __forceinline__ void fc_date_1(float y, float c0, float yh, float &W, float &msum, float &mx, int &cr,
-                                          uint32_t &wa, uint32_t rend, uint32_t hbytes, float &wv) {
+                                          uint32_t &wa, uint32_t rend, uint32_t hbytes, float &wv, float fnd) {
+  if constexpr (I16) {
+  asm volatile(
+      "{\n\t.reg .pred p, q;\n\t.reg .f32 r, o, t;\n\t"
+      "sub.f32 r, %6, %7;\n\t"
+      "sub.f32 r, r, %8;\n\t"
+      "setp.ne.f32 p, %6, %11;\n\t"
+      "ld.shared.f32 o, [%4];\n\t"
+      "@p st.shared.f32 [%4], r;\n\t"
+      "@p add.u32 %4, %4, 512;\n\t"
+      "setp.ge.u32 q, %4, %9;\n\t"
+      "@q sub.u32 %4, %4, %10;\n\t"
+      "@p add.s32 %3, %3, 1;\n\t"
+      "sub.f32 t, r, o;\n\t"
+      "@p add.f32 %0, %0, t;\n\t"
+      "@p add.f32 %1, %1, %0;\n\t"
+      "abs.f32 t, %0;\n\t"
+      "@p max.f32 %2, %2, t;\n\t"
+      "selp.f32 %5, %0, 0f7fc00000, p;\n\t}"
+      : "+f"(W), "+f"(msum), "+f"(mx), "+r"(cr), "+r"(wa), "=f"(wv)
+      : "f"(y), "f"(c0), "f"(yh), "r"(rend), "r"(hbytes), "f"(fnd)
+      : "memory");
+  } else {
   asm volatile(
       "{\n\t.reg .pred p, q;\n\t.reg .f32 r, o, t;\n\t"
       "sub.f32 r, %6, %7;\n\t"
@@ -333,6 +460,7 @@ __device__ __forceinline__ void fc_date_1(float y, float c0, float yh, float &W,
       : "+f"(W), "+f"(msum), "+f"(mx), "+r"(cr), "+r"(wa), "=f"(wv)
       : "f"(y), "f"(c0), "f"(yh), "r"(rend), "r"(hbytes)
       : "memory");
+  }
 }
 
 // the rare branch of the boundary test (Alg. 1 l.10-12), kept out of line:
@@ -428,11 +556,13 @@ __device__ __forceinline__ void fz_solve(const float (&L)[Tri<K>::kN], const flo
   });
 }
 
-template <int K>
+template <int K, bool I16>
 __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
     monitor_fused_kernel(MonitorParams p, FzTables tb, const __grid_constant__ CUtensorMap ymap,
                          const __grid_constant__ CUtensorMap hmap, const __grid_constant__ CUtensorMap pmap) {
   using C = FzCfg<K>;
+  constexpr int ESZ = I16 ? 2 : 4;           // bytes per stack element
+  constexpr int CB = C::CBYTES / 4 * ESZ;    // one [16 dates x 128 px] box
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ __align__(8) uint64_t sfull[C::TMAX][C::SCMAX];  // stack chunk stage landed (TMA tx)
   __shared__ __align__(8) uint64_t srel[C::TMAX][C::SCMAX];   // the tile's 4 warps consumed it
@@ -464,7 +594,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
   FZT_T0(t_kernel)
   const int SC = tb.sc;
   uint8_t *stack = smem;
-  uint8_t *tabs = stack + (size_t)T * SC * C::CBYTES;
+  uint8_t *tabs = stack + (size_t)T * SC * CB;
   uint8_t *ring = tabs + (size_t)C::ST * C::TSTAGE;
 
   // chunk sequence per tile group: A[0, nch), B[0, nch), C[0, ncm)
@@ -482,7 +612,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
   const uint32_t a_pub = sm100::opaque(sm100::smem_u32(&pub[tile][0]));
   const uint32_t a_sfull = sm100::opaque(sm100::smem_u32(&sfull[tile][0]));
   const uint32_t a_srel = sm100::opaque(sm100::smem_u32(&srel[tile][0]));
-  const uint32_t a_stack = sm100::opaque(sm100::smem_u32(stack + (size_t)tile * SC * C::CBYTES));
+  const uint32_t a_stack = sm100::opaque(sm100::smem_u32(stack + (size_t)tile * SC * CB));
 
   if (tid == 0) {
     for (int i = 0; i < T; ++i) {
@@ -608,8 +738,8 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
               if (ldc.y + tb.pfd < end) tma_prefetch_2d(&pmap, ldc.x, ldc.y + tb.pfd);
             }
           }
-          const uint32_t bar = a_sfull + 8 * ldst, dst = a_stack + ldst * C::CBYTES;
-          sm100::mbar_arrive_expect_tx_a(bar, C::CBYTES);
+          const uint32_t bar = a_sfull + 8 * ldst, dst = a_stack + ldst * CB;
+          sm100::mbar_arrive_expect_tx_a(bar, CB);
           if (ldc.region == 0)
             sm100::tma_load_2d_a(dst, &hmap, ldc.x, ldc.y, bar);  // read again in pass B (L2)
           else
@@ -777,7 +907,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
     FZT_T0(t0)
     mbar_wait_spin(a_sfull + 8 * ust, uph);
     FZT_ADD(3, t0)
-    return a_stack + ust * C::CBYTES + 4 * (tid & 127);
+    return a_stack + ust * CB + ESZ * (tid & 127);
   };
   auto release_chunk = [&]() {  // every value of the chunk has been consumed
     __syncwarp();
@@ -790,8 +920,29 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
   // the 8 dates of half hf of the chunk whose column address is a
   auto load8 = [&](uint32_t a, int hf, float (&yv)[8]) {
 #pragma unroll
-    for (int d = 0; d < 8; ++d) yv[d] = lds_f(a + 512 * (8 * hf + d));
+    for (int d = 0; d < 8; ++d) {
+      if constexpr (I16)
+        yv[d] = fz_code(lds_u16(a + 256 * (8 * hf + d)));
+      else
+        yv[d] = lds_f(a + 512 * (8 * hf + d));
+    }
   };
+  const float fnd = tb.fnd;
+  auto is_value = [&](float y) { return I16 ? y != fnd : y == y; };
+  // int16 stacks have no NaN out-of-bounds fill: the dates of a period's
+  // last chunk past its end (TMA zero fill) are set to the nodata code in
+  // this thread's own column before it reads them (then ordered before the
+  // stage's next TMA write)
+  const uint32_t nd16 = (uint32_t)(uint16_t)p.nodata;
+  auto patch_tail = [&](uint32_t a, int valid_rows) {
+    if constexpr (I16) {
+      if (valid_rows < C::DC) {
+        for (int d = valid_rows; d < C::DC; ++d) sts_u16(a + 256 * d, nd16);
+        sm100::fence_proxy_async_smem();
+      }
+    }
+  };
+  const int hist_tail = n - (nch - 1) * C::DC, mon_tail = p.N - n - (ncm - 1) * C::DC;
   uint32_t g = 0;  // group sequence
   auto wait_group = [&](uint32_t gg) {  // group gg's MMAs have completed
     mbar_wait_spin(a_mdone + 8 * (gg & 3), (gg >> 2) & 1);
@@ -826,6 +977,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
     for (int c = 0; c < nch; ++c) {
       uint32_t w[24];
       const uint32_t ya = acquire_chunk();
+      if (c == nch - 1) patch_tail(ya, hist_tail);
 #pragma unroll
       for (int hf = 0; hf < 2; ++hf) {
         float yv[8];
@@ -833,7 +985,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
         if (__any_sync(0xffffffffu, !have)) {  // offset c = first valid value
 #pragma unroll
           for (int d = 0; d < 8; ++d)
-            if (!have && yv[d] == yv[d]) {
+            if (!have && is_value(yv[d])) {
               c0 = yv[d];
               have = true;
             }
@@ -842,8 +994,10 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
         float yp[8];
 #pragma unroll
         for (int d = 0; d < 8; ++d) {
-          ymax = fmaxf(ymax, fabsf(yv[d]));  // NaN ignored
-          fa_date(yv[d], c0, vm[d], yp[d]);
+          fa_date<I16>(yv[d], c0, vm[d], yp[d], fnd);
+          // the signal scale of the sigma-hat refit trigger: max |y| (NaN
+          // ignored); codes: max |y - c| (their floats carry the 2^23 bias)
+          ymax = fmaxf(ymax, fabsf(I16 ? yp[d] : yv[d]));
         }
         if (hf == 1) release_chunk();
         // y' = hi (truncated to bf16, exact) + lo (exact in fp32, rounded
@@ -1012,6 +1166,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
       uint32_t w[24];
       sm100::tmem_ld_wait();
       const uint32_t ya = acquire_chunk();
+      if (c == nch - 1) patch_tail(ya, hist_tail);
 #pragma unroll
       for (int hf = 0; hf < 2; ++hf) {
         float yv[8], rz[8];
@@ -1020,21 +1175,21 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
         if (!ringmode) {
           SFor<0, 8>::run([&](auto dc) {
             constexpr int d = decltype(dc)::value;
-            fb_date<d>(yv[d], c0, yh[8 * hf + d], s2, v8, rz[d]);
+            fb_date<I16, d>(yv[d], c0, yh[8 * hf + d], s2, v8, rz[d], fnd);
           });
         } else if (ring8) {
           uint32_t kk = 0;
           const uint32_t jw = (rend - wa) >> 9;
           SFor<0, 8>::run([&](auto dc) {
             constexpr int d = decltype(dc)::value;
-            fb_date_ring<d>(yv[d], c0, yh[8 * hf + d], s2, v8, rz[d], kk, wa, jw, hbytes);
+            fb_date_ring<I16, d>(yv[d], c0, yh[8 * hf + d], s2, v8, rz[d], kk, wa, jw, hbytes, fnd);
           });
           const uint32_t a = wa + kk * 512;
           wa = a >= rend ? a - hbytes : a;
         } else {
           SFor<0, 8>::run([&](auto dc) {
             constexpr int d = decltype(dc)::value;
-            fb_date_ring1<d>(yv[d], c0, yh[8 * hf + d], s2, v8, rz[d], wa, rend, hbytes);
+            fb_date_ring1<I16, d>(yv[d], c0, yh[8 * hf + d], s2, v8, rz[d], wa, rend, hbytes, fnd);
           });
         }
         if (hf == 1) release_chunk();
@@ -1158,9 +1313,19 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
     const bool fit_ok = !((nbar < K + 1) || (h < 1));
     const bool inside = pix < p.p0 + p.P;  // the last tile group may be ragged
     if (inside) {
-      if (p.out_sigma) p.out_sigma[pix] = fit_ok ? sigma : qnan;
+      if constexpr (I16) {
+        // y = scale code + offset: sigma-hat scales by |scale|; beta' (the
+        // offset form) by scale, around the decoded first value
+        if (p.out_sigma) p.out_sigma[pix] = fit_ok ? fabsf(p.dscale) * sigma : qnan;
+        float bs[K];
+#pragma unroll
+        for (int i = 0; i < K; ++i) bs[i] = p.dscale * beta[i];
+        store_beta<K, float>(p, pix, bs, fmaf(p.dscale, c0 - kCodeBias, p.doffset), fit_ok);
+      } else {
+        if (p.out_sigma) p.out_sigma[pix] = fit_ok ? sigma : qnan;
+        store_beta<K, float>(p, pix, beta, c0, fit_ok);
+      }
       if (p.out_nbar) p.out_nbar[pix] = nbar;
-      store_beta<K, float>(p, pix, beta, c0, fit_ok);
     }
     write_beta();
     publish();
@@ -1184,6 +1349,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
       const int crm = __reduce_max_sync(0xffffffffu, deg ? 0 : cr - nbar);
       const bool fast = crm + C::DC <= rank_flat_min;
       const uint32_t ya = acquire_chunk();
+      if (c == ncm - 1) patch_tail(ya, mon_tail);
       sm100::tmem_ld_wait();
       publish();  // the slot is read: yhat of chunk c + NYS may overwrite it
       if (++ys == C::NYS) ys = 0;
@@ -1200,7 +1366,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
           const uint32_t jw = (rend - wa) >> 9;
 #pragma unroll
           for (int d = 0; d < 8; ++d)
-            fc_date_k(yv[d], c0, yh[8 * hf + d], W, msum, mx, kk, wa, jw, hbytes, wv[8 * hf + d]);
+            fc_date_k<I16>(yv[d], c0, yh[8 * hf + d], W, msum, mx, kk, wa, jw, hbytes, wv[8 * hf + d], fnd);
           cr += (int)kk;
           const uint32_t a = wa + kk * 512;
           wa = a >= rend ? a - hbytes : a;
@@ -1228,7 +1394,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
           for (int d = 0; d < 8; ++d) yq[d] = hf ? yh[8 + d] : yh[d];
 #pragma unroll
           for (int d = 0; d < 8; ++d) {
-            fc_date_1(yv[d], c0, yq[d], W, msum, mx, cr, wa, rend, hbytes, wv[d]);
+            fc_date_1<I16>(yv[d], c0, yq[d], W, msum, mx, cr, wa, rend, hbytes, wv[d], fnd);
             if (wv[d] == wv[d] && brk < 0 && !tie && first < 0 && fabsf(W) > thr_lo) {
               const int code = fz_boundary_rare(W * inv_scale, cr, nbar, lam);
               tie = tie || (code >> 1);
@@ -1250,7 +1416,9 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
     if (Nbar - nbar < 1) deg = true;
     if (inside) {
       p.out_break[pix] = deg ? -2 : brk;
-      p.out_mag[pix] = deg ? qnan : msum * inv_scale / (float)(Nbar - nbar);
+      // the MOSUM is scale-free up to the codec's sign (f4)
+      const float mag = msum * inv_scale / (float)(Nbar - nbar);
+      p.out_mag[pix] = deg ? qnan : (I16 && p.dscale < 0.f ? -mag : mag);
       if (p.out_flags) p.out_flags[pix] = deg ? 1u : 0u;
     }
     const bool want = (refit || tie) && fit_ok && (Nbar - nbar >= 1) && inside;

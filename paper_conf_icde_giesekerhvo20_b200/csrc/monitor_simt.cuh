@@ -50,6 +50,11 @@ struct MonitorParams {
   uint8_t *out_flags;
   int64_t *refit_list;   // absolute pixel indices (int64: P may exceed 2^31 across launches)
   int32_t *refit_count;
+  // int16 codec (Y16 == nullptr: the float32 stack Y):
+  // y = fmaf(dscale, (float)code, doffset), code == nodata -> missing
+  const int16_t *Y16;
+  float dscale, doffset;
+  int32_t nodata;
 };
 
 // Pivot-ratio thresholds of the fp32 solve.

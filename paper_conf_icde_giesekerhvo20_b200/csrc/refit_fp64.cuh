@@ -55,6 +55,23 @@ __device__ __forceinline__ void refit_fetch_column(float *Yc, const float *Y, in
   for (int t = lane; t < N; t += 32) cp_async4(Yc + t, ycol + (int64_t)t * ldY);
 }
 
+// an int16-coded stack (f4): the column decoded exactly as the oracle does,
+// y = fmaf(scale, code, offset) (one rounding), the nodata code -> NaN; plain
+// loads (cp.async has no 2-byte form), ordered by the caller's __syncwarp
+__device__ __forceinline__ void refit_decode_column(float *Yc, const MonitorParams &p, int64_t pix, int N, int lane) {
+  const int16_t *ycol = p.Y16 + pix;
+  for (int t = lane; t < N; t += 32) {
+    const int v = ycol[(int64_t)t * p.ldY];
+    Yc[t] = v == p.nodata ? __int_as_float(0x7fc00000) : fmaf(p.dscale, (float)v, p.doffset);
+  }
+}
+__device__ __forceinline__ void refit_column(float *Yc, const MonitorParams &p, int64_t pix, int N, int lane) {
+  if (p.Y16)
+    refit_decode_column(Yc, p, pix, N, lane);
+  else
+    refit_fetch_column(Yc, p.Y, pix, N, p.ldY, lane);
+}
+
 template <int K>
 __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
   // per warp: [N + 1] compacted residual prefix sums (fp64), then
@@ -78,7 +95,7 @@ __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
 #pragma unroll
   for (int q = 0; q < kRefitBufs - 1; ++q) {  // prologue: the first kRefitBufs - 1 columns
     const int it = item + q * stride;
-    if (it < count) refit_fetch_column(Ybuf + q * N, p.Y, p.refit_list[it], N, ldY, lane);
+    if (it < count) refit_column(Ybuf + q * N, p, p.refit_list[it], N, lane);
     cp_async_commit();
   }
   for (int buf = 0; item < count; item += stride, buf = buf + 1 == kRefitBufs ? 0 : buf + 1) {
@@ -87,7 +104,7 @@ __global__ void __launch_bounds__(128) refit_fp64_kernel(MonitorParams p) {
     // the buffer this column goes to was read by the previous item (whose
     // trailing __syncwarp ordered those reads before these copies)
     const int abuf = buf == 0 ? kRefitBufs - 1 : buf - 1;
-    if (ahead < count) refit_fetch_column(Ybuf + abuf * N, p.Y, p.refit_list[ahead], N, ldY, lane);
+    if (ahead < count) refit_column(Ybuf + abuf * N, p, p.refit_list[ahead], N, lane);
     cp_async_commit();
     cp_async_wait_prev();  // this lane's copies of the current column landed
     __syncwarp();          // ... and every other lane's

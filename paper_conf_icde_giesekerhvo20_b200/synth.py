@@ -228,3 +228,20 @@ def sample_columns(Y: torch.Tensor, P: int, count: int, seed: int = 0) -> np.nda
     rng = np.random.default_rng(seed)
     count = min(count, P)
     return np.sort(rng.choice(P, size=count, replace=False)).astype(np.int64)
+
+
+def quantize_i16(Y: torch.Tensor, scale: float, offset: float, nodata: int = -32768) -> torch.Tensor:
+    """Scaled int16 codes of a float stack (the NDMI product encoding of
+    SURVEY 8(f) f4): code = round((y - offset) / scale) clipped to the int16
+    range minus the nodata code, NaN -> nodata.  Input generation only."""
+    lo, hi = -32768.0, 32767.0
+    if nodata == -32768:
+        lo = -32767.0
+    elif nodata == 32767:
+        hi = 32766.0
+    codes = torch.empty(Y.shape, dtype=torch.int16, device=Y.device)
+    for r in range(0, Y.shape[0], 16):  # row blocks: bounded fp64 temporaries
+        y = Y[r:r + 16]
+        q = torch.round((y.double() - offset) / scale).clamp(lo, hi)
+        codes[r:r + 16] = torch.where(torch.isnan(y), torch.full_like(q, float(nodata)), q).to(torch.int16)
+    return codes

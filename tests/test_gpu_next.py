@@ -147,3 +147,36 @@ def test_f2_tile_level_resume_is_identical():
     assert done == spec.P
     np.testing.assert_array_equal(b1, b2)
     np.testing.assert_array_equal(m1.view(np.uint32), m2.view(np.uint32))
+
+
+@pytest.mark.parametrize("N,n,k,mask,miss,scale,offset,nodata,P,ldY", [
+    (228, 114, 3, "iid", 0.5, 1e-4, 0.0, -32768, 30_000, 30_000),      # tails of both periods (n % 16 = 2)
+    (400, 200, 3, "cloud", 0.6, 2e-4, -1.0, 0, 50_000, 50_008),        # nodata mid-range, padding columns
+    (250, 125, 5, "iid", 0.5, -1.5e-4, 0.25, 32767, 20_000, 20_000),  # negative scale: MOSUM sign flips
+    (100, 50, 1, "iid", 0.9, 1e-4, 0.0, -32768, 20_000, 20_000),       # mostly degenerate pixels
+])
+def test_f4_int16_codec_parity(N, n, k, mask, miss, scale, offset, nodata, P, ldY):
+    """f4: the hot path on int16 codes against the oracle on the decoded
+    stack (oracle.decode_i16: fmaf(scale, code, offset), nodata -> NaN)."""
+    spec = synth.StackSpec(P=P, N=N, n_hist=n, k=k, miss=miss, mask=mask, seed=1300 + N + k)
+    Y, dates = synth.generate(spec, DEV, ldY=ldY)
+    codes = synth.quantize_i16(Y, scale, offset, nodata)
+    out = binding.bfast_monitor_i16(codes, dates, n, k, spec.hf, spec.lam, scale, offset, nodata, P=P,
+                                    diagnostics=True)
+    torch.cuda.synchronize()
+    assert binding.last_launch_count() >= 2
+    Yd = oracle.decode_i16(codes[:, :P].cpu().numpy(), np.float32(scale), np.float32(offset), nodata)
+    orc = oracle.monitor(np.ascontiguousarray(Yd), dates, n, k, spec.hf, spec.lam)
+    gpu = {key: v.cpu().numpy() for key, v in out.items() if torch.is_tensor(v)}
+    rep = parity.compare(gpu, orc, dates, n, k)
+    assert rep["ok"], json.dumps(rep)
+    np.testing.assert_array_equal(gpu["nbar"], orc["nbar"])
+
+
+def test_f4_int16_rejects_misaligned_rows():
+    spec = synth.StackSpec(P=1000, N=100, n_hist=50, miss=0.3, seed=3)
+    Y, dates = synth.generate(spec, DEV, ldY=1004)
+    codes = synth.quantize_i16(Y, 1e-4, 0.0)
+    with pytest.raises(binding.BfastError) as e:
+        binding.bfast_monitor_i16(codes, dates, 50, 3, 0.25, 1.65, 1e-4, 0.0, -32768, P=1000)
+    assert e.value.status == -2  # BFAST_EUNSUPPORTED: TMA rows need ldY % 8 == 0

@@ -438,3 +438,31 @@ def test_p10_drop_empty_dates_brute_force():
     assert nc == sum(1 for t in brute if t < n) == n - 3
     assert np.array_equal(Yc.view(np.uint32), Y[brute, :P].view(np.uint32))
     assert np.array_equal(dc, dates[brute])
+
+
+def test_p11_decode_i16_is_one_rounding_of_the_exact_value():
+    """f4 (reading R15): every int16 code decodes to the fp32 nearest the
+    exact scale*code + offset (a multiply-then-add in fp32, two roundings,
+    misses it for some codes), the nodata code to NaN; a power-of-two scale
+    is exact."""
+    from fractions import Fraction
+    codes = np.arange(-32768, 32768, dtype=np.int64).astype(np.int16)
+    scale, offset = np.float32(1e-4), np.float32(0.1)
+    y = oracle.decode_i16(codes, scale, offset, -32768)
+    assert np.isnan(y[0]) and not np.isnan(y[1:]).any()
+    fs, fo = Fraction(float(scale)), Fraction(float(offset))
+    up = np.nextafter(y, np.float32(np.inf))
+    dn = np.nextafter(y, np.float32(-np.inf))
+    bad = 0
+    for i in range(1, len(codes), 7):
+        ex = fs * int(codes[i]) + fo
+        e0 = abs(Fraction(float(y[i])) - ex)
+        if e0 > abs(Fraction(float(up[i])) - ex) or e0 > abs(Fraction(float(dn[i])) - ex):
+            bad += 1
+    assert bad == 0
+    two = (codes[1:].astype(np.float32) * scale + offset).astype(np.float32)  # two roundings
+    assert np.any(two != y[1:])
+    y2 = oracle.decode_i16(codes, np.float32(2.0 ** -14), np.float32(0.5), 7)
+    ok = codes != 7
+    assert np.array_equal(y2[ok].astype(np.float64), codes[ok].astype(np.float64) * 2.0 ** -14 + 0.5)
+    assert np.isnan(y2[~ok]).all()
