@@ -56,7 +56,7 @@ def spec_for(name: str):
     if name.startswith("sweep:"):
         _, N, miss, k = name.split(":")
         return synth.sweep_spec(int(N), float(miss), int(k)), f"sweep N={N} miss={miss} k={k}"
-    spec = synth.CONFIGS["landsat" if name in ("stream", "int16") else name]
+    spec = synth.CONFIGS["landsat" if name in ("stream", "int16", "periods") else name]
     desc = {
         "landsat": "Landsat-like scene (BASELINE configs[1]): 4096x4096 px x N=400 dates "
                    "(n_hist=200), k=3, h=0.25, lambda=1.65, 60% missing (cloud masks)",
@@ -66,6 +66,9 @@ def spec_for(name: str):
                      "k=3, h=0.25, lambda=1.65, 50% NaN i.i.d.; pixel shards over the GPUs (strong scaling)",
         "stream": "continental streaming (BASELINE configs[4]): Landsat-shaped tiles (4096x4096 px x N=400, "
                   "60% cloud) from pinned host memory through the e2e path, H2D double-buffered",
+        "periods": "SURVEY 8(f) f1: the Landsat scene (4096x4096 px x N=400, k=3, 60% cloud) with 7 yearly "
+                   "monitoring periods in ONE fused launch (L391: 2010-2011, 2011-2012, ...; history = every "
+                   "date before the period, n_i = 230 + 23 i, N_i = n_i + 23)",
         "int16": "SURVEY 8(f) f4: the Landsat scene (BASELINE configs[1] shape) as scaled int16 codes "
                  "(y = 1e-4 code, nodata -32768), read by the fused kernel as codes: 2 bytes per stack element",
         "dense": "SURVEY 8(f) f3: Landsat-shaped scene (4096x4096 px x N=400, n_hist=200, k=3) with a complete "
@@ -600,8 +603,14 @@ def main():
         args.no_e2e = True
     torch.cuda.synchronize()
 
+    PERIODS = [(230 + 23 * i, 253 + 23 * i) for i in range(7)]  # config "periods" (L391)
+
     def step():
-        if codes is not None:
+        if args.config == "periods":
+            res = binding.bfast_monitor_periods(Y, dates, PERIODS, rspec.k, rspec.hf, rspec.lam, stream=stream)
+            out["break"], out["magnitude"] = res["break"][0], res["magnitude"][0]
+            out["_periods"] = res
+        elif codes is not None:
             binding.bfast_monitor_i16(codes, dates, rspec.n_hist, rspec.k, rspec.hf, rspec.lam, *I16,
                                       stream=stream, out=out)
         else:
@@ -648,6 +657,8 @@ def main():
 
     # roofline of the dominant (fused) kernel: algorithmic bytes per launch
     alg_bytes = P * ((2 if codes is not None else 4) * N + 8)
+    if args.config == "periods":  # the stack up to the last period's end, read once; M output maps
+        alg_bytes = P * (4 * max(e for _, e in PERIODS) + 8 * len(PERIODS))
     kms = sorted(kernel_ms)
     k_avg = sum(kms) / len(kms) if kms else float("nan")
     peak, peak_src = load_peaks()
@@ -658,6 +669,32 @@ def main():
                 "kernel": f"monitor_fused_kernel<{2 + 2 * rspec.k}>", "kernel_ms_avg": k_avg,
                 "kernel_share_of_step": k_avg / ms_step if ms_step else None,
                 "alg_bytes_per_launch": alg_bytes, "peak_source": peak_src}
+
+    if args.config == "periods":
+        # the same periods as separate single-period launches (each reads its stack slice from HBM)
+        plans = [binding.Plan(local, e, dates[:e], b, rspec.k, rspec.hf, rspec.lam) for b, e in PERIODS]
+        outs = [{"break": torch.empty(P, dtype=torch.int32, device=dev),
+                 "magnitude": torch.empty(P, dtype=torch.float32, device=dev)} for _ in PERIODS]
+        with torch.cuda.stream(stream):
+            for pl, (b, e), o in zip(plans, PERIODS, outs):
+                pl.execute(Y[:e], stream=stream, out=o)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(3):
+            for pl, (b, e), o in zip(plans, PERIODS, outs):
+                pl.execute(Y[:e], stream=stream, out=o)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        roofline["periods"] = {"M": len(PERIODS), "periods": PERIODS,
+                               "period_pixels_per_s": len(PERIODS) * P / (ms_step / 1e3),
+                               "separate_launches_ms_per_step": e0.elapsed_time(e1) / 3,
+                               "one_launch_ms_per_step": ms_step,
+                               "identical_to_separate": bool(all(
+                                   torch.equal(o["break"], out["_periods"]["break"][i]) and
+                                   torch.equal(o["magnitude"].view(torch.int32),
+                                               out["_periods"]["magnitude"][i].view(torch.int32))
+                                   for i, o in enumerate(outs)))}
+        del plans, outs
 
     if args.config == "dense":
         # f3 A/B on the same scene: the shared fp64 factor vs every pixel factoring its own Gram
@@ -708,15 +745,19 @@ def main():
                                                      "mag_fail", "mag_max_scaled_err")}
     elif rank == 0 and world == 1 and not args.no_cpu_baseline:
         from oracle import parity
+        Yo, do, so = Y, dates, rspec
+        if args.config == "periods":  # the sample checks period 0 on its own date slice
+            b0, e0_ = PERIODS[0]
+            Yo, do, so = Y[:e0_], dates[:e0_], synth.StackSpec(**{**rspec.asdict(), "N": e0_, "n_hist": b0})
         probe = 1 << 13
-        _, dt, threads, _ = oracle_sample(Y, dates, rspec, probe, seed=7)
+        _, dt, threads, _ = oracle_sample(Yo, do, so, probe, seed=7)
         count = int(min(1 << 21, max(probe, probe * args.cpu_seconds / max(dt, 1e-3))))
-        orc, dt, threads, idx = oracle_sample(Y, dates, rspec, count, seed=11)
+        orc, dt, threads, idx = oracle_sample(Yo, do, so, count, seed=11)
         it = torch.tensor(idx, device=dev)
         gpu = {"break": out["break"].index_select(0, it).cpu().numpy(),
                "magnitude": out["magnitude"].index_select(0, it).cpu().numpy()}
         rep = parity.compare(gpu, orc)
-        measure_one_thread(Y, dates, rspec)
+        measure_one_thread(Yo, do, so)
         line["cpu_baseline"] = cpu_baseline_entry(count / dt, threads,
                                                   f"{count} uniformly sampled pixel columns of the same scene, "
                                                   f"{dt:.1f} s")

@@ -205,6 +205,28 @@ int bfast_monitor_shards(const float *const *Y_dev, const int64_t *P, const int6
                          int32_t *out_break, float *out_magnitude);
 
 /*
+ * ---- Several monitoring periods per stack pass ------
+ * the large-scale runs vary "the start and the end of the
+ * monitoring periods ... each lasting one year (2010-2011, 2011-2012, ...)".
+ * Period i is the BFAST-Monitor problem on the dates [0, N_end[i]) with
+ * history [0, n_hist[i]) (each period its own fit, Alg. 1).
+ * bfast_monitor_periods runs all M periods in ONE fused launch: each
+ * persistent CTA runs every period of a pixel tile group before the next
+ * group, so the stack is read from HBM about once and re-read from L2.
+ * a: the stack and scalars as in bfast_monitor_ex (a->n_hist is ignored,
+ * a->N >= every N_end[i]); the outputs are period-major: out_break int32
+ * [M][P], out_magnitude float [M][P], optional out_beta [M][P][K],
+ * out_sigma / out_nbar / out_flags [M][P].  Result of period i = that of
+ * bfast_monitor_ex on the first N_end[i] dates with n_hist[i].
+ * Requirements: 1 <= M <= 8 distinct periods, each valid as a bfast_args
+ * (n_hist[i] in [1, N_end[i] - 1], N_end[i] <= a->N); the fused kernel
+ * (16-byte aligned Y, ldY % 4 == 0).  Errors: BFAST_EINVAL (NULL arrays,
+ * a period that fails validation, equal periods); BFAST_EUNSUPPORTED (M >
+ * 8, alignment, SIMT-only plans).  Asynchronous on a->stream.
+ */
+int bfast_monitor_periods(const bfast_args *a, const int32_t *n_hist, const int32_t *N_end, int32_t M);
+
+/*
  * ---- Compact input codec (not from the paper) --------
  * Landsat NDMI products are delivered as scaled int16 with a nodata code;
  * reading the codes halves the stack bytes per date.

@@ -193,3 +193,14 @@ def decode_i16(codes, scale: float, offset: float, nodata: int):
     y = np.empty(c.shape, dtype=np.float32)
     _load().oracle_decode_i16(_ptr(c), int(c.size), float(scale), float(offset), int(nodata), _ptr(y))
     return y
+
+
+def monitor_periods(Y, dates, periods, k, hf, lam, threads: int = 0):
+    """PAPER.md L391 (monitoring periods 2010-2011,
+    2011-2012, ... over one data cube): period (n_i, N_i) is Algorithm 1 on
+    the first N_i dates with history [0, n_i).  Plain definition: one
+    oracle run per period on that slice of the stack."""
+    Y = np.asarray(Y)
+    d = np.asarray(dates, dtype=np.float64)
+    return [monitor(np.ascontiguousarray(Y[:int(N_i)]), d[:int(N_i)], int(n_i), k, hf, lam, threads=threads)
+            for n_i, N_i in periods]

@@ -31,7 +31,7 @@ EXPORTS = ("bfast_monitor", "bfast_monitor_ex", "bfast_plan_create", "bfast_plan
            "bfast_shard_range", "bfast_last_launch_count", "bfast_last_error",
            "bfast_status_string", "bfast_abi_version", "bfast_profile_enable",
            "bfast_profile_collect", "bfast_valid_dates", "bfast_gather_dates",
-           "bfast_monitor_host_resume", "bfast_monitor_i16")
+           "bfast_monitor_host_resume", "bfast_monitor_i16", "bfast_monitor_periods")
 IPC_HANDLE_BYTES = 72
 
 
@@ -95,6 +95,8 @@ def lib():
         L.bfast_abi_version.restype = I
         L.bfast_profile_enable.argtypes = [I]
         L.bfast_profile_enable.restype = I
+        L.bfast_monitor_periods.argtypes = [ctypes.POINTER(_Args), V, V, i32]
+        L.bfast_monitor_periods.restype = I
         L.bfast_monitor_i16.argtypes = [ctypes.POINTER(_CodecI16), ctypes.POINTER(_Args)]
         L.bfast_monitor_i16.restype = I
         L.bfast_valid_dates.argtypes = [V, i64, i64, i64, V, V]
@@ -270,6 +272,29 @@ def bfast_monitor_i16(Y16, dates, n_hist, k, h, lam, scale, offset, nodata, P=No
         c = _CodecI16(_dptr(Y16), float(scale), float(offset), int(nodata))
         _check(lib().bfast_monitor_i16(ctypes.byref(c), ctypes.byref(a)))
     out["_dates_keepalive"] = d
+    return out
+
+
+def bfast_monitor_periods(Y, dates, periods, k, h, lam, P=None, diagnostics=False, stream=None):
+    """f1 (L391): several monitoring periods [(n_hist_i, N_end_i), ...] in one
+    fused launch over the stack (each period's fit on dates [0, N_end_i)).
+    Returns the outputs of bfast_monitor_ex stacked period-major: break
+    [M][P], magnitude [M][P] (+ beta [M][P][K], sigma, nbar, flags)."""
+    import torch
+    _check_stack(Y)
+    P = int(Y.shape[1]) if P is None else int(P)
+    M = len(periods)
+    n_arr = np.ascontiguousarray([int(p[0]) for p in periods], dtype=np.int32)
+    N_arr = np.ascontiguousarray([int(p[1]) for p in periods], dtype=np.int32)
+    flat = _outputs(Y, M * P, k, diagnostics)
+    d = _dates(dates)
+    with torch.cuda.device(Y.device):
+        a = _make_args(Y, d, int(n_arr[0]), k, h, lam, flat["break"], flat["magnitude"], P=P,
+                       out_beta=flat.get("beta"), out_sigma=flat.get("sigma"), out_nbar=flat.get("nbar"),
+                       out_flags=flat.get("flags"), stream=stream)
+        _check(lib().bfast_monitor_periods(ctypes.byref(a), n_arr.ctypes.data, N_arr.ctypes.data, M))
+    out = {key: (v.view(M, P, -1) if key == "beta" else v.view(M, P)) for key, v in flat.items()}
+    out["_keepalive"] = (d, n_arr, N_arr)
     return out
 
 

@@ -406,21 +406,36 @@ size_t simt_smem(const bfast_plan &pl, int bp) {
 // registers admit, and a persistent grid over the tile groups.
 // Returns BFAST_OK with `done` = false when the stack cannot be read by TMA
 // (row pitch not a multiple of 16 bytes): the caller falls back to SIMT.
+// the kernel argument of single-period launches (unused there)
+const bfast::FzMulti &no_multi() {
+  static const bfast::FzMulti m{};
+  return m;
+}
+
+template <int K, bool I16, bool MULTI>
+int fused_config(int device, cudaFuncAttributes &fa) {
+  static thread_local int configured_dev = -1;
+  CUDA_TRY(cudaFuncGetAttributes(&fa, bfast::monitor_fused_kernel<K, I16, MULTI>));
+  if (configured_dev != device) {
+    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_fused_kernel<K, I16, MULTI>,
+                                  cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmem - (int)fa.sharedSizeBytes));
+    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_fused_kernel<K, I16, MULTI>,
+                                  cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared));
+    configured_dev = device;
+  }
+  return BFAST_OK;
+}
+
 template <int K, bool I16>
 int launch_fused(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t st, bool &done) {
   using C = bfast::FzCfg<K>;
   done = false;
-  static thread_local int configured_dev = -1;
   cudaFuncAttributes fa{};
-  CUDA_TRY(cudaFuncGetAttributes(&fa, bfast::monitor_fused_kernel<K, I16>));
-  const int static_smem = (int)fa.sharedSizeBytes;
-  if (configured_dev != pl.device) {
-    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_fused_kernel<K, I16>,
-                                  cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmem - static_smem));
-    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_fused_kernel<K, I16>,
-                                  cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared));
-    configured_dev = pl.device;
+  {
+    const int rc = fused_config<K, I16, false>(pl.device, fa);
+    if (rc) return rc;
   }
+  const int static_smem = (int)fa.sharedSizeBytes;
   constexpr int esz = I16 ? 2 : 4;
   const void *Ybase = I16 ? (const void *)(prm.Y16 + prm.p0) : (const void *)(prm.Y + prm.p0);
   if (!pl.dtabf || (prm.ldY * esz) % 16 != 0 || ((uintptr_t)Ybase % 16) != 0) return BFAST_OK;
@@ -476,11 +491,15 @@ int launch_fused(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStre
   if (std::getenv("BFAST_VERBOSE"))
     std::fprintf(stderr, "bfast: fused k=%d T=%d sc=%d smem=%zu+%d regs=%d per_sm=%d grid=%lld tile groups=%lld\n",
                  pl.k, T, sc, smem, static_smem, fa.numRegs, per_sm, (long long)grid, (long long)tb.ntg);
-  bfast::monitor_fused_kernel<K, I16><<<(unsigned)grid, threads, smem, st>>>(prm, tb, ymap, hmap, pmap);
+  bfast::monitor_fused_kernel<K, I16, false><<<(unsigned)grid, threads, smem, st>>>(prm, tb, ymap, hmap, pmap,
+                                                                                   no_multi());
   CUDA_TRY(cudaGetLastError());
   done = true;
   return BFAST_OK;
 }
+
+template <int K>
+int launch_refit(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t st, int sms);
 
 template <int K>
 int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t st) {
@@ -533,10 +552,25 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
     CUDA_TRY(cudaEventRecord(e1, st));
     g_prof.emplace_back(e0, e1);
   }
-  // fp64 refit of flagged pixels; exits at once when the list is empty
+  const int rc = launch_refit<K>(pl, prm, st, sms);
+  if (rc) return rc;
+  g_launches = launches + 1;
+  return BFAST_OK;
+}
+
+// fp64 refit of the pixels the fused / SIMT kernel flagged (the plan's list);
+// exits at once when the list is empty.  Releases the plan's refit scratch.
+template <int K>
+int launch_refit(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t st, int sms) {
 #ifndef BFAST_REFIT_WARPS
 #define BFAST_REFIT_WARPS 4
 #endif
+  static thread_local int configured_dev = -1;
+  if (configured_dev != pl.device) {
+    CUDA_TRY(cudaFuncSetAttribute(bfast::refit_fp64_kernel<K>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  kMaxSmem));
+    configured_dev = pl.device;
+  }
   int rwarps = BFAST_REFIT_WARPS;  // fewer warps per CTA where a long series needs the room
   const size_t rwsmem = bfast::refit_warp_doubles((int)pl.N) * sizeof(double);
   while (rwarps > 1 && (size_t)rwarps * rwsmem > (size_t)kMaxSmem) rwarps >>= 1;
@@ -550,8 +584,114 @@ int launch_k(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t
   bfast::refit_fp64_kernel<K><<<sms * std::max(rblocks, 1), rwarps * 32, rsmem, st>>>(prm);
   CUDA_TRY(cudaGetLastError());
   CUDA_TRY(cudaEventRecord(pl.scratch_free, st));
-  g_launches = launches + 1;
   return BFAST_OK;
+}
+
+// f1: several monitoring periods in ONE fused launch (monitor_fused.cuh
+// FzMulti): period i = plans[i] with its MonitorParams; then the fp64 refit
+// of each period's flagged pixels.  Every plan has the same k and pixel range.
+template <int K>
+int launch_multi_k(const std::vector<bfast_plan *> &pls, const std::vector<bfast::MonitorParams> &prms,
+                   cudaStream_t st) {
+  using C = bfast::FzCfg<K>;
+  const int M = (int)pls.size();
+  const bfast_plan &p0 = *pls[0];
+  const bfast::MonitorParams &q0 = prms[0];
+  cudaFuncAttributes fa{};
+  {
+    const int rc = fused_config<K, false, true>(p0.device, fa);
+    if (rc) return rc;
+  }
+  const int static_smem = (int)fa.sharedSizeBytes;
+  int hcap = 1;
+  for (auto *pl : pls) hcap = std::max(hcap, pl->hcap);
+  int T = C::TMAX, sc = C::SCMAX;
+  auto fits = [&](int t, int c) { return C::smem_bytes(t, hcap, c) + static_smem <= (size_t)kMaxSmem; };
+  while (T > 1 && !fits(T, 2)) --T;
+  if (!fits(T, sc)) sc = 2;
+  const size_t smem = C::smem_bytes(T, hcap, sc);
+  if (smem + static_smem > (size_t)kMaxSmem)
+    return fail(BFAST_EUNSUPPORTED, "fused kernel: shared memory %zu B for window %d", smem, hcap);
+  int sms = 148;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, p0.device);
+  const int threads = 128 * (T + 1);
+  const int by_smem = (int)(kSmemPerSM / (smem + static_smem + 1024));
+  const int by_tmem = 512 / C::pow2cols(T * C::TCOLS);
+  const int by_regs = 65536 / (threads * std::max(fa.numRegs, 1));
+  const int per_sm = std::max(1, std::min(std::min(by_smem, by_tmem), std::min(by_regs, 2048 / threads)));
+  auto mp = std::make_unique<bfast::FzMulti>();
+  std::memset(mp.get(), 0, sizeof(bfast::FzMulti));
+  mp->M = M;
+  mp->Lg = 0;
+  const char *sfe = std::getenv("BFAST_SHARED_FACTOR");
+  for (int i = 0; i < M; ++i) {
+    const bfast_plan &pl = *pls[i];
+    bfast::FzPeriod &fp = mp->per[i];
+    fp.prm = prms[i];
+    fp.tabA = pl.dtabf;
+    fp.tabB = pl.dtabf + pl.tabfB_off;
+    fp.tabC = pl.dtabf + pl.tabfC_off;
+    fp.shared = (sfe && sfe[0] == '0') ? nullptr : pl.dshared;
+    fp.nch = pl.nch;
+    fp.ncm = pl.ncm;
+    mp->Lg += 2 * pl.nch + pl.ncm;
+    if (!make_stack_map(&fp.h, prms[i].Y + prms[i].p0, prms[i].ldY, prms[i].P, pl.n, 128, 16) ||
+        !make_stack_map(&fp.y, prms[i].Y + prms[i].p0, prms[i].ldY, prms[i].P, pl.N, 128, 16))
+      return fail(BFAST_EUNSUPPORTED, "tensor maps of the stack");
+  }
+  int64_t Nmax = 0;
+  for (auto *pl : pls) Nmax = std::max<int64_t>(Nmax, pl->N);
+  CUtensorMap pmap;
+  if (!make_stack_map(&pmap, q0.Y + q0.p0, q0.ldY, q0.P, Nmax, 128, C::PFB))
+    return fail(BFAST_EUNSUPPORTED, "tensor maps of the stack");
+  for (auto *pl : pls) CUDA_TRY(cudaStreamWaitEvent(st, pl->scratch_free, 0));
+  for (int i = 0; i < M; ++i) CUDA_TRY(cudaMemsetAsync(prms[i].refit_count, 0, sizeof(int32_t), st));
+  bfast::FzTables tb{};
+  tb.tabA = mp->per[0].tabA;
+  tb.tabB = mp->per[0].tabB;
+  tb.tabC = mp->per[0].tabC;
+  tb.nch = p0.nch;
+  tb.ncm = p0.ncm;
+  tb.T = T;
+  tb.hcap = hcap;
+  tb.pfd = 128;
+  tb.sc = sc;
+  tb.ntg = (q0.P + 128 * T - 1) / (128 * T);
+  tb.shared = nullptr;
+  const int64_t grid = std::min<int64_t>(tb.ntg, (int64_t)sms * per_sm);
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  if (g_prof_on) {
+    CUDA_TRY(cudaEventCreate(&e0));
+    CUDA_TRY(cudaEventCreate(&e1));
+    CUDA_TRY(cudaEventRecord(e0, st));
+  }
+  bfast::monitor_fused_kernel<K, false, true><<<(unsigned)grid, threads, smem, st>>>(q0, tb, mp->per[0].y,
+                                                                                    mp->per[0].h, pmap, *mp);
+  CUDA_TRY(cudaGetLastError());
+  if (g_prof_on) {
+    CUDA_TRY(cudaEventRecord(e1, st));
+    g_prof.emplace_back(e0, e1);
+  }
+  for (int i = 0; i < M; ++i) {
+    const int rc = launch_refit<K>(*pls[i], prms[i], st, sms);
+    if (rc) return rc;
+  }
+  g_launches = 1 + M;
+  return BFAST_OK;
+}
+
+int launch_multi(const std::vector<bfast_plan *> &pls, const std::vector<bfast::MonitorParams> &prms,
+                 cudaStream_t st) {
+  switch (pls[0]->k) {
+    case 0: return launch_multi_k<2>(pls, prms, st);
+    case 1: return launch_multi_k<4>(pls, prms, st);
+    case 2: return launch_multi_k<6>(pls, prms, st);
+    case 3: return launch_multi_k<8>(pls, prms, st);
+    case 4: return launch_multi_k<10>(pls, prms, st);
+    case 5: return launch_multi_k<12>(pls, prms, st);
+    case 6: return launch_multi_k<14>(pls, prms, st);
+  }
+  return fail(BFAST_EUNSUPPORTED, "k=%d", pls[0]->k);
 }
 
 int launch(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStream_t st) {
@@ -838,6 +978,85 @@ int bfast_monitor_ex(const bfast_args *a) {
   if (rc) return rc;
   std::lock_guard<std::mutex> g(pl->mu);
   return execute_range(*pl, a, 0, a->P);
+}
+
+int bfast_monitor_periods(const bfast_args *a, const int32_t *n_hist, const int32_t *N_end, int32_t M) {
+  if (!a || !n_hist || !N_end) return fail(BFAST_EINVAL, "args, n_hist or N_end NULL");
+  if (M < 1) return fail(BFAST_EINVAL, "M=%d < 1", M);
+  if (M > bfast::kMaxPeriods) return fail(BFAST_EUNSUPPORTED, "M=%d > %d periods", M, bfast::kMaxPeriods);
+  bfast_args v = *a;
+  v.n_hist = n_hist[0];
+  int rc = validate_args(&v);
+  if (rc) return rc;
+  for (int i = 0; i < M; ++i) {
+    if (N_end[i] > a->N || N_end[i] < 2) return fail(BFAST_EINVAL, "N_end[%d]=%d outside [2, N]", i, N_end[i]);
+    rc = validate_scalar(N_end[i], a->dates, n_hist[i], a->k, a->h, a->lambda);
+    if (rc) return fail(rc, "period %d: %s", i, g_err.c_str());
+    for (int j = 0; j < i; ++j)
+      if (n_hist[j] == n_hist[i] && N_end[j] == N_end[i]) return fail(BFAST_EINVAL, "periods %d and %d equal", j, i);
+  }
+  if (a->P == 0) {
+    g_launches = 0;
+    return BFAST_OK;
+  }
+  int dev = 0;
+  CUDA_TRY(cudaGetDevice(&dev));
+  std::vector<std::shared_ptr<bfast_plan>> hold(M);
+  std::vector<bfast_plan *> pls(M);
+  for (int i = 0; i < M; ++i) {
+    rc = cached_plan(dev, N_end[i], a->dates, n_hist[i], a->k, a->h, a->lambda, hold[i]);
+    if (rc) return rc;
+    pls[i] = hold[i].get();
+    if (pls[i]->mode != 0 || !pls[i]->dtabf)
+      return fail(BFAST_EUNSUPPORTED, "several periods run on the fused kernel only");
+  }
+  if (a->ldY % 4 != 0 || ((uintptr_t)a->Y) % 16 != 0)
+    return fail(BFAST_EUNSUPPORTED, "several periods: Y must be 16-byte aligned and ldY %% 4 == 0 (TMA)");
+  std::vector<bfast_plan *> order(pls);
+  std::sort(order.begin(), order.end());
+  std::vector<std::unique_lock<std::mutex>> locks;
+  for (auto *pl : order) locks.emplace_back(pl->mu);
+  const int K = 2 + 2 * a->k;
+  int total = 0;
+  for (int64_t b = 0; b < a->P; b += kMaxLaunchPixels) {
+    const int64_t w = std::min(kMaxLaunchPixels, a->P - b);
+    std::vector<bfast::MonitorParams> prms(M);
+    for (int i = 0; i < M; ++i) {
+      bfast_plan &pl = *pls[i];
+      rc = ensure_list(pl, w);
+      if (rc) return rc;
+      bfast::MonitorParams &q = prms[i];
+      q = bfast::MonitorParams{};
+      q.Y = a->Y;
+      q.ldY = a->ldY;
+      q.P = w;
+      q.p0 = b;
+      q.N = (int)pl.N;
+      q.n = pl.n;
+      q.X = pl.dX;
+      q.X64 = pl.dX64;
+      q.KP = pl.KP;
+      q.hf = pl.hf;
+      q.lambda = pl.lambda;
+      q.hcap = pl.hcap;
+      q.tc = pl.tc;
+      q.ts = pl.ts;
+      // outputs [M][P]: period i's map starts at i * P (the kernel indexes by absolute pixel)
+      q.out_break = a->out_break + (size_t)i * a->P;
+      q.out_mag = a->out_magnitude + (size_t)i * a->P;
+      q.out_beta = a->out_beta ? a->out_beta + (size_t)i * a->P * K : nullptr;
+      q.out_sigma = a->out_sigma ? a->out_sigma + (size_t)i * a->P : nullptr;
+      q.out_nbar = a->out_nbar ? a->out_nbar + (size_t)i * a->P : nullptr;
+      q.out_flags = a->out_flags ? a->out_flags + (size_t)i * a->P : nullptr;
+      q.refit_list = pl.dlist;
+      q.refit_count = pl.dcount;
+    }
+    rc = launch_multi(pls, prms, (cudaStream_t)a->stream);
+    if (rc) return rc;
+    total += g_launches;
+  }
+  g_launches = total;
+  return BFAST_OK;
 }
 
 int bfast_monitor_i16(const bfast_codec_i16 *codec, const bfast_args *a) {

@@ -144,6 +144,25 @@ struct FzTables {
   float fnd;
 };
 
+// Several monitoring periods per stack pass (PAPER.md L391:
+// yearly periods 2010-2011, 2011-2012, ... over one data cube).  Period i
+// is an independent BFAST-Monitor problem on the dates [0, N_i) with
+// history [0, n_i); the CTA runs every period of a tile group before the
+// next tile group, so the re-reads of the group's columns come from L2.
+constexpr int kMaxPeriods = 8;
+struct FzPeriod {
+  MonitorParams prm;                  // n, N, X, tc/ts, outputs, refit list of the period
+  const uint8_t *tabA, *tabB, *tabC;  // its chunk tables (history centring depends on n)
+  const float *shared;                // its NaN-free factor (f3) or nullptr
+  int nch, ncm;
+  CUtensorMap h, y;                   // its history [0, n) and full [0, N) stack maps
+};
+struct FzMulti {
+  FzPeriod per[kMaxPeriods];
+  int M;   // periods
+  int Lg;  // chunks per tile group: sum of 2 nch + ncm
+};
+
 // int16 codes (f4) enter the per-date arithmetic as the exact floats
 // 2^23 + (code + 32768): one LOP3 from the zero-extended 16-bit load.  The
 // path is invariant to an offset and, up to the sign of the MOSUM, to a
@@ -556,10 +575,13 @@ __device__ __forceinline__ void fz_solve(const float (&L)[Tri<K>::kN], const flo
   });
 }
 
-template <int K, bool I16>
+template <int K, bool I16, bool MULTI>
 __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
-    monitor_fused_kernel(MonitorParams p, FzTables tb, const __grid_constant__ CUtensorMap ymap,
-                         const __grid_constant__ CUtensorMap hmap, const __grid_constant__ CUtensorMap pmap) {
+    monitor_fused_kernel(MonitorParams pk, FzTables tb, const __grid_constant__ CUtensorMap ymap,
+                         const __grid_constant__ CUtensorMap hmap, const __grid_constant__ CUtensorMap pmap,
+                         const __grid_constant__ FzMulti mp) {
+  // MULTI (f1): the per-period values come from mp; otherwise from pk / tb
+  const MonitorParams &p = MULTI ? mp.per[0].prm : pk;
   using C = FzCfg<K>;
   constexpr int ESZ = I16 ? 2 : 4;           // bytes per stack element
   constexpr int CB = C::CBYTES / 4 * ESZ;    // one [16 dates x 128 px] box
@@ -589,7 +611,12 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
   const bool control = warp < 4;
   const int ctid = tid - 128;  // consumer thread index = pixel of the tile group
   const int tile = control ? warp : (warp - 4) >> 2;
-  const int nch = tb.nch, ncm = tb.ncm, n = p.n, hcap = tb.hcap;
+  const int nch = MULTI ? mp.per[0].nch : tb.nch, ncm = MULTI ? mp.per[0].ncm : tb.ncm, n = p.n, hcap = tb.hcap;
+  const int M = MULTI ? mp.M : 1;
+  auto P_nch = [&](int per) { return MULTI ? mp.per[per].nch : nch; };
+  auto P_ncm = [&](int per) { return MULTI ? mp.per[per].ncm : ncm; };
+  auto P_n = [&](int per) { return MULTI ? mp.per[per].prm.n : n; };
+  auto P_N = [&](int per) { return MULTI ? mp.per[per].prm.N : p.N; };
   FZT_DECL
   FZT_T0(t_kernel)
   const int SC = tb.sc;
@@ -597,8 +624,8 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
   uint8_t *tabs = stack + (size_t)T * SC * CB;
   uint8_t *ring = tabs + (size_t)C::ST * C::TSTAGE;
 
-  // chunk sequence per tile group: A[0, nch), B[0, nch), C[0, ncm)
-  const int Lg = 2 * nch + ncm;
+  // chunk sequence per tile group: A[0, nch), B[0, nch), C[0, ncm) (per period)
+  const int Lg = MULTI ? mp.Lg : 2 * nch + ncm;
   const uint32_t my_groups =
       tb.ntg > blockIdx.x ? (uint32_t)((tb.ntg - 1 - blockIdx.x) / gridDim.x + 1) : 0u;
   const uint32_t S_total = my_groups * (uint32_t)Lg;  // chunks this CTA runs
@@ -677,18 +704,21 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
       };
       auto load_table = [&](const ChunkPos &cp) {  // one elected lane
         if (cp.s >= S_total) return;
-        const int q = cp.q;
+        int q = cp.q, per = 0;
+        if (MULTI)
+          while (q >= 2 * P_nch(per) + P_ncm(per)) q -= 2 * P_nch(per) + P_ncm(per), ++per;
+        const int nq = P_nch(per);
         const uint8_t *src;
         uint32_t bytes;
-        if (q < nch) {
+        if (q < nq) {
           bytes = C::TABA;
-          src = tb.tabA + (size_t)q * C::TABA;
-        } else if (q < 2 * nch) {
+          src = (MULTI ? mp.per[per].tabA : tb.tabA) + (size_t)q * C::TABA;
+        } else if (q < 2 * nq) {
           bytes = C::TABB;
-          src = tb.tabB + (size_t)(q - nch) * C::TABB;
+          src = (MULTI ? mp.per[per].tabB : tb.tabB) + (size_t)(q - nq) * C::TABB;
         } else {
           bytes = C::TABC;
-          src = tb.tabC + (size_t)(q - 2 * nch) * C::TABC;
+          src = (MULTI ? mp.per[per].tabC : tb.tabC) + (size_t)(q - 2 * nq) * C::TABC;
         }
         sm100::mbar_arrive_expect_tx_a(a_tfull + 8 * cp.st, bytes);
         sm100::bulk_g2s_a(a_tabs + cp.st * C::TSTAGE, src, bytes, a_tfull + 8 * cp.st);
@@ -701,7 +731,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
       const int xstep = (int)gridDim.x * T * 128;
       struct ChunkCursor {
         uint32_t u;
-        int left, y, region, x;
+        int left, y, region, x, per;
       };
       auto chunk_next = [&](ChunkCursor &cc) {
         ++cc.u;
@@ -709,28 +739,33 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
         if (--cc.left == 0) {
           if (cc.region == 0) {
             cc.region = 1;
-            cc.left = nch;
+            cc.left = P_nch(cc.per);
             cc.y = 0;
           } else if (cc.region == 1) {
             cc.region = 2;
-            cc.left = ncm;
-            cc.y = n;
+            cc.left = P_ncm(cc.per);
+            cc.y = P_n(cc.per);
           } else {
+            if (++cc.per == M) {
+              cc.per = 0;
+              cc.x += xstep;
+            }
             cc.region = 0;
-            cc.left = nch;
+            cc.left = P_nch(cc.per);
             cc.y = 0;
-            cc.x += xstep;
           }
         }
       };
-      ChunkCursor ldc{0u, nch, 0, 0, (int)blockIdx.x * T * 128 + 128 * tile};
+      ChunkCursor ldc{0u, nch, 0, 0, (int)blockIdx.x * T * 128 + 128 * tile, 0};
       int ldst = 0;  // stage of the next chunk to load
       auto load_chunk = [&]() {
         if (ldc.u < U_total && lane == 0) {
           // first-touch periods (A: history, C: monitoring) are prefetched
           // into L2 in [PFB dates x 128 px] boxes, pfd dates ahead of the loads
-          if (tb.pfd > 0 && ldc.region != 1) {
-            const int base = ldc.region == 0 ? 0 : n, end = ldc.region == 0 ? n : p.N;
+          // (later periods re-read the history of earlier ones: no prefetch)
+          if (tb.pfd > 0 && ldc.region != 1 && (ldc.region == 2 || ldc.per == 0)) {
+            const int pn = P_n(ldc.per);
+            const int base = ldc.region == 0 ? 0 : pn, end = ldc.region == 0 ? pn : P_N(ldc.per);
             const int off = ldc.y - base;
             if (off % C::PFB == 0) {
               if (off == 0)
@@ -740,11 +775,13 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
           }
           const uint32_t bar = a_sfull + 8 * ldst, dst = a_stack + ldst * CB;
           sm100::mbar_arrive_expect_tx_a(bar, CB);
-          if (ldc.region == 0)
-            sm100::tma_load_2d_a(dst, &hmap, ldc.x, ldc.y, bar);  // read again in pass B (L2)
+          const void *hm = MULTI ? (const void *)&mp.per[ldc.per].h : (const void *)&hmap;
+          const void *ym = MULTI ? (const void *)&mp.per[ldc.per].y : (const void *)&ymap;
+          if (ldc.region == 0 || (MULTI && ldc.per + 1 < M))
+            // read again in pass B / by the next period (L2)
+            sm100::tma_load_2d_a(dst, ldc.region == 2 ? ym : hm, ldc.x, ldc.y, bar);
           else
-            sm100::tma_load_2d_hint_a(dst, ldc.region == 1 ? (const void *)&hmap : (const void *)&ymap, ldc.x,
-                                      ldc.y, bar, pol_first);
+            sm100::tma_load_2d_hint_a(dst, ldc.region == 1 ? hm : ym, ldc.x, ldc.y, bar, pol_first);
         }
         chunk_next(ldc);
         if (++ldst == SC) ldst = 0;
@@ -794,6 +831,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
       };
       // kind: 0 = A chunk c, 1 = beta0 (yhat of B0, B1), 2 = B chunk c, 3 =
       // beta (yhat of C0, C1), 4 = C chunk c
+      int cur_nch = nch, cur_ncm = ncm;  // the period being issued
       auto on_publish = [&](int kind, int c) {
         FZT_T0(tp)
         wait_sleep(a_pub + 8 * (g & 3), (g >> 2) & 1u);
@@ -817,7 +855,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
           sm100::umma_bf16_ts_e(tc + C::cB, at + 8, sm100::smem_desc(bx + C::BX_BYTES, C::KBn * 16, 128), idB, 1u);
           sm100::umma_bf16_ts_e(tc + C::cB, at + 16, sm100::smem_desc(bx, C::KBn * 16, 128), idB, 1u);
         } else if (kind == 1 || kind == 3) {
-          const int cnt = kind == 1 ? nch : ncm;
+          const int cnt = kind == 1 ? cur_nch : cur_ncm;
           for (int a = 0; a < C::NYS && a < cnt; ++a) issue_yhat(advance_pos(cpos, a), a);
           cslot = 0;
         } else if (kind == 2) {
@@ -836,9 +874,9 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
                                     sm100::smem_desc(bx + xx * C::BX_BYTES, C::KBn * 16, 128), idB,
                                     (c > 0 || e > 0 || xx > 0) ? 1u : 0u);
           sm100::umma_commit_e(a_mdone + 8 * (g & 3));
-          if (c + C::NYS < nch) issue_yhat(advance_pos(cpos, C::NYS), cslot);
+          if (c + C::NYS < cur_nch) issue_yhat(advance_pos(cpos, C::NYS), cslot);
         } else {
-          if (c + C::NYS < ncm) issue_yhat(advance_pos(cpos, C::NYS), cslot);
+          if (c + C::NYS < cur_ncm) issue_yhat(advance_pos(cpos, C::NYS), cslot);
         }
         if (kind == 2 || kind == 4)
           if (++cslot == C::NYS) cslot = 0;
@@ -868,19 +906,23 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
         FZT_ADD(4, ti)
       };
       for (uint32_t gi = 0; gi < my_groups; ++gi) {
-        for (int c = 0; c < nch; ++c) {
-          on_release();
-          on_publish(0, c);
-        }
-        on_publish(1, 0);
-        for (int c = 0; c < nch; ++c) {
-          on_release();
-          on_publish(2, c);
-        }
-        on_publish(3, 0);
-        for (int c = 0; c < ncm; ++c) {
-          on_publish(4, c);
-          on_release();
+        for (int per = 0; per < M; ++per) {
+          cur_nch = P_nch(per);
+          cur_ncm = P_ncm(per);
+          for (int c = 0; c < cur_nch; ++c) {
+            on_release();
+            on_publish(0, c);
+          }
+          on_publish(1, 0);
+          for (int c = 0; c < cur_nch; ++c) {
+            on_release();
+            on_publish(2, c);
+          }
+          on_publish(3, 0);
+          for (int c = 0; c < cur_ncm; ++c) {
+            on_publish(4, c);
+            on_release();
+          }
         }
       }
       // the MMAs of the last groups complete before the CTA releases TMEM
@@ -942,7 +984,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
       }
     }
   };
-  const int hist_tail = n - (nch - 1) * C::DC, mon_tail = p.N - n - (ncm - 1) * C::DC;
+
   uint32_t g = 0;  // group sequence
   auto wait_group = [&](uint32_t gg) {  // group gg's MMAs have completed
     mbar_wait_spin(a_mdone + 8 * (gg & 3), (gg >> 2) & 1);
@@ -969,7 +1011,13 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
   const uint32_t rbase = sm100::opaque(sm100::smem_u32(ring) + (uint32_t)tile * hcap * 512 + 4 * (tid & 127));
 
   int abuf = 0;  // pass-A operand buffer of the current chunk
-  for (int64_t tg = blockIdx.x; tg < tb.ntg; tg += gridDim.x) {
+  for (int64_t tg = blockIdx.x; tg < tb.ntg; tg += gridDim.x)
+  for (int per = 0; per < M; ++per) {
+    // the period's values (f1; the single period of pk / tb otherwise)
+    const MonitorParams &p = MULTI ? mp.per[per].prm : pk;
+    const int nch = P_nch(per), ncm = P_ncm(per), n = p.n;
+    const float *shared_factor = MULTI ? mp.per[per].shared : tb.shared;
+    const int hist_tail = n - (nch - 1) * C::DC, mon_tail = p.N - n - (ncm - 1) * C::DC;
     const int64_t pix = p.p0 + tg * (int64_t)T * 128 + ctid;
     // ================= pass A: masked Gram and moment on the tensor cores
     float c0 = qnan, ymax = 0.f;
@@ -1084,15 +1132,15 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
       // f3 (L93): a warp whose 32 histories have no missing value shares
       // one Gram, factored once on the host in fp64: beta0 = A^-1 (X_hist^T
       // y'), the moment b being the tensor-core GEMM of pass A
-      const bool dense = tb.shared != nullptr && __all_sync(0xffffffffu, nbar == n);
+      const bool dense = shared_factor != nullptr && __all_sync(0xffffffffu, nbar == n);
       float minratio, vif = 0.f;
       if (dense) {
 #pragma unroll
-        for (int i = 0; i < Tri<K>::kN; ++i) A[i] = __ldg(tb.shared + i);
+        for (int i = 0; i < Tri<K>::kN; ++i) A[i] = __ldg(shared_factor + i);
 #pragma unroll
-        for (int i = 0; i < K; ++i) dinv[i] = __ldg(tb.shared + Tri<K>::kN + i);
-        minratio = __ldg(tb.shared + Tri<K>::kN + K);
-        vif = __ldg(tb.shared + Tri<K>::kN + K + 1);
+        for (int i = 0; i < K; ++i) dinv[i] = __ldg(shared_factor + Tri<K>::kN + i);
+        minratio = __ldg(shared_factor + Tri<K>::kN + K);
+        vif = __ldg(shared_factor + Tri<K>::kN + K + 1);
       } else {
         minratio = fz_chol<K>(A, dinv);
       }

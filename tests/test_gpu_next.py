@@ -180,3 +180,48 @@ def test_f4_int16_rejects_misaligned_rows():
     with pytest.raises(binding.BfastError) as e:
         binding.bfast_monitor_i16(codes, dates, 50, 3, 0.25, 1.65, 1e-4, 0.0, -32768, P=1000)
     assert e.value.status == -2  # BFAST_EUNSUPPORTED: TMA rows need ldY % 8 == 0
+
+
+def _yearly(n0, M, year=23):
+    return [(n0 + year * i, n0 + year * (i + 1)) for i in range(M)]
+
+
+@pytest.mark.parametrize("N,periods,k,mask", [
+    (400, _yearly(230, 7), 3, "cloud"),                              # L391: yearly periods from 2010
+    (228, [(114, 228), (100, 180), (60, 77), (150, 201)], 1, "iid"),  # unordered, partial chunks
+    (300, _yearly(120, 8), 5, "iid"),                               # the maximum of 8 periods
+])
+def test_f1_several_periods_in_one_launch(N, periods, k, mask):
+    """Every period against the oracle on its own date slice, and bit-equal
+    to a separate single-period run of the same kernel code."""
+    spec = synth.StackSpec(P=20_000 + 11, N=N, n_hist=periods[0][0], k=k, miss=0.5, mask=mask, seed=1500 + N + k)
+    Y, dates = synth.generate(spec, DEV)
+    out = binding.bfast_monitor_periods(Y, dates, periods, k, spec.hf, spec.lam, diagnostics=True)
+    torch.cuda.synchronize()
+    assert binding.last_launch_count() == 1 + len(periods)
+    Yh = Y.cpu().numpy()
+    orcs = oracle.monitor_periods(Yh, dates, periods, k, spec.hf, spec.lam)
+    for i, ((n_i, N_i), orc) in enumerate(zip(periods, orcs)):
+        gpu = {key: v[i].cpu().numpy() for key, v in out.items() if torch.is_tensor(v)}
+        rep = parity.compare(gpu, orc, dates[:N_i], n_i, k)
+        assert rep["ok"], (i, json.dumps(rep))
+        np.testing.assert_array_equal(gpu["nbar"], orc["nbar"])
+        single = binding.bfast_monitor_ex(Y[:N_i], dates[:N_i], n_i, k, spec.hf, spec.lam, diagnostics=True)
+        torch.cuda.synchronize()
+        np.testing.assert_array_equal(single["break"].cpu().numpy(), gpu["break"])
+        np.testing.assert_array_equal(single["magnitude"].cpu().numpy().view(np.uint32),
+                                      gpu["magnitude"].view(np.uint32))
+
+
+def test_f1_rejects_bad_period_sets():
+    spec = synth.StackSpec(P=1000, N=200, n_hist=100, miss=0.3, seed=5)
+    Y, dates = synth.generate(spec, DEV)
+    with pytest.raises(binding.BfastError) as e:
+        binding.bfast_monitor_periods(Y, dates, [(50 + i, 150 + i) for i in range(9)], 3, 0.25, 1.65)
+    assert e.value.status == -2
+    with pytest.raises(binding.BfastError) as e:
+        binding.bfast_monitor_periods(Y, dates, [(100, 150), (100, 150)], 3, 0.25, 1.65)
+    assert e.value.status == -1
+    with pytest.raises(binding.BfastError) as e:
+        binding.bfast_monitor_periods(Y, dates, [(100, 201)], 3, 0.25, 1.65)
+    assert e.value.status == -1

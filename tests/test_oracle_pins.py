@@ -466,3 +466,27 @@ def test_p11_decode_i16_is_one_rounding_of_the_exact_value():
     ok = codes != 7
     assert np.array_equal(y2[ok].astype(np.float64), codes[ok].astype(np.float64) * 2.0 ** -14 + 0.5)
     assert np.isnan(y2[~ok]).all()
+
+
+def test_p12_periods_use_only_their_own_dates():
+    """f1 (L391): a period (n_i, N_i) is Algorithm 1 on the first N_i dates:
+    its result does not change when every date at or after N_i is replaced,
+    and the period ending at N equals the single-period oracle."""
+    rng = np.random.default_rng(12)
+    N, P = 160, 300
+    dates = 2000.0 + np.arange(1, N + 1) / 23.0
+    t = np.arange(N)[:, None]
+    Y = (0.5 + 0.1 * np.sin(2 * np.pi * dates)[:, None] + 0.02 * rng.normal(size=(N, P))).astype(np.float32)
+    Y[rng.random((N, P)) < 0.3] = np.nan
+    Y -= (np.float32(0.3) * ((t >= 120) & (rng.random(P) < 0.5)[None, :])).astype(np.float32)
+    periods = [(80, 103), (103, 126), (126, 160)]
+    res = oracle.monitor_periods(Y, dates, periods, 3, 0.25, 1.65)
+    Y2 = Y.copy()
+    Y2[103:] = np.float32(7.0)
+    r2 = oracle.monitor_periods(Y2, dates, periods[:1], 3, 0.25, 1.65)[0]
+    for key in ("break", "magnitude", "sigma", "nbar"):
+        np.testing.assert_array_equal(res[0][key], r2[key])
+    full = oracle.monitor(Y, dates, 126, 3, 0.25, 1.65)
+    for key in ("break", "magnitude", "nbar"):
+        np.testing.assert_array_equal(res[2][key], full[key])
+    assert (res[2]["break"] >= 0).sum() > 50  # the step at t = 120 is inside period 3 only
