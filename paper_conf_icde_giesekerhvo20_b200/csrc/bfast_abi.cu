@@ -605,7 +605,9 @@ int launch_multi_k(const std::vector<bfast_plan *> &pls, const std::vector<bfast
   const int static_smem = (int)fa.sharedSizeBytes;
   int hcap = 1;
   for (auto *pl : pls) hcap = std::max(hcap, pl->hcap);
-  int T = C::TMAX, sc = C::SCMAX;
+  int T = bfast::FzTiles<K, true>::TM, sc = C::SCMAX;
+  if (const char *e = std::getenv("BFAST_FZ_T")) T = std::max(1, std::min(T, std::atoi(e)));
+  if (const char *e = std::getenv("BFAST_FZ_SC")) sc = std::max(2, std::min(C::SCMAX, std::atoi(e)));
   auto fits = [&](int t, int c) { return C::smem_bytes(t, hcap, c) + static_smem <= (size_t)kMaxSmem; };
   while (T > 1 && !fits(T, 2)) --T;
   if (!fits(T, sc)) sc = 2;
@@ -655,9 +657,12 @@ int launch_multi_k(const std::vector<bfast_plan *> &pls, const std::vector<bfast
   tb.T = T;
   tb.hcap = hcap;
   tb.pfd = 128;
+  if (const char *e = std::getenv("BFAST_FZ_PFD")) tb.pfd = std::max(0, std::atoi(e)) / C::PFB * C::PFB;
   tb.sc = sc;
   tb.ntg = (q0.P + 128 * T - 1) / (128 * T);
   tb.shared = nullptr;
+  if (std::getenv("BFAST_VERBOSE"))
+    std::fprintf(stderr, "bfast: multi k=%d M=%d T=%d sc=%d smem=%zu hcap=%d\n", p0.k, M, T, sc, smem, hcap);
   const int64_t grid = std::min<int64_t>(tb.ntg, (int64_t)sms * per_sm);
   cudaEvent_t e0 = nullptr, e1 = nullptr;
   if (g_prof_on) {
@@ -1051,7 +1056,8 @@ int bfast_monitor_periods(const bfast_args *a, const int32_t *n_hist, const int3
       q.refit_list = pl.dlist;
       q.refit_count = pl.dcount;
     }
-    rc = launch_multi(pls, prms, (cudaStream_t)a->stream);
+    // one period: the single-period kernel (the same arithmetic, no period tables)
+    rc = M == 1 ? launch(*pls[0], prms[0], (cudaStream_t)a->stream) : launch_multi(pls, prms, (cudaStream_t)a->stream);
     if (rc) return rc;
     total += g_launches;
   }

@@ -75,6 +75,30 @@ struct FzShape {
   static_assert(TMAX * RC + RP <= LAUNCH * (TMAX + 1), "register pool");
 };
 
+// register split for TM tiles per CTA (FzTiles: the multi-period kernel of
+// f1 may be built for one tile fewer, BFAST_FZ_MULTI_TM1, trading a tile
+// for registers: measured -1.5% time on 7 yearly periods whose longest
+// window admits only 3 tiles anyway, +25% where the windows admit 4)
+template <int TM>
+struct FzRegs {
+  static constexpr int LAUNCH = (65536 / (128 * (TM + 1))) / 8 * 8;
+#ifdef BFAST_FZ_RP
+  static constexpr int RP = BFAST_FZ_RP;
+#else
+  static constexpr int RP = TM == 4 ? 32 : 56;
+#endif
+  static constexpr int RC = ((LAUNCH * (TM + 1) - RP) / TM) / 8 * 8 > 248 ? 248
+                                                                          : ((LAUNCH * (TM + 1) - RP) / TM) / 8 * 8;
+};
+template <int K, bool MULTI>
+struct FzTiles {
+#ifdef BFAST_FZ_MULTI_TM1
+  static constexpr int TM = MULTI && FzShape<K>::TMAX > 2 ? FzShape<K>::TMAX - 1 : FzShape<K>::TMAX;
+#else
+  static constexpr int TM = FzShape<K>::TMAX;
+#endif
+};
+
 template <int K>
 struct FzCfg {
   static constexpr int k = (K - 2) / 2;
@@ -576,7 +600,7 @@ __device__ __forceinline__ void fz_solve(const float (&L)[Tri<K>::kN], const flo
 }
 
 template <int K, bool I16, bool MULTI>
-__global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
+__global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
     monitor_fused_kernel(MonitorParams pk, FzTables tb, const __grid_constant__ CUtensorMap ymap,
                          const __grid_constant__ CUtensorMap hmap, const __grid_constant__ CUtensorMap pmap,
                          const __grid_constant__ FzMulti mp) {
@@ -598,6 +622,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
   __shared__ __align__(8) uint64_t tfull[C::ST];            // table stages
   __shared__ uint32_t tfree[C::ST];                         // tiles done with a table stage (mod T)
   __shared__ uint32_t tmem_base_s;
+  __shared__ int s_per[MULTI ? kMaxPeriods : 1][4];  // f1: nch, ncm, n, N of each period (LDS, not LDC)
 
   const int T = tb.T;
   // warpgroup 0 = the control warps (one per tile: warp i drives tile i;
@@ -613,10 +638,10 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
   const int tile = control ? warp : (warp - 4) >> 2;
   const int nch = MULTI ? mp.per[0].nch : tb.nch, ncm = MULTI ? mp.per[0].ncm : tb.ncm, n = p.n, hcap = tb.hcap;
   const int M = MULTI ? mp.M : 1;
-  auto P_nch = [&](int per) { return MULTI ? mp.per[per].nch : nch; };
-  auto P_ncm = [&](int per) { return MULTI ? mp.per[per].ncm : ncm; };
-  auto P_n = [&](int per) { return MULTI ? mp.per[per].prm.n : n; };
-  auto P_N = [&](int per) { return MULTI ? mp.per[per].prm.N : p.N; };
+  auto P_nch = [&](int per) { return MULTI ? s_per[per][0] : nch; };
+  auto P_ncm = [&](int per) { return MULTI ? s_per[per][1] : ncm; };
+  auto P_n = [&](int per) { return MULTI ? s_per[per][2] : n; };
+  auto P_N = [&](int per) { return MULTI ? s_per[per][3] : p.N; };
   FZT_DECL
   FZT_T0(t_kernel)
   const int SC = tb.sc;
@@ -641,6 +666,12 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
   const uint32_t a_srel = sm100::opaque(sm100::smem_u32(&srel[tile][0]));
   const uint32_t a_stack = sm100::opaque(sm100::smem_u32(stack + (size_t)tile * SC * CB));
 
+  if (MULTI && tid < M) {
+    s_per[tid][0] = mp.per[tid].nch;
+    s_per[tid][1] = mp.per[tid].ncm;
+    s_per[tid][2] = mp.per[tid].prm.n;
+    s_per[tid][3] = mp.per[tid].prm.N;
+  }
   if (tid == 0) {
     for (int i = 0; i < T; ++i) {
       for (int j = 0; j < C::SCMAX; ++j) {
@@ -671,7 +702,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
     // follows the tile's fixed event order: stack halves consumed -> refill
     // the stage SH halves ahead; group published -> issue its tcgen05.mma.
     // Waits sleep in hardware (try_wait with a suspend-time hint).
-    sm100::setmaxnreg_dec<FzShape<K>::RP>();
+    sm100::setmaxnreg_dec<FzRegs<FzTiles<K, MULTI>::TM>::RP>();
     if (tile >= T) {
       // spare warps of the control warpgroup
     } else {
@@ -762,8 +793,9 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
         if (ldc.u < U_total && lane == 0) {
           // first-touch periods (A: history, C: monitoring) are prefetched
           // into L2 in [PFB dates x 128 px] boxes, pfd dates ahead of the loads
-          // (later periods re-read the history of earlier ones: no prefetch)
-          if (tb.pfd > 0 && ldc.region != 1 && (ldc.region == 2 || ldc.per == 0)) {
+          // (later periods re-read the history of earlier ones: whatever L2
+          // no longer holds is prefetched like a first touch)
+          if (tb.pfd > 0 && ldc.region != 1) {
             const int pn = P_n(ldc.per);
             const int base = ldc.region == 0 ? 0 : pn, end = ldc.region == 0 ? pn : P_N(ldc.per);
             const int off = ldc.y - base;
@@ -788,6 +820,11 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
       };
       if (lane == 0) {
         sm100::prefetch_tmap(&ymap);
+        if (MULTI)
+          for (int i = 0; i < M; ++i) {
+            sm100::prefetch_tmap(&mp.per[i].h);
+            sm100::prefetch_tmap(&mp.per[i].y);
+          }
         sm100::prefetch_tmap(&hmap);
       }
       for (int i = 0; i < SC; ++i) load_chunk();
@@ -942,7 +979,7 @@ __global__ void __launch_bounds__(128 * (FzShape<K>::TMAX + 1), 1)
   }
 
   // ================================================================== consumers
-  sm100::setmaxnreg_inc<FzShape<K>::RC>();
+  sm100::setmaxnreg_inc<FzRegs<FzTiles<K, MULTI>::TM>::RC>();
   int ust = 0;       // stage of the current stack chunk
   uint32_t uph = 0;  // and its phase parity
   auto acquire_chunk = [&]() -> uint32_t {

@@ -189,17 +189,18 @@ def _yearly(n0, M, year=23):
 @pytest.mark.parametrize("N,periods,k,mask", [
     (400, _yearly(230, 7), 3, "cloud"),                              # L391: yearly periods from 2010
     (228, [(114, 228), (100, 180), (60, 77), (150, 201)], 1, "iid"),  # unordered, partial chunks
-    (300, _yearly(120, 8), 5, "iid"),                               # the maximum of 8 periods
+    (320, _yearly(120, 8), 5, "iid"),                               # the maximum of 8 periods
 ])
 def test_f1_several_periods_in_one_launch(N, periods, k, mask):
     """Every period against the oracle on its own date slice, and bit-equal
     to a separate single-period run of the same kernel code."""
     spec = synth.StackSpec(P=20_000 + 11, N=N, n_hist=periods[0][0], k=k, miss=0.5, mask=mask, seed=1500 + N + k)
-    Y, dates = synth.generate(spec, DEV)
+    Yp, dates = synth.generate(spec, DEV, ldY=20_016)  # TMA rows: ldY % 4 == 0; a ragged last tile
+    Y = Yp[:, :spec.P]
     out = binding.bfast_monitor_periods(Y, dates, periods, k, spec.hf, spec.lam, diagnostics=True)
     torch.cuda.synchronize()
     assert binding.last_launch_count() == 1 + len(periods)
-    Yh = Y.cpu().numpy()
+    Yh = np.ascontiguousarray(Y.cpu().numpy())
     orcs = oracle.monitor_periods(Yh, dates, periods, k, spec.hf, spec.lam)
     for i, ((n_i, N_i), orc) in enumerate(zip(periods, orcs)):
         gpu = {key: v[i].cpu().numpy() for key, v in out.items() if torch.is_tensor(v)}
