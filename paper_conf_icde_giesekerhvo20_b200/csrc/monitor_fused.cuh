@@ -1,7 +1,12 @@
 // monitor_fused.cuh -- the BFAST-Monitor hot path as one persistent kernel
 // per SM: every (pixel, date) step on the CUDA cores, every contraction a
-// tile of 128 pixels shares on the 5th-generation tensor cores, and no
-// thread whose only job is to wait.
+// tile of 128 pixels shares on the 5th-generation tensor cores, one control
+// warp per tile that only moves data (TMA) and issues tcgen05.mma.
+//
+// Variants (template parameters): I16 -- the stack as scaled int16 codes
+// (SURVEY 8(f) f4); MULTI -- several monitoring periods per stack pass
+// (f1, FzMulti).  NaN-free histories share one host-factored Gram (f3,
+// FzTables::shared).
 //
 // Algorithm 1, Fig. 12 (L478-L537); readings R1-R14 of
 // DESIGN.md.  Per tile of 128 pixels (one pixel per thread = one TMEM lane),
@@ -78,7 +83,7 @@ struct FzShape {
 // register split for TM tiles per CTA (FzTiles: the multi-period kernel of
 // f1 may be built for one tile fewer, BFAST_FZ_MULTI_TM1, trading a tile
 // for registers: measured -1.5% time on 7 yearly periods whose longest
-// window admits only 3 tiles anyway, +25% where the windows admit 4)
+// window admits only 3 tiles anyway, +17% where the windows admit 4)
 template <int TM>
 struct FzRegs {
   static constexpr int LAUNCH = (65536 / (128 * (TM + 1))) / 8 * 8;
