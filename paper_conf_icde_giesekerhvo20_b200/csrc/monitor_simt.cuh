@@ -198,7 +198,7 @@ __device__ __forceinline__ void store_beta(const MonitorParams &p, int64_t pix, 
 constexpr int kUnroll = 8;
 
 template <int K>
-__global__ void __launch_bounds__(128, 4) monitor_simt_kernel(MonitorParams p) {
+__global__ void __launch_bounds__(128, K >= 12 ? 2 : 4) monitor_simt_kernel(MonitorParams p) {
   extern __shared__ float4 smem4[];
   const int KP = p.KP;
   float *sX = reinterpret_cast<float *>(smem4);
