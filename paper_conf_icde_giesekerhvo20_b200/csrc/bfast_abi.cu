@@ -102,6 +102,11 @@ struct bfast_plan {
     float *dY[2] = {nullptr, nullptr};
     int32_t *dB[2] = {nullptr, nullptr};
     float *dM[2] = {nullptr, nullptr};
+    // pinned staging of each slab's results: a D2H into pageable caller
+    // memory would block the host thread until the slab's kernel is done and
+    // so serialise the next slab's upload behind it
+    int32_t *hB[2] = {nullptr, nullptr};
+    float *hM[2] = {nullptr, nullptr};
     cudaStream_t cs = nullptr, ks = nullptr;
     cudaEvent_t loaded[2] = {nullptr, nullptr}, done[2] = {nullptr, nullptr};
   } host;
@@ -131,6 +136,8 @@ struct bfast_plan {
       cudaFree(host.dY[i]);
       cudaFree(host.dB[i]);
       cudaFree(host.dM[i]);
+      cudaFreeHost(host.hB[i]);
+      cudaFreeHost(host.hM[i]);
       if (host.loaded[i]) cudaEventDestroy(host.loaded[i]);
       if (host.done[i]) cudaEventDestroy(host.done[i]);
     }
@@ -1128,15 +1135,21 @@ int host_path_ensure(bfast_plan &pl, int64_t slab) {
     cudaFree(hp.dY[i]);
     cudaFree(hp.dB[i]);
     cudaFree(hp.dM[i]);
+    cudaFreeHost(hp.hB[i]);
+    cudaFreeHost(hp.hM[i]);
     hp.dY[i] = nullptr;
     hp.dB[i] = nullptr;
     hp.dM[i] = nullptr;
+    hp.hB[i] = nullptr;
+    hp.hM[i] = nullptr;
   }
   hp.slab = 0;
   for (int i = 0; i < 2; ++i) {
     CUDA_TRY(cudaMalloc(&hp.dY[i], sizeof(float) * (size_t)pl.N * slab));
     CUDA_TRY(cudaMalloc(&hp.dB[i], sizeof(int32_t) * slab));
     CUDA_TRY(cudaMalloc(&hp.dM[i], sizeof(float) * slab));
+    CUDA_TRY(cudaMallocHost(&hp.hB[i], sizeof(int32_t) * slab));
+    CUDA_TRY(cudaMallocHost(&hp.hM[i], sizeof(float) * slab));
   }
   hp.slab = slab;
   return BFAST_OK;
@@ -1175,6 +1188,19 @@ int bfast_monitor_host(const float *Y_host, int64_t N, int64_t P, int64_t ldY, c
   int launches = 0;
   cudaError_t e = cudaSuccess;
   int slot = 0;
+  // results of the previous slab, drained to the caller's arrays from the
+  // pinned staging once its D2H is done (while the next upload runs)
+  int64_t pend_b = -1, pend_w = 0;
+  int pend_slot = 0;
+  auto drain = [&]() -> cudaError_t {
+    if (pend_b < 0) return cudaSuccess;
+    const cudaError_t ee = cudaEventSynchronize(hp.done[pend_slot]);
+    if (ee != cudaSuccess) return ee;
+    std::memcpy(out_break_host + pend_b, hp.hB[pend_slot], sizeof(int32_t) * pend_w);
+    std::memcpy(out_magnitude_host + pend_b, hp.hM[pend_slot], sizeof(float) * pend_w);
+    pend_b = -1;
+    return cudaSuccess;
+  };
   for (int64_t b0 = 0; b0 < P && rc == BFAST_OK; b0 += slab, slot ^= 1) {
     const int64_t w = std::min(slab, P - b0);
     // the buffer is free once the kernel that used it two slabs ago is done
@@ -1201,12 +1227,17 @@ int bfast_monitor_host(const float *Y_host, int64_t N, int64_t P, int64_t ldY, c
     rc = execute_range(*pl, &a, 0, w);
     launches += g_launches;
     if (rc) break;
-    e = cudaMemcpyAsync(out_break_host + b0, hp.dB[slot], sizeof(int32_t) * w, cudaMemcpyDeviceToHost, hp.ks);
+    e = cudaMemcpyAsync(hp.hB[slot], hp.dB[slot], sizeof(int32_t) * w, cudaMemcpyDeviceToHost, hp.ks);
     if (e == cudaSuccess)
-      e = cudaMemcpyAsync(out_magnitude_host + b0, hp.dM[slot], sizeof(float) * w, cudaMemcpyDeviceToHost, hp.ks);
+      e = cudaMemcpyAsync(hp.hM[slot], hp.dM[slot], sizeof(float) * w, cudaMemcpyDeviceToHost, hp.ks);
     if (e == cudaSuccess) e = cudaEventRecord(hp.done[slot], hp.ks);
+    if (e == cudaSuccess) e = drain();  // the slab before this one
     if (e != cudaSuccess) break;
+    pend_b = b0;
+    pend_w = w;
+    pend_slot = slot;
   }
+  if (e == cudaSuccess && rc == BFAST_OK) e = drain();
   const cudaError_t es = cudaStreamSynchronize(hp.ks);
   if (rc) return rc;
   if (e == cudaSuccess) e = es;
