@@ -475,7 +475,7 @@ int launch_fused(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStre
     return BFAST_OK;
   int pfd = 128;
   if (const char *e = std::getenv("BFAST_FZ_PFD")) pfd = std::max(0, std::atoi(e)) / C::PFB * C::PFB;
-  bfast::FzTables tb;
+  bfast::FzTables tb{};
   tb.tabA = pl.dtabf;
   tb.tabB = pl.dtabf + pl.tabfB_off;
   tb.tabC = pl.dtabf + pl.tabfC_off;

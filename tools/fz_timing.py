@@ -17,14 +17,24 @@ NAMES = ["cons A: wait operand buffer (g-2)", "cons: wait yhat", "-", "cons: acq
          "ctl: on_publish work (after the wait)", "ctl: wait publish", "ctl: wait table", "ctl: wait release",
          "kernel (per warp, all warps)", "cons: solve wait Gram", "cons: refine wait db", "-",
          "ctl: load_half (TMA issue)", "ctl: wait mdone g-1 (table release)"]
-spec = synth.CONFIGS[sys.argv[2] if len(sys.argv) > 2 else "landsat"]
+mode = sys.argv[2] if len(sys.argv) > 2 else "landsat"
+spec = synth.CONFIGS["landsat" if mode in ("periods", "single7") else mode]
 Y, dates = synth.generate(spec, "cuda:0")
+PER = [(230 + 23 * i, 253 + 23 * i) for i in range(7)]
+
+
+def run():
+    if mode == "periods":  # f1: one multi-period launch
+        return binding.bfast_monitor_periods(Y, dates, PER, spec.k, spec.hf, spec.lam)
+    if mode == "single7":  # the same periods as separate launches
+        return [binding.bfast_monitor_ex(Y[:e], dates[:e], b, spec.k, spec.hf, spec.lam) for b, e in PER]
+    return binding.bfast_monitor_ex(Y, dates, spec.n_hist, spec.k, spec.hf, spec.lam)
 L = binding.lib()
 L.bfast_debug_fz_timing.argtypes = [ctypes.c_void_p, ctypes.c_int]
 buf = (ctypes.c_ulonglong * 16)()
 for rep in range(2):
     L.bfast_debug_fz_timing(buf, 16)
-    out = binding.bfast_monitor_ex(Y, dates, spec.n_hist, spec.k, spec.hf, spec.lam)
+    out = run()
     torch.cuda.synchronize()
 L.bfast_debug_fz_timing(buf, 16)
 tot = buf[8]
