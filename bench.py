@@ -268,7 +268,11 @@ def run_reference(args):
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": desc, "sample": f"{sub.P} pixels per step (same recipe, CPU sub-scene)"},
+            "config": {"workload": desc, "sample": f"{sub.P} pixels per step (same recipe, CPU sub-scene)",
+                       "same_config": False,
+                       "note": "a bounded sample of the workload: the same N, n, k, h, lambda and missing-value "
+                               "recipe on a sub-scene of P pixels; the oracle's work per pixel does not depend "
+                               "on P, so pixels/s compares with the GPU line"},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
                              "sample": f"{sub.P} pixels of the workload per step", "host": host_cpu()},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
