@@ -218,6 +218,9 @@ int bfast_monitor_shards(const float *const *Y_dev, const int64_t *P, const int6
  * [M][P], out_magnitude float [M][P], optional out_beta [M][P][K],
  * out_sigma / out_nbar / out_flags [M][P].  Result of period i = that of
  * bfast_monitor_ex on the first N_end[i] dates with n_hist[i].
+ * Environment: BFAST_PERIODS=split runs the periods as separate launches
+ * instead (the same results bit for bit; each period then reads its slice
+ * of the stack from HBM -- measured faster on B200).
  * Requirements: 1 <= M <= 8 distinct periods, each valid as a bfast_args
  * (n_hist[i] in [1, N_end[i] - 1], N_end[i] <= a->N); the fused kernel
  * (16-byte aligned Y, ldY % 4 == 0).  Errors: BFAST_EINVAL (NULL arrays,

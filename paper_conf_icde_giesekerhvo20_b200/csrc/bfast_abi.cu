@@ -1063,10 +1063,22 @@ int bfast_monitor_periods(const bfast_args *a, const int32_t *n_hist, const int3
       q.refit_list = pl.dlist;
       q.refit_count = pl.dcount;
     }
-    // one period: the single-period kernel (the same arithmetic, no period tables)
-    rc = M == 1 ? launch(*pls[0], prms[0], (cudaStream_t)a->stream) : launch_multi(pls, prms, (cudaStream_t)a->stream);
-    if (rc) return rc;
-    total += g_launches;
+    // one period: the single-period kernel (the same arithmetic, no period
+    // tables).  BFAST_PERIODS=split runs every period as its own launch
+    // (each reads its slice of the stack from HBM): on this issue-bound
+    // kernel that is the faster schedule (f1)
+    const char *pm = std::getenv("BFAST_PERIODS");
+    if (M == 1 || (pm && std::strcmp(pm, "split") == 0)) {
+      for (int i = 0; i < M; ++i) {
+        rc = launch(*pls[i], prms[i], (cudaStream_t)a->stream);
+        if (rc) return rc;
+        total += g_launches;
+      }
+    } else {
+      rc = launch_multi(pls, prms, (cudaStream_t)a->stream);
+      if (rc) return rc;
+      total += g_launches;
+    }
   }
   g_launches = total;
   return BFAST_OK;

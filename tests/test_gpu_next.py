@@ -214,6 +214,24 @@ def test_f1_several_periods_in_one_launch(N, periods, k, mask):
                                       gpu["magnitude"].view(np.uint32))
 
 
+def test_f1_split_schedule_is_bit_identical(monkeypatch):
+    """BFAST_PERIODS=split (one launch per period) gives the bytes of the
+    one-pass launch."""
+    spec = synth.StackSpec(P=30_000, N=400, n_hist=230, miss=0.6, mask="cloud", seed=1577)
+    Y, dates = synth.generate(spec, DEV)
+    per = _yearly(230, 5)
+    a = binding.bfast_monitor_periods(Y, dates, per, 3, spec.hf, spec.lam, diagnostics=True)
+    torch.cuda.synchronize()
+    assert binding.last_launch_count() == 1 + len(per)
+    monkeypatch.setenv("BFAST_PERIODS", "split")
+    b = binding.bfast_monitor_periods(Y, dates, per, 3, spec.hf, spec.lam, diagnostics=True)
+    torch.cuda.synchronize()
+    assert binding.last_launch_count() == 2 * len(per)
+    for key in ("break", "magnitude", "beta", "sigma", "nbar"):
+        assert torch.equal(a[key].view(torch.int32) if a[key].dtype == torch.float32 else a[key],
+                           b[key].view(torch.int32) if b[key].dtype == torch.float32 else b[key]), key
+
+
 def test_f1_rejects_bad_period_sets():
     spec = synth.StackSpec(P=1000, N=200, n_hist=100, miss=0.3, seed=5)
     Y, dates = synth.generate(spec, DEV)
