@@ -244,3 +244,33 @@ def test_f1_rejects_bad_period_sets():
     with pytest.raises(binding.BfastError) as e:
         binding.bfast_monitor_periods(Y, dates, [(100, 201)], 3, 0.25, 1.65)
     assert e.value.status == -1
+
+
+def test_f2_edge_cases():
+    """An all-empty stack keeps no date; P = 0 and Nc = 0 are no-ops; a stack
+    without empty slices keeps every date."""
+    spec = synth.StackSpec(P=5000, N=64, n_hist=32, miss=0.3, seed=961)
+    Y, dates = synth.generate(spec, DEV)
+    keep = binding.bfast_valid_dates(Y).cpu().numpy()
+    assert keep.tolist() == [1] * 64
+    Yn = torch.full_like(Y, float("nan"))
+    assert binding.bfast_valid_dates(Yn).cpu().numpy().sum() == 0
+    Yc, dc, nc, kept = binding.drop_empty_dates(Yn, dates, spec.n_hist)
+    assert Yc.shape == (0, spec.P) and nc == 0 and len(kept) == 0
+    assert binding.bfast_valid_dates(Y, P=0).cpu().numpy().sum() == 0
+
+
+@pytest.mark.parametrize("k", [4, 5, 6])
+def test_f4_int16_wide_designs(k):
+    """The int16 kernel at the wide designs (K = 10, 12, 14: fewer tiles per
+    CTA, more TMEM per tile)."""
+    spec = synth.StackSpec(P=12_000, N=300, n_hist=150, k=k, miss=0.4, mask="iid", seed=1700 + k)
+    Y, dates = synth.generate(spec, DEV)
+    codes = synth.quantize_i16(Y, 1e-4, 0.0, -32768)
+    out = binding.bfast_monitor_i16(codes, dates, 150, k, spec.hf, spec.lam, 1e-4, 0.0, -32768, diagnostics=True)
+    torch.cuda.synchronize()
+    Yd = oracle.decode_i16(codes.cpu().numpy(), np.float32(1e-4), np.float32(0.0), -32768)
+    orc = oracle.monitor(np.ascontiguousarray(Yd), dates, 150, k, spec.hf, spec.lam)
+    gpu = {key: v.cpu().numpy() for key, v in out.items() if torch.is_tensor(v)}
+    rep = parity.compare(gpu, orc, dates, 150, k)
+    assert rep["ok"], json.dumps(rep)
