@@ -453,6 +453,7 @@ int launch_fused(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStre
   if (const char *e = std::getenv("BFAST_FZ_SC")) sc = std::max(2, std::min(C::SCMAX, std::atoi(e)));
   auto fits = [&](int t, int c) { return C::smem_bytes(t, pl.hcap, c, esz) + static_smem <= (size_t)kMaxSmem; };
   while (T > 1 && !fits(T, 2)) --T;
+  T = std::max(C::TPC, T / C::TPC * C::TPC);  // whole control groups
   if (!fits(T, sc)) sc = 2;
   const size_t smem = C::smem_bytes(T, pl.hcap, sc, esz);
   if (smem + static_smem > (size_t)kMaxSmem)
@@ -469,9 +470,9 @@ int launch_fused(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStre
   const int per_sm = std::max(1, std::min(std::min(by_smem, by_tmem), std::min(by_regs, by_thr)));
   // full stack; history only (dates >= n out of bounds -> NaN); L2 prefetch boxes
   CUtensorMap ymap, hmap, pmap;
-  if (!make_stack_map(&ymap, Ybase, prm.ldY, prm.P, pl.N, 128, 16, I16) ||
-      !make_stack_map(&hmap, Ybase, prm.ldY, prm.P, pl.n, 128, 16, I16) ||
-      !make_stack_map(&pmap, Ybase, prm.ldY, prm.P, pl.N, 128, C::PFB, I16))
+  if (!make_stack_map(&ymap, Ybase, prm.ldY, prm.P, pl.N, 128 * C::TPC, 16, I16) ||
+      !make_stack_map(&hmap, Ybase, prm.ldY, prm.P, pl.n, 128 * C::TPC, 16, I16) ||
+      !make_stack_map(&pmap, Ybase, prm.ldY, prm.P, pl.N, 128 * C::TPC, C::PFB, I16))
     return BFAST_OK;
   int pfd = 128;
   if (const char *e = std::getenv("BFAST_FZ_PFD")) pfd = std::max(0, std::atoi(e)) / C::PFB * C::PFB;
@@ -617,6 +618,7 @@ int launch_multi_k(const std::vector<bfast_plan *> &pls, const std::vector<bfast
   if (const char *e = std::getenv("BFAST_FZ_SC")) sc = std::max(2, std::min(C::SCMAX, std::atoi(e)));
   auto fits = [&](int t, int c) { return C::smem_bytes(t, hcap, c) + static_smem <= (size_t)kMaxSmem; };
   while (T > 1 && !fits(T, 2)) --T;
+  T = std::max(C::TPC, T / C::TPC * C::TPC);  // whole control groups
   if (!fits(T, sc)) sc = 2;
   const size_t smem = C::smem_bytes(T, hcap, sc);
   if (smem + static_smem > (size_t)kMaxSmem)
@@ -644,14 +646,14 @@ int launch_multi_k(const std::vector<bfast_plan *> &pls, const std::vector<bfast
     fp.nch = pl.nch;
     fp.ncm = pl.ncm;
     mp->Lg += 2 * pl.nch + pl.ncm;
-    if (!make_stack_map(&fp.h, prms[i].Y + prms[i].p0, prms[i].ldY, prms[i].P, pl.n, 128, 16) ||
-        !make_stack_map(&fp.y, prms[i].Y + prms[i].p0, prms[i].ldY, prms[i].P, pl.N, 128, 16))
+    if (!make_stack_map(&fp.h, prms[i].Y + prms[i].p0, prms[i].ldY, prms[i].P, pl.n, 128 * C::TPC, 16) ||
+        !make_stack_map(&fp.y, prms[i].Y + prms[i].p0, prms[i].ldY, prms[i].P, pl.N, 128 * C::TPC, 16))
       return fail(BFAST_EUNSUPPORTED, "tensor maps of the stack");
   }
   int64_t Nmax = 0;
   for (auto *pl : pls) Nmax = std::max<int64_t>(Nmax, pl->N);
   CUtensorMap pmap;
-  if (!make_stack_map(&pmap, q0.Y + q0.p0, q0.ldY, q0.P, Nmax, 128, C::PFB))
+  if (!make_stack_map(&pmap, q0.Y + q0.p0, q0.ldY, q0.P, Nmax, 128 * C::TPC, C::PFB))
     return fail(BFAST_EUNSUPPORTED, "tensor maps of the stack");
   for (auto *pl : pls) CUDA_TRY(cudaStreamWaitEvent(st, pl->scratch_free, 0));
   for (int i = 0; i < M; ++i) CUDA_TRY(cudaMemsetAsync(prms[i].refit_count, 0, sizeof(int32_t), st));

@@ -104,6 +104,12 @@ struct FzTiles {
 #endif
 };
 
+// tiles per control warp (BFAST_FZ_TPC): 2 = one control warp drives a pair
+// of tiles in lockstep (one stack box of 256 px, one MMA event per pair)
+#ifndef BFAST_FZ_TPC
+#define BFAST_FZ_TPC 1
+#endif
+
 template <int K>
 struct FzCfg {
   static constexpr int k = (K - 2) / 2;
@@ -152,6 +158,7 @@ struct FzCfg {
   static constexpr int PFB = 64;                 // dates per L2-prefetch box
   static constexpr int SCMAX = 3;                // stack chunk stages per tile (2 or 3, by shared memory)
   static constexpr int CBYTES = DC * 128 * 4;    // one [16 dates x 128 px] box (8 KB; 4 KB of int16 codes)
+  static constexpr int TPC = BFAST_FZ_TPC;
   static constexpr size_t smem_bytes(int T, int hcap, int sc, int esz = 4) {
     return (size_t)T * sc * (CBYTES / 4 * esz) + (size_t)ST * TSTAGE + (size_t)T * hcap * 512;
   }
@@ -613,7 +620,8 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
   const MonitorParams &p = MULTI ? mp.per[0].prm : pk;
   using C = FzCfg<K>;
   constexpr int ESZ = I16 ? 2 : 4;           // bytes per stack element
-  constexpr int CB = C::CBYTES / 4 * ESZ;    // one [16 dates x 128 px] box
+  constexpr int TPC = C::TPC;                // tiles per control warp
+  constexpr int CB = C::CBYTES / 4 * ESZ * TPC;  // one [16 dates x 128 TPC px] box (a group's stage)
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ __align__(8) uint64_t sfull[C::TMAX][C::SCMAX];  // stack chunk stage landed (TMA tx)
   __shared__ __align__(8) uint64_t srel[C::TMAX][C::SCMAX];   // the tile's 4 warps consumed it
@@ -641,6 +649,9 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
   const bool control = warp < 4;
   const int ctid = tid - 128;  // consumer thread index = pixel of the tile group
   const int tile = control ? warp : (warp - 4) >> 2;
+  // control group: tiles grp * TPC ... grp * TPC + TPC - 1 share one control
+  // warp (warp grp), its barriers and its stack stages; sub = tile in group
+  const int grp = control ? warp : tile / TPC, sub = control ? 0 : tile % TPC;
   const int nch = MULTI ? mp.per[0].nch : tb.nch, ncm = MULTI ? mp.per[0].ncm : tb.ncm, n = p.n, hcap = tb.hcap;
   const int M = MULTI ? mp.M : 1;
   auto P_nch = [&](int per) { return MULTI ? s_per[per][0] : nch; };
@@ -651,7 +662,7 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
   FZT_T0(t_kernel)
   const int SC = tb.sc;
   uint8_t *stack = smem;
-  uint8_t *tabs = stack + (size_t)T * SC * CB;
+  uint8_t *tabs = stack + (size_t)(T / TPC) * SC * CB;
   uint8_t *ring = tabs + (size_t)C::ST * C::TSTAGE;
 
   // chunk sequence per tile group: A[0, nch), B[0, nch), C[0, ncm) (per period)
@@ -664,12 +675,12 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
   const uint32_t a_tabs = sm100::opaque(sm100::smem_u32(tabs));
   const uint32_t a_tfull = sm100::opaque(sm100::smem_u32(&tfull[0]));
   const uint32_t a_tfree = sm100::opaque(sm100::smem_u32(&tfree[0]));
-  const uint32_t a_mdone = sm100::opaque(sm100::smem_u32(&mdone[tile][0]));
-  const uint32_t a_ybar = sm100::opaque(sm100::smem_u32(&ybar[tile][0]));
-  const uint32_t a_pub = sm100::opaque(sm100::smem_u32(&pub[tile][0]));
-  const uint32_t a_sfull = sm100::opaque(sm100::smem_u32(&sfull[tile][0]));
-  const uint32_t a_srel = sm100::opaque(sm100::smem_u32(&srel[tile][0]));
-  const uint32_t a_stack = sm100::opaque(sm100::smem_u32(stack + (size_t)tile * SC * CB));
+  const uint32_t a_mdone = sm100::opaque(sm100::smem_u32(&mdone[grp][0]));
+  const uint32_t a_ybar = sm100::opaque(sm100::smem_u32(&ybar[grp][0]));
+  const uint32_t a_pub = sm100::opaque(sm100::smem_u32(&pub[grp][0]));
+  const uint32_t a_sfull = sm100::opaque(sm100::smem_u32(&sfull[grp][0]));
+  const uint32_t a_srel = sm100::opaque(sm100::smem_u32(&srel[grp][0]));
+  const uint32_t a_stack = sm100::opaque(sm100::smem_u32(stack + (size_t)grp * SC * CB));
 
   if (MULTI && tid < M) {
     s_per[tid][0] = mp.per[tid].nch;
@@ -681,9 +692,9 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
     for (int i = 0; i < T; ++i) {
       for (int j = 0; j < C::SCMAX; ++j) {
         sm100::mbar_init(&sfull[i][j], 1);
-        sm100::mbar_init(&srel[i][j], 4);
+        sm100::mbar_init(&srel[i][j], 4 * TPC);
       }
-      for (int j = 0; j < 4; ++j) sm100::mbar_init(&pub[i][j], 4);
+      for (int j = 0; j < 4; ++j) sm100::mbar_init(&pub[i][j], 4 * TPC);
       for (int j = 0; j < 4; ++j) sm100::mbar_init(&mdone[i][j], 1);
       for (int j = 0; j < C::NYS; ++j) sm100::mbar_init(&ybar[i][j], 1);
     }
@@ -698,7 +709,8 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
   __syncthreads();
   sm100::tc_fence_after();
   const uint32_t tbase = tmem_base_s;
-  const uint32_t tc = tbase + tile * C::TCOLS;  // this tile's TMEM columns (lane 0)
+  // this tile's TMEM columns (lane 0); a control warp: its group's first tile
+  const uint32_t tc = tbase + (control ? grp * TPC : tile) * C::TCOLS;
 
   if (control) {
     // ================================================================ control
@@ -708,7 +720,7 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
     // the stage SH halves ahead; group published -> issue its tcgen05.mma.
     // Waits sleep in hardware (try_wait with a suspend-time hint).
     sm100::setmaxnreg_dec<FzRegs<FzTiles<K, MULTI>::TM>::RP>();
-    if (tile >= T) {
+    if (grp * TPC >= T) {
       // spare warps of the control warpgroup
     } else {
       auto wait_sleep = [&](uint32_t bar, uint32_t par) {
@@ -792,7 +804,7 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
           }
         }
       };
-      ChunkCursor ldc{0u, nch, 0, 0, (int)blockIdx.x * T * 128 + 128 * tile, 0};
+      ChunkCursor ldc{0u, nch, 0, 0, (int)blockIdx.x * T * 128 + 128 * TPC * grp, 0};
       int ldst = 0;  // stage of the next chunk to load
       auto load_chunk = [&]() {
         if (ldc.u < U_total && lane == 0) {
@@ -866,9 +878,13 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
         sm100::tc_fence_after();
         const uint32_t b3 = tstage(cp);
 #pragma unroll
-        for (int j = 0; j < C::KY / 16; ++j)
-          sm100::umma_bf16_ts_e(tc + C::cY + 16 * slot, tc + C::cA3 + 8 * j,
-                                sm100::smem_desc(b3 + j * 2 * 256, 256, 128), idY, j > 0);
+        for (int u = 0; u < TPC; ++u) {
+          const uint32_t tcu = tc + u * C::TCOLS;
+#pragma unroll
+          for (int j = 0; j < C::KY / 16; ++j)
+            sm100::umma_bf16_ts_e(tcu + C::cY + 16 * slot, tcu + C::cA3 + 8 * j,
+                                  sm100::smem_desc(b3 + j * 2 * 256, 256, 128), idY, j > 0);
+        }
         sm100::umma_commit_e(a_ybar + 8 * slot);
       };
       // kind: 0 = A chunk c, 1 = beta0 (yhat of B0, B1), 2 = B chunk c, 3 =
@@ -886,16 +902,20 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
         if (kind == 0) {
           wait_table(cpos);
           sm100::tc_fence_after();
-          const uint32_t bf = tstage(cpos), bx = bf + 3 * C::BF_BYTES, at = tc + C::cOPA + 24 * abuf;
-          if (++abuf == C::NOPA) abuf = 0;
+          const uint32_t bf = tstage(cpos), bx = bf + 3 * C::BF_BYTES;
 #pragma unroll
-          for (int e = 0; e < 3; ++e)
-            sm100::umma_bf16_ts_e(tc + C::cG, at, sm100::smem_desc(bf + e * C::BF_BYTES, C::NGn * 16, 128), idG,
-                                  (c > 0 || e > 0) ? 1u : 0u);
-          // y' hi x_hi, y' hi x_mid, y' lo x_hi
-          sm100::umma_bf16_ts_e(tc + C::cB, at + 8, sm100::smem_desc(bx, C::KBn * 16, 128), idB, c > 0 ? 1u : 0u);
-          sm100::umma_bf16_ts_e(tc + C::cB, at + 8, sm100::smem_desc(bx + C::BX_BYTES, C::KBn * 16, 128), idB, 1u);
-          sm100::umma_bf16_ts_e(tc + C::cB, at + 16, sm100::smem_desc(bx, C::KBn * 16, 128), idB, 1u);
+          for (int u = 0; u < TPC; ++u) {
+            const uint32_t tcu = tc + u * C::TCOLS, at = tcu + C::cOPA + 24 * abuf;
+#pragma unroll
+            for (int e = 0; e < 3; ++e)
+              sm100::umma_bf16_ts_e(tcu + C::cG, at, sm100::smem_desc(bf + e * C::BF_BYTES, C::NGn * 16, 128), idG,
+                                    (c > 0 || e > 0) ? 1u : 0u);
+            // y' hi x_hi, y' hi x_mid, y' lo x_hi
+            sm100::umma_bf16_ts_e(tcu + C::cB, at + 8, sm100::smem_desc(bx, C::KBn * 16, 128), idB, c > 0 ? 1u : 0u);
+            sm100::umma_bf16_ts_e(tcu + C::cB, at + 8, sm100::smem_desc(bx + C::BX_BYTES, C::KBn * 16, 128), idB, 1u);
+            sm100::umma_bf16_ts_e(tcu + C::cB, at + 16, sm100::smem_desc(bx, C::KBn * 16, 128), idB, 1u);
+          }
+          if (++abuf == C::NOPA) abuf = 0;
         } else if (kind == 1 || kind == 3) {
           const int cnt = kind == 1 ? cur_nch : cur_ncm;
           for (int a = 0; a < C::NYS && a < cnt; ++a) issue_yhat(advance_pos(cpos, a), a);
@@ -906,15 +926,19 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
           // has just released
           wait_table(cpos);
           sm100::tc_fence_after();
-          const uint32_t bx = tstage(cpos) + C::B3_BYTES, at = tc + C::cOPB;
+          const uint32_t bx = tstage(cpos) + C::B3_BYTES;
           // r0 hi (x hi + mid + lo) + r0 mid (x hi + mid) + r0 lo x hi
 #pragma unroll
-          for (int e = 0; e < 3; ++e)
+          for (int u = 0; u < TPC; ++u) {
+            const uint32_t tcu = tc + u * C::TCOLS, at = tcu + C::cOPB;
 #pragma unroll
-            for (int xx = 0; xx < 3 - e; ++xx)
-              sm100::umma_bf16_ts_e(tc + C::cDB, at + 8 * e,
-                                    sm100::smem_desc(bx + xx * C::BX_BYTES, C::KBn * 16, 128), idB,
-                                    (c > 0 || e > 0 || xx > 0) ? 1u : 0u);
+            for (int e = 0; e < 3; ++e)
+#pragma unroll
+              for (int xx = 0; xx < 3 - e; ++xx)
+                sm100::umma_bf16_ts_e(tcu + C::cDB, at + 8 * e,
+                                      sm100::smem_desc(bx + xx * C::BX_BYTES, C::KBn * 16, 128), idB,
+                                      (c > 0 || e > 0 || xx > 0) ? 1u : 0u);
+          }
           sm100::umma_commit_e(a_mdone + 8 * (g & 3));
           if (c + C::NYS < cur_nch) issue_yhat(advance_pos(cpos, C::NYS), cslot);
         } else {
@@ -934,8 +958,9 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
             const ChunkPos nxt = advance_pos(cpos, C::ST - 2);
             if (lane == 0) {
               const uint32_t old = atom_add_acqrel(a_tfree + 4 * nxt.st, 1u);
-              const bool last = T == 4 ? (old & 3u) == 3u : T == 2 ? (old & 1u) == 1u : T == 1 ? true
-                                                                                           : old % 3u == 2u;
+              const int NGc = T / TPC;  // control groups sharing the table ring
+              const bool last = NGc == 4 ? (old & 3u) == 3u : NGc == 2 ? (old & 1u) == 1u : NGc == 1 ? true
+                                                                                                   : old % 3u == 2u;
               if (last) load_table(nxt);
             }
             __syncwarp();
@@ -991,7 +1016,7 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
     FZT_T0(t0)
     mbar_wait_spin(a_sfull + 8 * ust, uph);
     FZT_ADD(3, t0)
-    return a_stack + ust * CB + ESZ * (tid & 127);
+    return a_stack + ust * CB + ESZ * (128 * sub + (tid & 127));
   };
   auto release_chunk = [&]() {  // every value of the chunk has been consumed
     __syncwarp();
@@ -1006,9 +1031,9 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
 #pragma unroll
     for (int d = 0; d < 8; ++d) {
       if constexpr (I16)
-        yv[d] = fz_code(lds_u16(a + 256 * (8 * hf + d)));
+        yv[d] = fz_code(lds_u16(a + 256 * TPC * (8 * hf + d)));
       else
-        yv[d] = lds_f(a + 512 * (8 * hf + d));
+        yv[d] = lds_f(a + 512 * TPC * (8 * hf + d));
     }
   };
   const float fnd = tb.fnd;
@@ -1021,7 +1046,7 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
   auto patch_tail = [&](uint32_t a, int valid_rows) {
     if constexpr (I16) {
       if (valid_rows < C::DC) {
-        for (int d = valid_rows; d < C::DC; ++d) sts_u16(a + 256 * d, nd16);
+        for (int d = valid_rows; d < C::DC; ++d) sts_u16(a + 256 * TPC * d, nd16);
         sm100::fence_proxy_async_smem();
       }
     }
