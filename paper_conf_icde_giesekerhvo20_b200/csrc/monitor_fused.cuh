@@ -62,9 +62,9 @@ struct FzShape {
   // tiles per CTA: the register budget of 128 threads per tile (the
   // Cholesky factor of the K x K Gram lives in registers through pass B)
 #ifdef BFAST_FZ_TMAX8
-  static constexpr int TMAX = K <= 8 ? BFAST_FZ_TMAX8 : K == 10 ? 3 : 2;
+  static constexpr int TMAX = K <= 8 ? BFAST_FZ_TMAX8 : K <= 12 ? 3 : 2;
 #else
-  static constexpr int TMAX = K <= 8 ? 4 : K == 10 ? 3 : 2;
+  static constexpr int TMAX = K <= 8 ? 4 : K <= 12 ? 3 : 2;
 #endif
   // registers after setmaxnreg: consumers RC, the control warpgroup RP
   // (128 TMAX RC + 128 RP <= 65536)
@@ -135,7 +135,11 @@ struct FzCfg {
   static constexpr __host__ __device__ int pow2cols(int c) {
     return c <= 32 ? 32 : c <= 64 ? 64 : c <= 128 ? 128 : c <= 256 ? 256 : 512;
   }
-  static constexpr int TCOLS = pow2cols(USED > PB_COLS + 4 ? USED : PB_COLS + 4);  // >= 4 mask columns
+  // per-tile columns (>= 4 mask columns): a power of two, except K = 12,
+  // whose 136 columns round to 160 (32-aligned) so that three tiles fit the
+  // 512 TMEM columns (measured -20% at N = 250, k = 5 against two tiles)
+  static constexpr int TCOLS = K == 12 ? ((USED > PB_COLS + 4 ? USED : PB_COLS + 4) + 31) / 32 * 32
+                                       : pow2cols(USED > PB_COLS + 4 ? USED : PB_COLS + 4);
   // the validity bits of the last 2 MKC history chunks (two per column) live
   // in the columns pass B leaves free (the ring correction reads them back)
   static constexpr int cMK = PB_COLS, MKC = TCOLS - PB_COLS;
