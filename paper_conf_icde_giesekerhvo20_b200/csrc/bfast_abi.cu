@@ -91,6 +91,7 @@ struct bfast_plan {
   float *dX = nullptr;      // [N][KP] fp32
   double *dX64 = nullptr;   // [N][K] fp64
   int32_t *dcount = nullptr;
+  int *dprobe = nullptr;  // window probe result (max h over a sample)
   int64_t *dlist = nullptr;
   int64_t list_cap = 0;
   cudaEvent_t scratch_free = nullptr;  // orders executions sharing the refit scratch
@@ -128,6 +129,7 @@ struct bfast_plan {
     cudaFree(dX);
     cudaFree(dX64);
     cudaFree(dcount);
+    cudaFree(dprobe);
     cudaFree(dlist);
     cudaFree(dtabf);
     cudaFree(dshared);
@@ -451,13 +453,34 @@ int launch_fused(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStre
   int T = C::TMAX, sc = C::SCMAX;
   if (const char *e = std::getenv("BFAST_FZ_T")) T = std::max(1, std::min(C::TMAX, std::atoi(e)));
   if (const char *e = std::getenv("BFAST_FZ_SC")) sc = std::max(2, std::min(C::SCMAX, std::atoi(e)));
-  auto fits = [&](int t, int c) { return C::smem_bytes(t, pl.hcap, c, esz) + static_smem <= (size_t)kMaxSmem; };
+  int hcap = pl.hcap;  // MOSUM ring slots per pixel
+  auto fits = [&](int t, int c) { return C::smem_bytes(t, hcap, c, esz) + static_smem <= (size_t)kMaxSmem; };
+  // the ring sized for a complete history (h = floor(hf n)) costs tiles:
+  // size it from the widest window of a sample of the stack (+ a margin;
+  // wider windows go to the fp64 refit).  Synchronises the stream once.
+  const char *wpe = std::getenv("BFAST_WINDOW_PROBE");
+  if (!fits(T, 2) && prm.P >= 32 * 64 && pl.dprobe && !(wpe && wpe[0] == '0')) {
+    const int64_t groups = std::min<int64_t>(2048, prm.P / 32);
+    const int64_t gstride = prm.P / groups;
+    CUDA_TRY(cudaMemsetAsync(pl.dprobe, 0, sizeof(int), st));
+    if (I16)
+      bfast::window_probe_kernel<int16_t><<<(unsigned)groups, 32, 0, st>>>(
+          prm.Y16 + prm.p0, prm.ldY, prm.P, pl.n, pl.hf, gstride, prm.nodata, pl.dprobe);
+    else
+      bfast::window_probe_kernel<float><<<(unsigned)groups, 32, 0, st>>>(prm.Y + prm.p0, prm.ldY, prm.P, pl.n,
+                                                                         pl.hf, gstride, 0, pl.dprobe);
+    CUDA_TRY(cudaGetLastError());
+    int hmax = 0;
+    CUDA_TRY(cudaMemcpyAsync(&hmax, pl.dprobe, sizeof(int), cudaMemcpyDeviceToHost, st));
+    CUDA_TRY(cudaStreamSynchronize(st));
+    hcap = std::min(pl.hcap, std::max(std::min(pl.hcap, 8), hmax + std::max(8, hmax / 8)));
+  }
   while (T > 1 && !fits(T, 2)) --T;
   T = std::max(C::TPC, T / C::TPC * C::TPC);  // whole control groups
   if (!fits(T, sc)) sc = 2;
-  const size_t smem = C::smem_bytes(T, pl.hcap, sc, esz);
+  const size_t smem = C::smem_bytes(T, hcap, sc, esz);
   if (smem + static_smem > (size_t)kMaxSmem)
-    return fail(BFAST_EUNSUPPORTED, "fused kernel: shared memory %zu B for window %d", smem, pl.hcap);
+    return fail(BFAST_EUNSUPPORTED, "fused kernel: shared memory %zu B for window %d", smem, hcap);
   int sms = 148;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, pl.device);
   // CTAs per SM: shared memory (228 KB per SM, 1 KB reserved per CTA), TMEM
@@ -491,14 +514,15 @@ int launch_fused(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStre
   tb.nch = pl.nch;
   tb.ncm = pl.ncm;
   tb.T = T;
-  tb.hcap = pl.hcap;
+  tb.hcap = hcap;
   tb.pfd = pfd;
   tb.sc = sc;
   tb.ntg = (prm.P + 128 * T - 1) / (128 * T);
   const int64_t grid = std::min<int64_t>(tb.ntg, (int64_t)sms * per_sm);
   if (std::getenv("BFAST_VERBOSE"))
-    std::fprintf(stderr, "bfast: fused k=%d T=%d sc=%d smem=%zu+%d regs=%d per_sm=%d grid=%lld tile groups=%lld\n",
-                 pl.k, T, sc, smem, static_smem, fa.numRegs, per_sm, (long long)grid, (long long)tb.ntg);
+    std::fprintf(stderr, "bfast: fused k=%d T=%d sc=%d smem=%zu+%d regs=%d per_sm=%d grid=%lld tile groups=%lld "
+                 "ring=%d of %d\n", pl.k, T, sc, smem, static_smem, fa.numRegs, per_sm, (long long)grid,
+                 (long long)tb.ntg, hcap, pl.hcap);
   bfast::monitor_fused_kernel<K, I16, false><<<(unsigned)grid, threads, smem, st>>>(prm, tb, ymap, hmap, pmap,
                                                                                    no_multi());
   CUDA_TRY(cudaGetLastError());
@@ -946,6 +970,7 @@ int bfast_plan_create(bfast_plan **out, int device, int64_t N, const double *dat
   cudaError_t e = cudaMalloc(&pl->dX, X.size() * sizeof(float));
   if (e == cudaSuccess) e = cudaMalloc(&pl->dX64, X64.size() * sizeof(double));
   if (e == cudaSuccess) e = cudaMalloc(&pl->dcount, sizeof(int32_t));
+  if (e == cudaSuccess) e = cudaMalloc(&pl->dprobe, sizeof(int));
   if (e == cudaSuccess) e = cudaMemcpy(pl->dX, X.data(), X.size() * sizeof(float), cudaMemcpyHostToDevice);
   if (e == cudaSuccess)
     e = cudaMemcpy(pl->dX64, X64.data(), X64.size() * sizeof(double), cudaMemcpyHostToDevice);

@@ -1265,7 +1265,11 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
     // ================= pass B: residuals of the first fit, sigma-hat sums,
     // the refinement moment, validity bits, and the history's last
     // residuals into the MOSUM ring
-    const int hh = deg ? (hcap < 8 ? hcap : 8) : h;  // a degenerate pixel's ring is never read
+    // a window wider than the ring (capacity sized from a sample of the
+    // stack by the launcher) goes to the fp64 refit; the ring then holds
+    // what fits and the pixel's fp32 outputs are overwritten
+    if (!deg && h > hcap) refit = true;
+    const int hh = deg ? (hcap < 8 ? hcap : 8) : (h < hcap ? h : hcap);  // a degenerate pixel's ring is never read
     const uint32_t hbytes = (uint32_t)hh * 512, rend = rbase + hbytes;
     const int ring_from = deg ? 0x7fffffff : nbar - hh;  // first rank the ring must hold
     const bool ring8 = __all_sync(0xffffffffu, hh >= 8);

@@ -68,4 +68,30 @@ __global__ void __launch_bounds__(256) gather_dates_kernel(const float *__restri
   }
 }
 
+// The fused kernel's MOSUM ring holds h = floor(hf * nbar) residuals per
+// pixel; the plan sizes it for nbar = n (a complete history), which on a
+// cloudy scene wastes most of it and can cost a tile per CTA.  This probe
+// finds max h over a sample of 32-pixel groups spread over the stack (one
+// warp per group, coalesced rows); the launcher sizes the ring from it (plus
+// a margin) and the kernel hands any pixel whose window does not fit to the
+// fp64 refit.  E = float (NaN missing) or int16_t (code == nodata missing).
+template <typename E>
+__global__ void __launch_bounds__(32) window_probe_kernel(const E *__restrict__ Y, int64_t ldY, int64_t P, int n,
+                                                          float hf, int64_t gstride, int32_t nodata, int *hmax) {
+  const int64_t p = (int64_t)blockIdx.x * gstride + threadIdx.x;
+  int cnt = 0;
+  if (p < P)
+    for (int t = 0; t < n; ++t) {
+      const E v = Y[(int64_t)t * ldY + p];
+      if constexpr (sizeof(E) == 2)
+        cnt += (int)v != nodata;
+      else
+        cnt += v == v;
+    }
+  int h = (int)__fmul_rn(__int2float_rn(cnt), hf);  // Fig. 12 L516 in f32 (R3)
+#pragma unroll
+  for (int o = 16; o; o >>= 1) h = max(h, __shfl_xor_sync(0xffffffffu, h, o));
+  if (threadIdx.x == 0) atomicMax(hmax, h);
+}
+
 }  // namespace bfast

@@ -174,3 +174,26 @@ def test_two_process_ipc_gather(tmp_path):
     torch.cuda.synchronize()
     np.testing.assert_array_equal(got["brk"], ref["break"].cpu().numpy())
     np.testing.assert_array_equal(np.nan_to_num(got["mag"]), np.nan_to_num(ref["magnitude"].cpu().numpy()))
+
+
+def test_ring_sized_from_a_sample_refits_wider_windows():
+    """Sentinel-2 shape (N = 700, n = 350: a complete history's window, 87,
+    would cost a tile per CTA): the launcher sizes the MOSUM ring from a
+    sample of the stack, and pixels whose window is wider -- here complete
+    histories placed outside the sampled 32-pixel groups -- go to the fp64
+    refit: every one of them and a sample of the rest match the oracle."""
+    P = 1 << 20
+    spec = synth.StackSpec(P=P, N=700, n_hist=350, miss=0.5, mask="iid", f=73.0, year0=2016.0, seed=421)
+    Y, dates = synth.generate(spec, DEV)
+    Y0, _ = synth.generate(synth.StackSpec(**{**spec.asdict(), "mask": "none"}), DEV)
+    wide = np.arange(200, P, 512)  # the probe samples the first 32 pixels of every 512
+    it = torch.from_numpy(wide).to(DEV)
+    Y[:350, it] = Y0[:350, it]
+    out = binding.bfast_monitor_ex(Y, dates, spec.n_hist, spec.k, spec.hf, spec.lam, diagnostics=True)
+    torch.cuda.synchronize()
+    flags = out["flags"].cpu().numpy()
+    assert np.all(flags[wide] & 2), "complete histories must be refitted in fp64"
+    rng = np.random.default_rng(3)
+    idx = np.sort(np.concatenate([wide, rng.choice(P, 20000, replace=False)]))
+    idx = np.unique(idx)
+    _parity(out, Y, idx, dates, spec.n_hist, spec.k, spec.hf, spec.lam)
