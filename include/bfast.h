@@ -132,7 +132,15 @@ int bfast_monitor(const float *Y, int64_t N, int64_t P, const double *dates,
                   int32_t *out_break, float *out_magnitude);
 
 /* Extended form: leading dimension, optional outputs, stream.  Asynchronous
-   with respect to the host: returns after enqueueing on a->stream. */
+   with respect to the host: returns after enqueueing on a->stream -- except
+   when a complete history's MOSUM window (floor(h * n_hist) slots per pixel)
+   would cost the fused kernel a tile per CTA (long histories, e.g. N = 700):
+   the call then samples the stack on a->stream (window_probe_kernel, 2048
+   groups of 32 pixels), synchronises the stream once to size the window ring
+   from the widest sampled window, and pixels whose window is wider are
+   recomputed by the fp64 refit (results unchanged; BFAST_WINDOW_PROBE=0
+   keeps the full ring and the asynchrony).  The same holds for
+   bfast_plan_execute and the entries built on them. */
 int bfast_monitor_ex(const bfast_args *a);
 
 /*

@@ -15,3 +15,4 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:monitor_fused -s 3 -c 1 \
   -o gpurun_out/${TAG}_full python bench.py --steps 1 --warmup 3 --no-e2e --no-cpu-baseline \
   > gpurun_out/${TAG}_ncu.log 2>&1; echo full=$?
+timeout 1500 python tools/sweep_table.py gpurun_out/${TAG}_sweep.json > gpurun_out/${TAG}_sweep.log 2>&1; echo sweep=$?
