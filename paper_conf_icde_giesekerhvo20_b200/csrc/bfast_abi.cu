@@ -421,14 +421,14 @@ const bfast::FzMulti &no_multi() {
   return m;
 }
 
-template <int K, bool I16, bool MULTI>
+template <int K, bool I16, bool MULTI, bool CLAMP = false>
 int fused_config(int device, cudaFuncAttributes &fa) {
   static thread_local int configured_dev = -1;
-  CUDA_TRY(cudaFuncGetAttributes(&fa, bfast::monitor_fused_kernel<K, I16, MULTI>));
+  CUDA_TRY(cudaFuncGetAttributes(&fa, bfast::monitor_fused_kernel<K, I16, MULTI, CLAMP>));
   if (configured_dev != device) {
-    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_fused_kernel<K, I16, MULTI>,
+    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_fused_kernel<K, I16, MULTI, CLAMP>,
                                   cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmem - (int)fa.sharedSizeBytes));
-    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_fused_kernel<K, I16, MULTI>,
+    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_fused_kernel<K, I16, MULTI, CLAMP>,
                                   cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared));
     configured_dev = device;
   }
@@ -523,8 +523,16 @@ int launch_fused(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStre
     std::fprintf(stderr, "bfast: fused k=%d T=%d sc=%d smem=%zu+%d regs=%d per_sm=%d grid=%lld tile groups=%lld "
                  "ring=%d of %d\n", pl.k, T, sc, smem, static_smem, fa.numRegs, per_sm, (long long)grid,
                  (long long)tb.ntg, hcap, pl.hcap);
-  bfast::monitor_fused_kernel<K, I16, false><<<(unsigned)grid, threads, smem, st>>>(prm, tb, ymap, hmap, pmap,
-                                                                                   no_multi());
+  if (hcap < pl.hcap) {  // the sampled ring: the instantiation that clamps windows
+    cudaFuncAttributes fc{};
+    const int rc = fused_config<K, I16, false, true>(pl.device, fc);
+    if (rc) return rc;
+    bfast::monitor_fused_kernel<K, I16, false, true><<<(unsigned)grid, threads, smem, st>>>(prm, tb, ymap, hmap,
+                                                                                          pmap, no_multi());
+  } else {
+    bfast::monitor_fused_kernel<K, I16, false><<<(unsigned)grid, threads, smem, st>>>(prm, tb, ymap, hmap, pmap,
+                                                                                     no_multi());
+  }
   CUDA_TRY(cudaGetLastError());
   done = true;
   return BFAST_OK;

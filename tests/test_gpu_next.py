@@ -274,3 +274,21 @@ def test_f4_int16_wide_designs(k):
     gpu = {key: v.cpu().numpy() for key, v in out.items() if torch.is_tensor(v)}
     rep = parity.compare(gpu, orc, dates, 150, k)
     assert rep["ok"], json.dumps(rep)
+
+
+def test_f4_int16_long_history_sampled_ring():
+    """int16 codes at the Sentinel-2 shape (N = 700, n = 350): the window
+    probe reads codes (nodata = missing) to size the ring; parity on a
+    sample."""
+    spec = synth.StackSpec(P=300_000, N=700, n_hist=350, miss=0.5, mask="iid", f=73.0, year0=2016.0, seed=1811)
+    Y, dates = synth.generate(spec, DEV)
+    codes = synth.quantize_i16(Y, 1e-4, 0.0, -32768)
+    out = binding.bfast_monitor_i16(codes, dates, 350, 3, spec.hf, spec.lam, 1e-4, 0.0, -32768, diagnostics=True)
+    torch.cuda.synchronize()
+    idx = np.sort(np.random.default_rng(4).choice(spec.P, 20_000, replace=False))
+    Yd = oracle.decode_i16(codes[:, torch.from_numpy(idx).to(DEV)].cpu().numpy(), np.float32(1e-4),
+                           np.float32(0.0), -32768)
+    orc = oracle.monitor(np.ascontiguousarray(Yd), dates, 350, 3, spec.hf, spec.lam)
+    gpu = {key: v.cpu().numpy()[idx] for key, v in out.items() if torch.is_tensor(v)}
+    rep = parity.compare(gpu, orc, dates, 350, 3)
+    assert rep["ok"], json.dumps(rep)
