@@ -140,7 +140,12 @@ int bfast_monitor(const float *Y, int64_t N, int64_t P, const double *dates,
    from the widest sampled window, and pixels whose window is wider are
    recomputed by the fp64 refit (results unchanged; BFAST_WINDOW_PROBE=0
    keeps the full ring and the asynchrony).  The same holds for
-   bfast_plan_execute and the entries built on them. */
+   bfast_plan_execute and the entries built on them.
+   BFAST_SHARED_FACTOR=1: warps whose 32
+   pixels have no missing history value use the plan's Gram factor,
+   computed once in fp64, instead of factoring their own (a separate
+   kernel instantiation, off by default: its per-warp test costs scenes
+   with gaps; results identical up to fp32 rounding). */
 int bfast_monitor_ex(const bfast_args *a);
 
 /*

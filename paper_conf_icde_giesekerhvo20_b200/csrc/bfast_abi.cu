@@ -421,14 +421,14 @@ const bfast::FzMulti &no_multi() {
   return m;
 }
 
-template <int K, bool I16, bool MULTI, bool CLAMP = false>
+template <int K, bool I16, bool MULTI, bool CLAMP = false, bool DENSE = false>
 int fused_config(int device, cudaFuncAttributes &fa) {
   static thread_local int configured_dev = -1;
-  CUDA_TRY(cudaFuncGetAttributes(&fa, bfast::monitor_fused_kernel<K, I16, MULTI, CLAMP>));
+  CUDA_TRY(cudaFuncGetAttributes(&fa, bfast::monitor_fused_kernel<K, I16, MULTI, CLAMP, DENSE>));
   if (configured_dev != device) {
-    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_fused_kernel<K, I16, MULTI, CLAMP>,
+    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_fused_kernel<K, I16, MULTI, CLAMP, DENSE>,
                                   cudaFuncAttributeMaxDynamicSharedMemorySize, kMaxSmem - (int)fa.sharedSizeBytes));
-    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_fused_kernel<K, I16, MULTI, CLAMP>,
+    CUDA_TRY(cudaFuncSetAttribute(bfast::monitor_fused_kernel<K, I16, MULTI, CLAMP, DENSE>,
                                   cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared));
     configured_dev = device;
   }
@@ -508,9 +508,12 @@ int launch_fused(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStre
     const uint32_t u = (((uint32_t)(uint16_t)prm.nodata) ^ 0x8000u) | 0x4B000000u;
     std::memcpy(&tb.fnd, &u, 4);
   }
-  // BFAST_SHARED_FACTOR=0: every pixel factors its own Gram (A/B of f3)
+  // f3: BFAST_SHARED_FACTOR=1 launches the instantiation in which warps of
+  // complete histories use the plan's fp64 factor (off by default: its warp
+  // test costs the cloudy scenes)
   const char *sfe = std::getenv("BFAST_SHARED_FACTOR");
-  tb.shared = (sfe && sfe[0] == '0') ? nullptr : pl.dshared;
+  const bool dense = !I16 && sfe && sfe[0] == '1' && pl.dshared;
+  tb.shared = dense ? pl.dshared : nullptr;
   tb.nch = pl.nch;
   tb.ncm = pl.ncm;
   tb.T = T;
@@ -523,7 +526,13 @@ int launch_fused(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStre
     std::fprintf(stderr, "bfast: fused k=%d T=%d sc=%d smem=%zu+%d regs=%d per_sm=%d grid=%lld tile groups=%lld "
                  "ring=%d of %d\n", pl.k, T, sc, smem, static_smem, fa.numRegs, per_sm, (long long)grid,
                  (long long)tb.ntg, hcap, pl.hcap);
-  if (hcap < pl.hcap) {  // the sampled ring: the instantiation that clamps windows
+  if (dense && hcap == pl.hcap) {
+    cudaFuncAttributes fd{};
+    const int rc = fused_config<K, false, false, false, true>(pl.device, fd);
+    if (rc) return rc;
+    bfast::monitor_fused_kernel<K, false, false, false, true><<<(unsigned)grid, threads, smem, st>>>(
+        prm, tb, ymap, hmap, pmap, no_multi());
+  } else if (hcap < pl.hcap) {  // the sampled ring: the instantiation that clamps windows
     cudaFuncAttributes fc{};
     const int rc = fused_config<K, I16, false, true>(pl.device, fc);
     if (rc) return rc;
@@ -666,7 +675,6 @@ int launch_multi_k(const std::vector<bfast_plan *> &pls, const std::vector<bfast
   std::memset(mp.get(), 0, sizeof(bfast::FzMulti));
   mp->M = M;
   mp->Lg = 0;
-  const char *sfe = std::getenv("BFAST_SHARED_FACTOR");
   for (int i = 0; i < M; ++i) {
     const bfast_plan &pl = *pls[i];
     bfast::FzPeriod &fp = mp->per[i];
@@ -674,7 +682,7 @@ int launch_multi_k(const std::vector<bfast_plan *> &pls, const std::vector<bfast
     fp.tabA = pl.dtabf;
     fp.tabB = pl.dtabf + pl.tabfB_off;
     fp.tabC = pl.dtabf + pl.tabfC_off;
-    fp.shared = (sfe && sfe[0] == '0') ? nullptr : pl.dshared;
+    fp.shared = nullptr;  // f3 is not part of the multi-period kernel
     fp.nch = pl.nch;
     fp.ncm = pl.ncm;
     mp->Lg += 2 * pl.nch + pl.ncm;

@@ -615,7 +615,7 @@ __device__ __forceinline__ void fz_solve(const float (&L)[Tri<K>::kN], const flo
   });
 }
 
-template <int K, bool I16, bool MULTI, bool CLAMP = false>
+template <int K, bool I16, bool MULTI, bool CLAMP = false, bool DENSE = false>
 __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
     monitor_fused_kernel(MonitorParams pk, FzTables tb, const __grid_constant__ CUtensorMap ymap,
                          const __grid_constant__ CUtensorMap hmap, const __grid_constant__ CUtensorMap pmap,
@@ -1200,24 +1200,33 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
       float diagA[K];
 #pragma unroll
       for (int i = 0; i < K; ++i) diagA[i] = A[Tri<K>::idx(i, i)];
-      // f3 (L93): a warp whose 32 histories have no missing value shares
-      // one Gram, factored once on the host in fp64: beta0 = A^-1 (X_hist^T
-      // y'), the moment b being the tensor-core GEMM of pass A
-      const bool dense = shared_factor != nullptr && __all_sync(0xffffffffu, nbar == n);
-      float minratio, vif = 0.f;
-      if (dense) {
+      if constexpr (DENSE) {
+        // f3 (L93): a warp whose 32 histories have no missing value shares
+        // one Gram, factored once on the host in fp64: beta0 = A^-1 (X_hist^T
+        // y'), the moment b being the tensor-core GEMM of pass A.  A separate
+        // instantiation (BFAST_SHARED_FACTOR=1): the warp test in the common
+        // kernel cost +0.3% on the Landsat scene and +5% at N = 100
+        const bool dense = shared_factor != nullptr && __all_sync(0xffffffffu, nbar == n);
+        float minratio, vif = 0.f;
+        if (dense) {
 #pragma unroll
-        for (int i = 0; i < Tri<K>::kN; ++i) A[i] = __ldg(shared_factor + i);
+          for (int i = 0; i < Tri<K>::kN; ++i) A[i] = __ldg(shared_factor + i);
 #pragma unroll
-        for (int i = 0; i < K; ++i) dinv[i] = __ldg(shared_factor + Tri<K>::kN + i);
-        minratio = __ldg(shared_factor + Tri<K>::kN + K);
-        vif = __ldg(shared_factor + Tri<K>::kN + K + 1);
+          for (int i = 0; i < K; ++i) dinv[i] = __ldg(shared_factor + Tri<K>::kN + i);
+          minratio = __ldg(shared_factor + Tri<K>::kN + K);
+          vif = __ldg(shared_factor + Tri<K>::kN + K + 1);
+        } else {
+          minratio = fz_chol<K>(A, dinv);
+        }
+        fz_solve<K>(A, dinv, b, beta);
+        if (!deg && !(minratio >= (float)kRefitRatio)) refit = true;
+        if (!deg && !refit && !((dense ? vif : fz_vif_max<K>(A, dinv, diagA)) <= kRefitVif)) refit = true;
       } else {
-        minratio = fz_chol<K>(A, dinv);
+        const float minratio = fz_chol<K>(A, dinv);
+        fz_solve<K>(A, dinv, b, beta);
+        if (!deg && !(minratio >= (float)kRefitRatio)) refit = true;
+        if (!deg && !refit && !(fz_vif_max<K>(A, dinv, diagA) <= kRefitVif)) refit = true;
       }
-      fz_solve<K>(A, dinv, b, beta);
-      if (!deg && !(minratio >= (float)kRefitRatio)) refit = true;
-      if (!deg && !refit && !((dense ? vif : fz_vif_max<K>(A, dinv, diagA)) <= kRefitVif)) refit = true;
       if (deg || !have) {
 #pragma unroll
         for (int i = 0; i < K; ++i) beta[i] = 0.f;
