@@ -1,4 +1,9 @@
-# bench one config in several repo snapshots (ab/<dir>), interleaved: tools/ab_bisect.sh CFG dir1 dir2 ...
+#!/bin/bash
+# Bench one config in several repository snapshots, interleaved (GPU box):
+#   tools/ab_bisect.sh CFG dir1 dir2 ...     ("." = this tree)
+# A snapshot dir holds bench.py, oracle/, include/, MEASURED_PEAKS.json and the
+# package with its built libbfast.so (e.g. from a git worktree of an older
+# commit, copied under ab/, which gpurun ships and git ignores).
 CFG=$1; shift
 for r in 1 2; do
   for D in "$@"; do
