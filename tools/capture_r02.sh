@@ -7,6 +7,7 @@ timeout 900 python bench.py > gpurun_out/${TAG}_bench.json 2> gpurun_out/${TAG}_
 for c in dense africa int16 periods; do
   timeout 600 python bench.py --config $c --steps 10 > gpurun_out/${TAG}_$c.json 2> gpurun_out/${TAG}_$c.err; echo $c=$?
 done
+timeout 900 python bench.py --config stream --steps 8 --warmup 2 --no-cpu-baseline > gpurun_out/${TAG}_stream.json 2> gpurun_out/${TAG}_stream.err; echo stream=$?
 timeout 600 python tools/periods_exp.py > gpurun_out/${TAG}_periods_exp.log 2>&1; echo pexp=$?
 timeout 900 python bench.py --config sentinel2 --steps 3 --warmup 3 > gpurun_out/${TAG}_s2.json 2> gpurun_out/${TAG}_s2.err; echo s2=$?
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"monitor|refit" -c 20 --csv \
