@@ -699,7 +699,9 @@ def main():
                 "alg_bytes_per_launch": alg_bytes, "peak_source": peak_src}
 
     if args.config == "periods":
-        # the same periods as separate single-period launches (each reads its stack slice from HBM)
+        # the same periods as separate single-period launches (each reads its stack slice from HBM;
+        # each sizes its own MOSUM ring, so a pixel near a ring's capacity may take the fp64 refit in
+        # one schedule and not the other: equal up to the parity tolerances, usually to the bit)
         plans = [binding.Plan(local, e, dates[:e], b, rspec.k, rspec.hf, rspec.lam) for b, e in PERIODS]
         outs = [{"break": torch.empty(P, dtype=torch.int32, device=dev),
                  "magnitude": torch.empty(P, dtype=torch.float32, device=dev)} for _ in PERIODS]

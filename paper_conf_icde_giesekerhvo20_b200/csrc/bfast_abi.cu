@@ -652,12 +652,30 @@ int launch_multi_k(const std::vector<bfast_plan *> &pls, const std::vector<bfast
     if (rc) return rc;
   }
   const int static_smem = (int)fa.sharedSizeBytes;
-  int hcap = 1;
-  for (auto *pl : pls) hcap = std::max(hcap, pl->hcap);
+  int hcap = 1, hfull = 1;
+  const bfast_plan *plong = pls[0];  // the period with the longest history
+  for (auto *pl : pls) {
+    hfull = std::max(hfull, pl->hcap);
+    if (pl->n > plong->n) plong = pl;
+  }
+  hcap = hfull;
   int T = bfast::FzTiles<K, true>::TM, sc = C::SCMAX;
   if (const char *e = std::getenv("BFAST_FZ_T")) T = std::max(1, std::min(T, std::atoi(e)));
   if (const char *e = std::getenv("BFAST_FZ_SC")) sc = std::max(2, std::min(C::SCMAX, std::atoi(e)));
   auto fits = [&](int t, int c) { return C::smem_bytes(t, hcap, c) + static_smem <= (size_t)kMaxSmem; };
+  // the ring from a sample of the longest history's windows (as launch_fused)
+  const char *wpe = std::getenv("BFAST_WINDOW_PROBE");
+  if (!fits(T, 2) && q0.P >= 32 * 64 && plong->dprobe && !(wpe && wpe[0] == '0')) {
+    const int64_t groups = std::min<int64_t>(2048, q0.P / 32);
+    CUDA_TRY(cudaMemsetAsync(plong->dprobe, 0, sizeof(int), st));
+    bfast::window_probe_kernel<float><<<(unsigned)groups, 32, 0, st>>>(q0.Y + q0.p0, q0.ldY, q0.P, plong->n,
+                                                                       plong->hf, q0.P / groups, 0, plong->dprobe);
+    CUDA_TRY(cudaGetLastError());
+    int hmax = 0;
+    CUDA_TRY(cudaMemcpyAsync(&hmax, plong->dprobe, sizeof(int), cudaMemcpyDeviceToHost, st));
+    CUDA_TRY(cudaStreamSynchronize(st));
+    hcap = std::min(hfull, std::max(std::min(hfull, 8), hmax + std::max(8, hmax / 8)));
+  }
   while (T > 1 && !fits(T, 2)) --T;
   T = std::max(C::TPC, T / C::TPC * C::TPC);  // whole control groups
   if (!fits(T, sc)) sc = 2;
@@ -705,7 +723,9 @@ int launch_multi_k(const std::vector<bfast_plan *> &pls, const std::vector<bfast
   tb.ncm = p0.ncm;
   tb.T = T;
   tb.hcap = hcap;
-  tb.pfd = 128;
+  // no L2 prefetch in the multi-period kernel: most of its reads are L2
+  // re-reads of earlier periods (measured -3% on 4 and 7 yearly periods)
+  tb.pfd = 0;
   if (const char *e = std::getenv("BFAST_FZ_PFD")) tb.pfd = std::max(0, std::atoi(e)) / C::PFB * C::PFB;
   tb.sc = sc;
   tb.ntg = (q0.P + 128 * T - 1) / (128 * T);
@@ -719,8 +739,16 @@ int launch_multi_k(const std::vector<bfast_plan *> &pls, const std::vector<bfast
     CUDA_TRY(cudaEventCreate(&e1));
     CUDA_TRY(cudaEventRecord(e0, st));
   }
-  bfast::monitor_fused_kernel<K, false, true><<<(unsigned)grid, threads, smem, st>>>(q0, tb, mp->per[0].y,
-                                                                                    mp->per[0].h, pmap, *mp);
+  if (hcap < hfull) {  // the sampled ring: windows wider than it go to the refit
+    cudaFuncAttributes fc{};
+    const int rc = fused_config<K, false, true, true>(p0.device, fc);
+    if (rc) return rc;
+    bfast::monitor_fused_kernel<K, false, true, true><<<(unsigned)grid, threads, smem, st>>>(
+        q0, tb, mp->per[0].y, mp->per[0].h, pmap, *mp);
+  } else {
+    bfast::monitor_fused_kernel<K, false, true><<<(unsigned)grid, threads, smem, st>>>(q0, tb, mp->per[0].y,
+                                                                                      mp->per[0].h, pmap, *mp);
+  }
   CUDA_TRY(cudaGetLastError());
   if (g_prof_on) {
     CUDA_TRY(cudaEventRecord(e1, st));

@@ -191,9 +191,11 @@ def _yearly(n0, M, year=23):
     (228, [(114, 228), (100, 180), (60, 77), (150, 201)], 1, "iid"),  # unordered, partial chunks
     (320, _yearly(120, 8), 5, "iid"),                               # the maximum of 8 periods
 ])
-def test_f1_several_periods_in_one_launch(N, periods, k, mask):
-    """Every period against the oracle on its own date slice, and bit-equal
-    to a separate single-period run of the same kernel code."""
+def test_f1_several_periods_in_one_launch(N, periods, k, mask, monkeypatch):
+    """Every period against the oracle on its own date slice (the MOSUM ring
+    sized from a sample: wider windows refitted in fp64), and -- both with
+    the full ring (BFAST_WINDOW_PROBE=0), so that the same pixels take the
+    same path -- bit-equal to a separate single-period run."""
     spec = synth.StackSpec(P=20_000 + 11, N=N, n_hist=periods[0][0], k=k, miss=0.5, mask=mask, seed=1500 + N + k)
     Yp, dates = synth.generate(spec, DEV, ldY=20_016)  # TMA rows: ldY % 4 == 0; a ragged last tile
     Y = Yp[:, :spec.P]
@@ -207,11 +209,13 @@ def test_f1_several_periods_in_one_launch(N, periods, k, mask):
         rep = parity.compare(gpu, orc, dates[:N_i], n_i, k)
         assert rep["ok"], (i, json.dumps(rep))
         np.testing.assert_array_equal(gpu["nbar"], orc["nbar"])
-        single = binding.bfast_monitor_ex(Y[:N_i], dates[:N_i], n_i, k, spec.hf, spec.lam, diagnostics=True)
+    monkeypatch.setenv("BFAST_WINDOW_PROBE", "0")
+    full = binding.bfast_monitor_periods(Y, dates, periods, k, spec.hf, spec.lam)
+    for i, (n_i, N_i) in enumerate(periods):
+        single = binding.bfast_monitor_ex(Y[:N_i], dates[:N_i], n_i, k, spec.hf, spec.lam)
         torch.cuda.synchronize()
-        np.testing.assert_array_equal(single["break"].cpu().numpy(), gpu["break"])
-        np.testing.assert_array_equal(single["magnitude"].cpu().numpy().view(np.uint32),
-                                      gpu["magnitude"].view(np.uint32))
+        assert torch.equal(single["break"], full["break"][i])
+        assert torch.equal(single["magnitude"].view(torch.int32), full["magnitude"][i].view(torch.int32))
 
 
 def test_f1_split_schedule_is_bit_identical(monkeypatch):

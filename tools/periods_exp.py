@@ -26,7 +26,7 @@ sets = {"same_n": [(200, 300 + 10 * i) for i in range(4)],
 for name, per in sets.items():
     sep = timed(lambda: [binding.bfast_monitor_ex(Y[:e], dates[:e], b, 3, spec.hf, spec.lam) for b, e in per])
     res = {"set": name, "separate_ms": round(sep, 2)}
-    for env in ("", "BFAST_FZ_PFD=0", "BFAST_FZ_T=2"):
+    for env in ("", "BFAST_FZ_PFD=128", "BFAST_FZ_T=2"):
         for kv in [env] if env else []:
             k, v = kv.split("=")
             os.environ[k] = v
