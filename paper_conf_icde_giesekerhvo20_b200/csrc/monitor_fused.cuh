@@ -3,10 +3,12 @@
 // tile of 128 pixels shares on the 5th-generation tensor cores, one control
 // warp per tile that only moves data (TMA) and issues tcgen05.mma.
 //
-// Variants (template parameters): I16 -- the stack as scaled int16 codes
-// (SURVEY 8(f) f4); MULTI -- several monitoring periods per stack pass
-// (f1, FzMulti).  NaN-free histories share one host-factored Gram (f3,
-// FzTables::shared).
+// Variants (template parameters, each its own instantiation so that the
+// common kernel carries none of their code): I16 -- the stack as scaled
+// int16 codes; MULTI -- several monitoring periods per
+// stack pass (f1, FzMulti); CLAMP -- the MOSUM ring sized from a sample of
+// the stack, wider windows to the fp64 refit; DENSE -- warps of complete
+// histories use the plan's fp64 Gram factor (f3, FzTables::shared).
 //
 // Algorithm 1, Fig. 12 (L478-L537); readings R1-R14 of
 // DESIGN.md.  Per tile of 128 pixels (one pixel per thread = one TMEM lane),
