@@ -294,14 +294,15 @@ int bfast_valid_dates(const float *Y, int64_t N, int64_t P, int64_t ldY, int32_t
 
 /*
  * bfast_gather_dates -- Yc[i][p] = Y[idx[i]][p] for i < Nc, p < P: the
- * kept slices (idx: device int32[Nc], values in [0, N), normally
- * increasing) as a compact DEVICE stack Yc float32 [Nc][ldYc].  Y and Yc
- * must not overlap.  Asynchronous on `stream`.  Errors: BFAST_EINVAL (P <
- * 0, Nc < 0, ldY < P, ldYc < P, NULL pointer); BFAST_EUNSUPPORTED (Nc >
- * 65535).
+ * kept slices (idx: device int32[Nc], normally increasing) of the DEVICE
+ * stack Y float32 [N][ldY] as a compact DEVICE stack Yc float32 [Nc][ldYc].
+ * A row whose idx[i] is outside [0, N) is filled with NaN (the kernel never
+ * reads outside the stack).  Y and Yc must not overlap.  Asynchronous on
+ * `stream`.  Errors: BFAST_EINVAL (N < 0, P < 0, Nc < 0, ldY < P, ldYc < P,
+ * NULL pointer); BFAST_EUNSUPPORTED (Nc > 65535).
  */
-int bfast_gather_dates(const float *Y, int64_t ldY, int64_t P, const int32_t *idx, int64_t Nc, float *Yc,
-                       int64_t ldYc, void *stream);
+int bfast_gather_dates(const float *Y, int64_t N, int64_t ldY, int64_t P, const int32_t *idx, int64_t Nc,
+                       float *Yc, int64_t ldYc, void *stream);
 
 /*
  * bfast_monitor_host_resume -- a scene streamed tile by tile with

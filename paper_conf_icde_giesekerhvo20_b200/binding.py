@@ -101,7 +101,7 @@ def lib():
         L.bfast_monitor_i16.restype = I
         L.bfast_valid_dates.argtypes = [V, i64, i64, i64, V, V]
         L.bfast_valid_dates.restype = I
-        L.bfast_gather_dates.argtypes = [V, i64, i64, V, i64, V, i64, V]
+        L.bfast_gather_dates.argtypes = [V, i64, i64, i64, V, i64, V, i64, V]
         L.bfast_gather_dates.restype = I
         L.bfast_monitor_host_resume.argtypes = [V, i64, i64, i64, V, i32, i32, f32, f32, V, V, I, i64, i64,
                                                 ctypes.POINTER(i64)]
@@ -403,7 +403,7 @@ def bfast_gather_dates(Y, idx, P=None, stream=None):
     assert idx.dtype == torch.int32 and idx.device == Y.device
     Yc = torch.empty((int(idx.numel()), P), dtype=torch.float32, device=Y.device)
     with torch.cuda.device(Y.device):
-        _check(lib().bfast_gather_dates(_dptr(Y), ldY, P, _dptr(idx), int(idx.numel()), _dptr(Yc), P,
+        _check(lib().bfast_gather_dates(_dptr(Y), int(Y.shape[0]), ldY, P, _dptr(idx), int(idx.numel()), _dptr(Yc), P,
                                         _stream_ptr(stream)))
     return Yc
 

@@ -1384,9 +1384,10 @@ int bfast_valid_dates(const float *Y, int64_t N, int64_t P, int64_t ldY, int32_t
   return BFAST_OK;
 }
 
-int bfast_gather_dates(const float *Y, int64_t ldY, int64_t P, const int32_t *idx, int64_t Nc, float *Yc,
-                       int64_t ldYc, void *stream) {
-  if (P < 0 || Nc < 0 || ldY < P || ldYc < P) return fail(BFAST_EINVAL, "P < 0, Nc < 0, ldY < P or ldYc < P");
+int bfast_gather_dates(const float *Y, int64_t N, int64_t ldY, int64_t P, const int32_t *idx, int64_t Nc,
+                       float *Yc, int64_t ldYc, void *stream) {
+  if (N < 0 || P < 0 || Nc < 0 || ldY < P || ldYc < P)
+    return fail(BFAST_EINVAL, "N < 0, P < 0, Nc < 0, ldY < P or ldYc < P");
   g_launches = 0;
   if (P == 0 || Nc == 0) return BFAST_OK;
   if (!Y || !idx || !Yc) return fail(BFAST_EINVAL, "NULL pointer");
@@ -1399,7 +1400,7 @@ int bfast_gather_dates(const float *Y, int64_t ldY, int64_t P, const int32_t *id
   const int64_t per_row = std::max<int64_t>(1, std::min<int64_t>((P / (vec4 ? 4 : 1) + 255) / 256,
                                                                std::max<int64_t>(1, 8 * sms / Nc)));
   bfast::gather_dates_kernel<<<dim3((unsigned)per_row, (unsigned)Nc), 256, 0, (cudaStream_t)stream>>>(
-      Y, ldY, P, idx, Yc, ldYc, vec4);
+      Y, N, ldY, P, idx, Yc, ldYc, vec4);
   CUDA_TRY(cudaGetLastError());
   g_launches = 1;
   return BFAST_OK;

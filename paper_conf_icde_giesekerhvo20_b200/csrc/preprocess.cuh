@@ -48,14 +48,21 @@ __global__ void __launch_bounds__(kScanThreads) slice_any_kernel(const float *__
   if (__syncthreads_or(any) && threadIdx.x == 0) keep[t] = 1;
 }
 
-// grid (column blocks, Nc rows): row i of Yc = row idx[i] of Y, columns [0, P)
-__global__ void __launch_bounds__(256) gather_dates_kernel(const float *__restrict__ Y, int64_t ldY, int64_t P,
-                                                           const int32_t *__restrict__ idx, float *__restrict__ Yc,
-                                                           int64_t ldYc, int vec4) {
+// grid (column blocks, Nc rows): row i of Yc = row idx[i] of Y, columns [0,
+// P); an index outside [0, N) gives a row of NaN
+__global__ void __launch_bounds__(256) gather_dates_kernel(const float *__restrict__ Y, int64_t N, int64_t ldY,
+                                                           int64_t P, const int32_t *__restrict__ idx,
+                                                           float *__restrict__ Yc, int64_t ldYc, int vec4) {
   const int64_t i = blockIdx.y;
-  const float *src = Y + (int64_t)idx[i] * ldY;
+  const int32_t t = idx[i];
   float *dst = Yc + i * ldYc;
   const int64_t step = (int64_t)gridDim.x * blockDim.x;
+  if (t < 0 || t >= N) {
+    for (int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < P; p += step)
+      dst[p] = __int_as_float(0x7fc00000);
+    return;
+  }
+  const float *src = Y + (int64_t)t * ldY;
   if (vec4) {
     const int64_t P4 = P / 4;
     const float4 *s4 = reinterpret_cast<const float4 *>(src);

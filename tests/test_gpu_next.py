@@ -262,6 +262,12 @@ def test_f2_edge_cases():
     Yc, dc, nc, kept = binding.drop_empty_dates(Yn, dates, spec.n_hist)
     assert Yc.shape == (0, spec.P) and nc == 0 and len(kept) == 0
     assert binding.bfast_valid_dates(Y, P=0).cpu().numpy().sum() == 0
+    bad = torch.tensor([3, 64, -1, 5], dtype=torch.int32, device=DEV)  # indices outside [0, N) -> NaN rows
+    Yc = binding.bfast_gather_dates(Y, bad)
+    torch.cuda.synchronize()
+    assert torch.equal(Yc[0].view(torch.int32), Y[3].view(torch.int32))
+    assert torch.equal(Yc[3].view(torch.int32), Y[5].view(torch.int32))
+    assert torch.isnan(Yc[1]).all() and torch.isnan(Yc[2]).all()
 
 
 @pytest.mark.parametrize("k", [4, 5, 6])
