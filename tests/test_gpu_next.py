@@ -302,3 +302,30 @@ def test_f4_int16_long_history_sampled_ring():
     gpu = {key: v.cpu().numpy()[idx] for key, v in out.items() if torch.is_tensor(v)}
     rep = parity.compare(gpu, orc, dates, 350, 3)
     assert rep["ok"], json.dumps(rep)
+
+
+def test_f1_sampled_ring_refits_wider_windows():
+    """The multi-period launch sizes its ring from a sample of the longest
+    history; complete histories placed outside the sampled 32-pixel groups
+    have wider windows in every period and are refitted in fp64 -- all of
+    them and a sample of the rest match the oracle, period by period."""
+    P = 1 << 18
+    spec = synth.StackSpec(P=P, N=400, n_hist=230, miss=0.6, mask="iid", seed=1901)
+    Y, dates = synth.generate(spec, DEV)
+    Y0, _ = synth.generate(synth.StackSpec(**{**spec.asdict(), "mask": "none"}), DEV)
+    gstride = P // 2048
+    wide = np.arange(gstride // 2, P, gstride)  # never in a sampled group (the first 32 of each stride)
+    it = torch.from_numpy(wide).to(DEV)
+    Y[:391, it] = Y0[:391, it]
+    per = _yearly(230, 7)
+    out = binding.bfast_monitor_periods(Y, dates, per, 3, spec.hf, spec.lam, diagnostics=True)
+    torch.cuda.synchronize()
+    rng = np.random.default_rng(8)
+    idx = np.unique(np.concatenate([wide, rng.choice(P, 4000, replace=False)]))
+    Ys = np.ascontiguousarray(Y[:, torch.from_numpy(idx).to(DEV)].cpu().numpy())
+    orcs = oracle.monitor_periods(Ys, dates, per, 3, spec.hf, spec.lam)
+    for i, ((n_i, N_i), orc) in enumerate(zip(per, orcs)):
+        gpu = {key: v[i].cpu().numpy()[idx] for key, v in out.items() if torch.is_tensor(v)}
+        assert np.all(out["flags"][i].cpu().numpy()[wide] & 2), i
+        rep = parity.compare(gpu, orc, dates[:N_i], n_i, 3)
+        assert rep["ok"], (i, json.dumps(rep))
