@@ -276,10 +276,12 @@ __device__ __forceinline__ void tmem_ld1(uint32_t taddr, float (&v)[1]) {
   v[0] = __uint_as_float(r);
 }
 // consumer-side waits: BFAST_FZ_CWAIT 0 = probe in a loop (try_wait's own
-// time limit), 1 = try_wait with a suspend-time hint (the warp sleeps in
-// hardware and leaves its issue slots to the other warps)
+// time limit), 1 = try_wait with a suspend-time hint (compiles to TRYWAIT +
+// NANOSLEEP.SYNCS + PHASECHK per iteration).  0 measured -0.7% on the
+// Landsat scene, -1.4% at N = 1000, +-0 at N = 100 (round 2); the control
+// warps keep the suspend hint (0 there: +0.2%)
 #ifndef BFAST_FZ_CWAIT
-#define BFAST_FZ_CWAIT 1
+#define BFAST_FZ_CWAIT 0
 #endif
 __device__ __forceinline__ void mbar_wait_spin(uint32_t bar, uint32_t parity) {
 #if BFAST_FZ_CWAIT == 1
