@@ -497,7 +497,9 @@ int launch_fused(const bfast_plan &pl, const bfast::MonitorParams &prm, cudaStre
       !make_stack_map(&hmap, Ybase, prm.ldY, prm.P, pl.n, 128 * C::TPC, 16, I16) ||
       !make_stack_map(&pmap, Ybase, prm.ldY, prm.P, pl.N, 128 * C::TPC, C::PFB, I16))
     return BFAST_OK;
-  int pfd = 128;
+  // L2 prefetch of first-touch dates ahead of the TMA loads: off (measured
+  // -1..-5% without it across the configs in round 2; BFAST_FZ_PFD=128 re-enables)
+  int pfd = 0;
   if (const char *e = std::getenv("BFAST_FZ_PFD")) pfd = std::max(0, std::atoi(e)) / C::PFB * C::PFB;
   bfast::FzTables tb{};
   tb.tabA = pl.dtabf;
