@@ -903,7 +903,10 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
         wait_sleep(a_pub + 8 * (g & 3), (g >> 2) & 1u);
         FZT_ADD(5, tp)
         FZT_T0(ti)
-        sm100::tc_fence_after();
+        // (no fence::after_thread_sync here: every MMA below follows a table
+        // wait and its own fence, which orders it after this publish wait as
+        // well; a bare commit reads no TMEM -- measured with the atom.inc
+        // below: -0.6%)
         // group g commits to the barrier of group g - 4 without observing
         // that phase: one thread (this warp's elected lane) issues every
         // commit of the tile, whose arrivals come in issue order as the
@@ -969,10 +972,13 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
             FZT_ADD(13, tm)
             const ChunkPos nxt = advance_pos(cpos, C::ST - 2);
             if (lane == 0) {
-              const uint32_t old = atom_add_acqrel(a_tfree + 4 * nxt.st, 1u);
-              const int NGc = T / TPC;  // control groups sharing the table ring
-              const bool last = NGc == 4 ? (old & 3u) == 3u : NGc == 2 ? (old & 1u) == 1u : NGc == 1 ? true
-                                                                                                   : old % 3u == 2u;
+              // counts 0 .. NGc - 1 and wraps: the last group sees NGc - 1
+              uint32_t old;
+              asm volatile("atom.acq_rel.cta.shared::cta.inc.u32 %0, [%1], %2;"
+                           : "=r"(old)
+                           : "r"(a_tfree + 4 * nxt.st), "r"((uint32_t)(T / TPC - 1))
+                           : "memory");
+              const bool last = old == (uint32_t)(T / TPC - 1);
               if (last) load_table(nxt);
             }
             __syncwarp();
