@@ -1215,26 +1215,22 @@ __global__ void __launch_bounds__(128 * (FzTiles<K, MULTI>::TM + 1), 1)
 #pragma unroll
       for (int i = 0; i < K; ++i) diagA[i] = A[Tri<K>::idx(i, i)];
       if constexpr (DENSE) {
-        // f3 (L93): a warp whose 32 histories have no missing value shares
-        // one Gram, factored once on the host in fp64: beta0 = A^-1 (X_hist^T
-        // y'), the moment b being the tensor-core GEMM of pass A.  A separate
-        // instantiation (BFAST_SHARED_FACTOR=1): the warp test in the common
-        // kernel cost +0.3% on the Landsat scene and +5% at N = 100
-        const bool dense = shared_factor != nullptr && __all_sync(0xffffffffu, nbar == n);
-        float minratio, vif = 0.f;
-        if (dense) {
+        // f3 (L93, the [27] special case), for a scene declared to have
+        // complete histories (BFAST_SHARED_FACTOR=1): every pixel shares one
+        // Gram, factored once on the host in fp64 -- beta0 = A^-1 (X_hist^T
+        // y'), the moment b being pass A's tensor-core GEMM -- and no pixel
+        // factors its own.  A pixel whose history does have a gap (nbar < n)
+        // is recomputed by the fp64 refit, so the result stays exact for any
+        // input; the kernel carries no Cholesky code (a per-warp choice
+        // between the two spilled and measured +2.7%)
 #pragma unroll
-          for (int i = 0; i < Tri<K>::kN; ++i) A[i] = __ldg(shared_factor + i);
+        for (int i = 0; i < Tri<K>::kN; ++i) A[i] = __ldg(shared_factor + i);
 #pragma unroll
-          for (int i = 0; i < K; ++i) dinv[i] = __ldg(shared_factor + Tri<K>::kN + i);
-          minratio = __ldg(shared_factor + Tri<K>::kN + K);
-          vif = __ldg(shared_factor + Tri<K>::kN + K + 1);
-        } else {
-          minratio = fz_chol<K>(A, dinv);
-        }
+        for (int i = 0; i < K; ++i) dinv[i] = __ldg(shared_factor + Tri<K>::kN + i);
         fz_solve<K>(A, dinv, b, beta);
-        if (!deg && !(minratio >= (float)kRefitRatio)) refit = true;
-        if (!deg && !refit && !((dense ? vif : fz_vif_max<K>(A, dinv, diagA)) <= kRefitVif)) refit = true;
+        if (!deg && nbar != n) refit = true;
+        if (!deg && !(__ldg(shared_factor + Tri<K>::kN + K) >= (float)kRefitRatio)) refit = true;
+        if (!deg && !(__ldg(shared_factor + Tri<K>::kN + K + 1) <= kRefitVif)) refit = true;
       } else {
         const float minratio = fz_chol<K>(A, dinv);
         fz_solve<K>(A, dinv, b, beta);
